@@ -1,0 +1,68 @@
+"""Coordinated checkpoint across the ranks of one box (global snapshot).
+
+PAPER.md L40 §IV-C: "The checkpoint files of individual computing nodes, called
+local snapshots, are aggregated into a global snapshot [14]" (Open MPI's CPR). Here
+each rank snapshots its own GPU's buffers independently (no data crosses ranks);
+the only exchange is a 40-byte status all-reduce over the process group (NCCL over
+NVLink on GPUs, gloo in CPU tests): SUM of [failures, buffers, bytes] and MAX of
+[epoch, -epoch]. The global snapshot commits iff no rank failed and every rank
+checkpointed the same epoch (reading 16: a two-phase commit); otherwise
+every rank frees its local image.
+"""
+from __future__ import annotations
+
+from dataclasses import dataclass
+from typing import Callable, Optional, Tuple
+
+
+@dataclass
+class GlobalSnapshot:
+    committed: bool
+    image: object  # the local Image, or None when aborted
+    failures: int
+    n_buffers: int
+    total_bytes: int
+    epoch: int
+    epochs_agree: bool
+
+
+def agree(failed: bool, n_buffers: int, nbytes: int, epoch: int, group=None, device=None) -> Tuple[int, int, int, bool, int]:
+    """The coordination all-reduce. Returns (failures, buffers, bytes, epochs_agree, epoch)."""
+    import torch
+    import torch.distributed as dist
+
+    dev = torch.device("cuda", device) if (device is not None and dist.get_backend(group) == "nccl") else torch.device("cpu")
+    s = torch.tensor([1 if failed else 0, n_buffers, nbytes], dtype=torch.int64, device=dev)
+    e = torch.tensor([epoch, -epoch], dtype=torch.int64, device=dev)
+    dist.all_reduce(s, op=dist.ReduceOp.SUM, group=group)
+    dist.all_reduce(e, op=dist.ReduceOp.MAX, group=group)
+    s, e = s.cpu().tolist(), e.cpu().tolist()
+    return int(s[0]), int(s[1]), int(s[2]), e[0] == -e[1], int(e[0])
+
+
+def coordinated(take_local: Callable[[], Tuple[object, int, int]], epoch: int, group=None,
+                device: Optional[int] = None) -> GlobalSnapshot:
+    """Runs `take_local()` -> (image, n_buffers, bytes) on every rank, then the
+    status all-reduce; frees the local image if the global snapshot aborts."""
+    img, n, b, failed = None, 0, 0, False
+    try:
+        img, n, b = take_local()
+    except Exception:
+        failed = True
+    f, tn, tb, same, ep = agree(failed, n, b, epoch, group, device)
+    ok = f == 0 and same
+    if not ok and img is not None:
+        img.free()
+        img = None
+    return GlobalSnapshot(ok, img, f, tn, tb, ep, same)
+
+
+def coordinated_checkpoint(ctx, device: int, epoch: int, group=None, stream=None, into=None,
+                           on_device: bool = False) -> GlobalSnapshot:
+    """Local checl_checkpoint (host image, or HBM image with on_device) + commit barrier."""
+    def local():
+        n, b = ctx.count(device)
+        if on_device:
+            return ctx.checkpoint_device(device, stream, epoch), n, b
+        return ctx.checkpoint(device, stream, epoch, into=into), n, b
+    return coordinated(local, epoch, group, device)

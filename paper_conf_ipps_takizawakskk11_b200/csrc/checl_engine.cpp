@@ -1,0 +1,1342 @@
+// checl_engine.cpp — libchecl host engine and C ABI (include/checl.h).
+//
+// Object database + handle table (§III-B, L19 §III-C), checkpoint
+// (L16 §III-C steps 1, 2, 4), restart (L16 restart steps 2-3, restore order
+// L19-L20 reduced to device -> buffers -> rebind), migration (L40 §IV-C), over the
+// image layout of FORMAT.md. The data path runs in checl_kernels.cu; this file
+// plans it (flat chunk list, stages), drives the staging pipeline on two streams
+// (copy engine D2H/H2D overlapped with the pack / verify kernels), and commits.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <atomic>
+#include <chrono>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <map>
+#include <memory>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/checl.h"
+#include "checl_internal.h"
+
+namespace checl {
+size_t snapshot_smem_bytes();
+cudaError_t snapshot_configure();
+cudaError_t launch_snapshot(bool verify, const LaunchParams& p, int n_sms, cudaStream_t s);
+cudaError_t launch_fill(uint8_t* ptr, uint64_t bytes, uint64_t key, int kind, int n_sms, cudaStream_t s);
+cudaError_t launch_compare(const uint8_t* a, const uint8_t* b, uint64_t bytes, unsigned long long* n_diff, int n_sms,
+                           cudaStream_t s);
+uint32_t host_crc32c_update(uint32_t crc, const void* data, size_t n);
+uint32_t host_crc32c(const void* data, size_t n);
+}  // namespace checl
+
+using namespace checl;
+
+namespace {
+
+constexpr int kMaxDevices = 64;
+constexpr uint32_t kMaxSlots = 8;
+constexpr size_t kSlotSlack = 256;  // pack writes whole 16-B granules past a last buffer's end
+constexpr size_t kDefaultSlotBytes = 64ull << 20;
+
+thread_local std::string t_last_cuda_error;
+
+double now_ms() {
+  return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
+}
+
+uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+uint64_t chunks_of(uint64_t size) { return (size + kChunkBytes - 1) / kChunkBytes; }
+
+void put_u32(uint8_t* p, uint32_t v) { std::memcpy(p, &v, 4); }
+void put_u64(uint8_t* p, uint64_t v) { std::memcpy(p, &v, 8); }
+uint32_t get_u32(const uint8_t* p) {
+  uint32_t v;
+  std::memcpy(&v, p, 4);
+  return v;
+}
+uint64_t get_u64(const uint8_t* p) {
+  uint64_t v;
+  std::memcpy(&v, p, 8);
+  return v;
+}
+
+struct CudaFail {
+  cudaError_t e;
+};
+
+// Throws on a CUDA error; the C ABI converts it into CHECL_ERR_CUDA.
+void ck(cudaError_t e) {
+  if (e != cudaSuccess) {
+    t_last_cuda_error = cudaGetErrorName(e);
+    cudaGetLastError();
+    throw CudaFail{e};
+  }
+}
+
+int fake_devices() {
+  static const int n = [] {
+    const char* s = std::getenv("CHECL_FAKE_DEVICES");
+    return s ? std::atoi(s) : 0;
+  }();
+  return n;
+}
+
+int device_count() {
+  static const int n = [] {
+    int c = 0;
+    if (cudaGetDeviceCount(&c) != cudaSuccess) {
+      cudaGetLastError();
+      c = 0;
+    }
+    return c;
+  }();
+  return n > 0 ? n : fake_devices();
+}
+
+bool valid_device(int d) { return d >= 0 && d < device_count() && d < kMaxDevices; }
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int d) {
+    ck(cudaGetDevice(&prev));
+    if (prev != d) ck(cudaSetDevice(d));
+  }
+  ~DeviceGuard() {
+    if (prev >= 0) cudaSetDevice(prev);
+  }
+};
+
+// x^(-8z) mod P for z in [0, 65536): the short-chunk correction of the kernels.
+const std::vector<uint32_t>& inv_z_table() {
+  static const std::vector<uint32_t> t = [] {
+    std::vector<uint32_t> v(kChunkBytes);
+    uint32_t r = kOne;
+    for (uint32_t z = 0; z < kChunkBytes; ++z) {
+      v[z] = r;
+      for (int b = 0; b < 8; ++b) r = gf_divx(r);
+    }
+    return v;
+  }();
+  return t;
+}
+
+void fill_fold(uint32_t fold[kFoldLevels]) {
+  for (int k = 0; k < kFoldLevels; ++k) fold[k] = gf_x_pow2k(14 + k);  // x^(8*2048*2^k)
+}
+
+// ---- per-device resources ---------------------------------------------------
+
+struct EventPool {
+  std::vector<cudaEvent_t> ev;
+  size_t used = 0;
+  cudaEvent_t get() {
+    if (used == ev.size()) {
+      cudaEvent_t e;
+      ck(cudaEventCreate(&e));
+      ev.push_back(e);
+    }
+    return ev[used++];
+  }
+  void reset() { used = 0; }
+  ~EventPool() {
+    for (auto e : ev) cudaEventDestroy(e);
+  }
+};
+
+template <typename T>
+struct DevBuf {  // grow-only device scratch (cudaMalloc)
+  T* p = nullptr;
+  size_t cap = 0;
+  void ensure(size_t n) {
+    if (n <= cap) return;
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+    ck(cudaMalloc(&p, std::max<size_t>(n, 1) * sizeof(T)));
+    cap = n;
+  }
+  void release() {
+    if (p) cudaFree(p);
+    p = nullptr;
+    cap = 0;
+  }
+};
+
+template <typename T>
+struct PinnedBuf {  // grow-only pinned host scratch
+  T* p = nullptr;
+  size_t cap = 0;
+  void ensure(size_t n) {
+    if (n <= cap) return;
+    if (p) cudaFreeHost(p);
+    p = nullptr;
+    cap = 0;
+    ck(cudaHostAlloc(reinterpret_cast<void**>(&p), std::max<size_t>(n, 1) * sizeof(T), cudaHostAllocDefault));
+    cap = n;
+  }
+  void release() {
+    if (p) cudaFreeHost(p);
+    p = nullptr;
+    cap = 0;
+  }
+};
+
+struct Stage {
+  uint64_t c0, c1, img_lo, img_hi;
+};
+
+struct BufRec {
+  uint64_t handle, size, off, first_chunk;
+  uint32_t flags;
+  uint8_t* ptr;
+};
+
+// Everything a checkpoint of one device needs that depends only on the registry
+// (cached until the registry of that device changes).
+struct Plan {
+  uint64_t version = ~0ull;
+  size_t slot_bytes = 0;
+  std::vector<BufRec> bufs;
+  uint64_t n_chunks = 0, payload_bytes = 0, crc_off = 0, payload_off = 0, image_bytes = 0;
+  std::vector<ChunkDesc> desc;
+  std::vector<Stage> stages;
+  std::vector<uint8_t> meta;  // header (meta_crc = 0, epoch = 0) + manifest
+  DevBuf<ChunkDesc> d_desc;
+};
+
+struct DevState {
+  int dev = -1, n_sms = 0;
+  cudaStream_t compute = nullptr, copy = nullptr;
+  DevBuf<uint8_t> slots;
+  size_t slot_bytes = 0;
+  uint32_t n_slots = 0;
+  DevBuf<uint32_t> inv_z, crc_scratch;
+  DevBuf<ChunkDesc> desc_scratch;
+  DevBuf<unsigned long long> status;
+  PinnedBuf<unsigned long long> h_status;
+  PinnedBuf<ChunkDesc> h_desc;
+  EventPool events;
+  Plan plan;
+  uint32_t fold[kFoldLevels];
+
+  void init(int d) {
+    dev = d;
+    DeviceGuard g(d);
+    ck(cudaDeviceGetAttribute(&n_sms, cudaDevAttrMultiProcessorCount, d));
+    ck(cudaStreamCreateWithFlags(&compute, cudaStreamNonBlocking));
+    ck(cudaStreamCreateWithFlags(&copy, cudaStreamNonBlocking));
+    ck(snapshot_configure());
+    inv_z.ensure(kChunkBytes);
+    ck(cudaMemcpy(inv_z.p, inv_z_table().data(), kChunkBytes * 4, cudaMemcpyHostToDevice));
+    status.ensure(2);
+    h_status.ensure(2);
+    fill_fold(fold);
+  }
+  void ensure_slots(size_t bytes, uint32_t n) {
+    if (slot_bytes == bytes && n_slots == n && slots.p) return;
+    slots.release();
+    slots.ensure(n * (bytes + kSlotSlack));
+    slot_bytes = bytes;
+    n_slots = n;
+  }
+  uint8_t* slot(uint32_t i) { return slots.p + (size_t)i * (slot_bytes + kSlotSlack); }
+  void destroy() {
+    if (dev < 0) return;
+    int prev = -1;
+    cudaGetDevice(&prev);
+    cudaSetDevice(dev);
+    cudaDeviceSynchronize();
+    slots.release();
+    inv_z.release();
+    crc_scratch.release();
+    desc_scratch.release();
+    status.release();
+    plan.d_desc.release();
+    h_status.release();
+    h_desc.release();
+    for (auto e : events.ev) cudaEventDestroy(e);
+    events.ev.clear();
+    if (compute) cudaStreamDestroy(compute);
+    if (copy) cudaStreamDestroy(copy);
+    if (prev >= 0) cudaSetDevice(prev);
+    dev = -1;
+  }
+};
+
+// ---- library-owned memory (buffers re-created by restore / migrate) ----------
+
+struct Arena {  // one allocation holding every buffer of one restore (payload layout)
+  checl_allocator alloc;
+  int device;
+  void* stream;
+  void* base = nullptr;
+  ~Arena() {
+    if (!base) return;
+    if (alloc.free)
+      alloc.free(base, device, stream, alloc.user);
+    else {
+      int prev = -1;
+      cudaGetDevice(&prev);
+      cudaSetDevice(device);
+      cudaFree(base);
+      if (prev >= 0) cudaSetDevice(prev);
+    }
+  }
+};
+
+struct Entry {
+  int device;
+  uint8_t* ptr;
+  uint64_t bytes;
+  uint32_t flags;
+  bool owned;
+  std::shared_ptr<Arena> arena;  // owned buffers keep their arena alive
+};
+
+// Phase-time events for checl_timing.
+struct KernelTimer {
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> spans;
+  double sum_ms() const {
+    double t = 0;
+    for (auto& s : spans) {
+      float ms = 0;
+      if (cudaEventElapsedTime(&ms, s.first, s.second) == cudaSuccess) t += ms;
+    }
+    return t;
+  }
+};
+
+}  // namespace
+
+// ---- opaque types -------------------------------------------------------------
+
+struct checl_image {
+  int location = CHECL_IMAGE_HOST;
+  int device = -1;  // device image: where payload and CRC table live
+  bool owned = true;
+  bool pinned = false;
+  const uint8_t* host = nullptr;  // host: full image; device: mirror of [0, payload_off)
+  uint8_t* host_mut = nullptr;    // same pointer when library-owned
+  size_t host_cap = 0;
+  uint64_t image_bytes = 0, payload_off = 0;
+  uint8_t* d_payload = nullptr;
+  size_t d_payload_cap = 0;
+  uint32_t* d_crc = nullptr;
+  size_t d_crc_cap = 0;
+
+  void free_device() {
+    if (device >= 0 && (d_payload || d_crc)) {
+      int prev = -1;
+      cudaGetDevice(&prev);
+      cudaSetDevice(device);
+      if (d_payload) cudaFree(d_payload);
+      if (d_crc) cudaFree(d_crc);
+      if (prev >= 0) cudaSetDevice(prev);
+    }
+    d_payload = nullptr;
+    d_crc = nullptr;
+    d_payload_cap = d_crc_cap = 0;
+  }
+  void free_host() {
+    if (owned && host_mut) {
+      if (pinned)
+        cudaFreeHost(host_mut);
+      else
+        std::free(host_mut);
+    }
+    host = host_mut = nullptr;
+    host_cap = 0;
+  }
+  void ensure_host(size_t n, bool want_pinned) {
+    if (owned && host_mut && host_cap >= n && pinned == want_pinned) return;
+    free_host();
+    owned = true;
+    void* p = nullptr;
+    if (want_pinned) {
+      ck(cudaHostAlloc(&p, std::max<size_t>(n, 1), cudaHostAllocDefault));
+    } else {
+      p = std::malloc(std::max<size_t>(n, 1));
+      if (!p) throw std::bad_alloc();
+    }
+    host = host_mut = static_cast<uint8_t*>(p);
+    host_cap = n;
+    pinned = want_pinned;
+  }
+};
+
+struct checl_ctx {
+  mutable std::mutex mu;
+  checl_allocator alloc{nullptr, nullptr, nullptr};
+  std::map<uint64_t, Entry> entries;                  // ascending handle = database order (L19)
+  std::map<uintptr_t, uint64_t> by_addr[kMaxDevices];  // start address -> handle (overlap checks)
+  uint64_t version[kMaxDevices] = {};
+  uint64_t next_id = 1;
+  std::atomic<bool> busy{false};
+  DevState* devs[kMaxDevices] = {};
+  size_t slot_bytes = kDefaultSlotBytes;
+  uint32_t n_slots = 2;
+  checl_timing last{};
+
+  DevState& dev(int d) {
+    if (!devs[d]) {
+      auto* s = new DevState();
+      try {
+        s->init(d);
+      } catch (...) {
+        s->destroy();
+        delete s;
+        throw;
+      }
+      devs[d] = s;
+    }
+    return *devs[d];
+  }
+};
+
+namespace {
+
+struct BusyGuard {
+  checl_ctx* ctx;
+  bool ok;
+  explicit BusyGuard(checl_ctx* c) : ctx(c) {
+    bool expected = false;
+    ok = ctx->busy.compare_exchange_strong(expected, true);
+  }
+  ~BusyGuard() {
+    if (ok) ctx->busy.store(false);
+  }
+};
+
+template <typename F>
+checl_status guarded(F&& f) {
+  try {
+    return f();
+  } catch (const CudaFail&) {
+    return CHECL_ERR_CUDA;
+  } catch (const std::bad_alloc&) {
+    return CHECL_ERR_OUT_OF_HOST_MEMORY;
+  } catch (...) {
+    return CHECL_ERR_INVALID_VALUE;
+  }
+}
+
+// -- layout (FORMAT.md), independent of the oracle ------------------------------
+
+struct Layout {
+  uint64_t n_chunks = 0, payload_bytes = 0, crc_off = 0, payload_off = 0, image_bytes = 0;
+};
+
+// Fills off / first_chunk of each record (ascending handle) and the region offsets.
+Layout layout_records(std::vector<BufRec>& bufs) {
+  Layout L;
+  uint64_t end = 0;
+  for (size_t b = 0; b < bufs.size(); ++b) {
+    bufs[b].off = b == 0 ? 0 : align_up(end, kBufferAlign);
+    bufs[b].first_chunk = L.n_chunks;
+    end = bufs[b].off + bufs[b].size;
+    L.n_chunks += chunks_of(bufs[b].size);
+  }
+  L.payload_bytes = bufs.empty() ? 0 : end;
+  L.crc_off = kHeaderBytes + (uint64_t)kRecordBytes * bufs.size();
+  L.payload_off = align_up(L.crc_off + 4 * L.n_chunks, kPayloadAlign);
+  L.image_bytes = L.payload_off + L.payload_bytes;
+  return L;
+}
+
+// Flat chunk list; ptr(b) is the device address chunk k of record b is read from
+// (pack) or written to (restore).
+template <typename PtrOf>
+void build_desc(const std::vector<BufRec>& bufs, uint64_t payload_bytes, PtrOf ptr_of, ChunkDesc* out) {
+  size_t c = 0;
+  for (size_t b = 0; b < bufs.size(); ++b) {
+    const uint64_t nch = chunks_of(bufs[b].size);
+    const uint64_t pad_end = b + 1 < bufs.size() ? bufs[b + 1].off : payload_bytes;
+    uint8_t* base = ptr_of(b);
+    for (uint64_t k = 0; k < nch; ++k) {
+      const uint64_t lo = k * kChunkBytes;
+      const uint32_t len = (uint32_t)std::min<uint64_t>(kChunkBytes, bufs[b].size - lo);
+      const uint32_t pad = k + 1 == nch ? (uint32_t)(pad_end - (bufs[b].off + bufs[b].size)) : 0u;
+      ChunkDesc d;
+      d.ptr = reinterpret_cast<uint64_t>(base + lo);
+      d.img_off_256 = (uint32_t)((bufs[b].off + lo) / kBufferAlign);
+      d.len_pad = make_len_pad(len, pad);
+      out[c++] = d;
+    }
+  }
+}
+
+// Consecutive chunks whose image span fits in one staging slot.
+std::vector<Stage> build_stages(const ChunkDesc* desc, uint64_t n, size_t slot_bytes) {
+  std::vector<Stage> st;
+  uint64_t c = 0;
+  while (c < n) {
+    Stage s;
+    s.c0 = c;
+    s.img_lo = (uint64_t)desc[c].img_off_256 * kBufferAlign;
+    s.img_hi = s.img_lo;
+    while (c < n) {
+      const uint64_t hi = (uint64_t)desc[c].img_off_256 * kBufferAlign + desc_len(desc[c]) + desc_pad(desc[c]);
+      if (c > s.c0 && hi - s.img_lo > slot_bytes) break;
+      s.img_hi = hi;
+      ++c;
+    }
+    s.c1 = c;
+    st.push_back(s);
+  }
+  return st;
+}
+
+void write_header(uint8_t* h, const Layout& L, uint64_t n_buffers, int device, uint64_t epoch) {
+  std::memset(h, 0, kHeaderBytes);
+  std::memcpy(h, "CHECLIM1", 8);
+  put_u32(h + 8, 1);
+  put_u32(h + 12, kHeaderBytes);
+  put_u32(h + 16, kChunkBytes);
+  put_u32(h + 20, kBufferAlign);
+  put_u64(h + 24, n_buffers);
+  put_u64(h + 32, L.n_chunks);
+  put_u64(h + 40, kHeaderBytes);
+  put_u64(h + 48, L.crc_off);
+  put_u64(h + 56, L.payload_off);
+  put_u64(h + 64, L.payload_bytes);
+  put_u64(h + 72, L.image_bytes);
+  put_u32(h + 80, (uint32_t)device);
+  put_u32(h + 84, 0);
+  put_u64(h + 88, epoch);
+}
+
+void write_manifest(uint8_t* m, const std::vector<BufRec>& bufs, int device) {
+  for (size_t b = 0; b < bufs.size(); ++b) {
+    uint8_t* r = m + (size_t)kRecordBytes * b;
+    put_u64(r, bufs[b].handle);
+    put_u64(r + 8, bufs[b].size);
+    put_u64(r + 16, bufs[b].off);
+    put_u64(r + 24, bufs[b].first_chunk);
+    put_u32(r + 32, bufs[b].flags);
+    put_u32(r + 36, (uint32_t)device);
+    put_u64(r + 40, 0);
+  }
+}
+
+uint32_t meta_crc(const uint8_t* img, uint64_t payload_off) {
+  uint32_t c = host_crc32c_update(0xFFFFFFFFu, img, 124);
+  c = host_crc32c_update(c, img + kHeaderBytes, payload_off - kHeaderBytes);
+  return ~c;
+}
+
+// -- validation (FORMAT.md "Validation order" step 1) -----------------------------
+
+bool add_ok(uint64_t a, uint64_t b, uint64_t* out) {
+  if (a > ~0ull - b) return false;
+  *out = a + b;
+  return true;
+}
+
+struct Parsed {
+  int source_device = 0;
+  Layout L;
+  std::vector<BufRec> bufs;
+};
+
+checl_status parse_image(const uint8_t* img, size_t len, bool meta_only, Parsed* out) {
+  // meta_only: `len` covers [0, payload_off) only (device image mirror)
+  if (!img || len < kHeaderBytes) return CHECL_ERR_BAD_IMAGE;
+  if (std::memcmp(img, "CHECLIM1", 8) != 0) return CHECL_ERR_BAD_IMAGE;
+  if (get_u32(img + 8) != 1 || get_u32(img + 12) != kHeaderBytes || get_u32(img + 16) != kChunkBytes ||
+      get_u32(img + 20) != kBufferAlign || get_u64(img + 40) != kHeaderBytes || get_u32(img + 84) != 0)
+    return CHECL_ERR_BAD_IMAGE;
+  for (int i = 96; i < 124; ++i)
+    if (img[i]) return CHECL_ERR_BAD_IMAGE;
+  const uint64_t n = get_u64(img + 24), nch = get_u64(img + 32);
+  Layout L;
+  L.n_chunks = nch;
+  L.crc_off = get_u64(img + 48);
+  L.payload_off = get_u64(img + 56);
+  L.payload_bytes = get_u64(img + 64);
+  L.image_bytes = get_u64(img + 72);
+  if (n > (~0ull - kHeaderBytes) / kRecordBytes || L.crc_off != kHeaderBytes + kRecordBytes * n)
+    return CHECL_ERR_BAD_IMAGE;
+  if (nch > (~0ull - L.crc_off - kPayloadAlign) / 4) return CHECL_ERR_BAD_IMAGE;
+  if (L.payload_off != align_up(L.crc_off + 4 * nch, kPayloadAlign)) return CHECL_ERR_BAD_IMAGE;
+  uint64_t want;
+  if (!add_ok(L.payload_off, L.payload_bytes, &want) || want != L.image_bytes) return CHECL_ERR_BAD_IMAGE;
+  if ((uint64_t)len < (meta_only ? L.payload_off : L.image_bytes)) return CHECL_ERR_BAD_IMAGE;
+  if (get_u32(img + 124) != meta_crc(img, L.payload_off)) return CHECL_ERR_BAD_IMAGE;
+  for (uint64_t i = L.crc_off + 4 * nch; i < L.payload_off; ++i)
+    if (img[i]) return CHECL_ERR_BAD_IMAGE;
+  const int device = (int32_t)get_u32(img + 80);
+  std::vector<BufRec> bufs(n);
+  uint64_t off = 0, end = 0, chunk = 0, prev = 0;
+  for (uint64_t b = 0; b < n; ++b) {
+    const uint8_t* r = img + kHeaderBytes + kRecordBytes * b;
+    const uint64_t h = get_u64(r), size = get_u64(r + 8);
+    if (h == 0 || (b > 0 && h <= prev)) return CHECL_ERR_BAD_IMAGE;
+    if (b > 0) {
+      if (!add_ok(end, kBufferAlign - 1, &off)) return CHECL_ERR_BAD_IMAGE;
+      off = off / kBufferAlign * kBufferAlign;
+    }
+    if (get_u64(r + 16) != off || get_u64(r + 24) != chunk) return CHECL_ERR_BAD_IMAGE;
+    if ((int32_t)get_u32(r + 36) != device || get_u64(r + 40) != 0) return CHECL_ERR_BAD_IMAGE;
+    if (!add_ok(off, size, &end)) return CHECL_ERR_BAD_IMAGE;
+    chunk += chunks_of(size);
+    bufs[b] = BufRec{h, size, off, get_u64(r + 24), get_u32(r + 32), nullptr};
+    prev = h;
+  }
+  if (chunk != nch || L.payload_bytes != (n ? end : 0)) return CHECL_ERR_BAD_IMAGE;
+  // the kernels address chunk offsets as u32 multiples of 256 (1 TiB payload)
+  if (L.payload_bytes > (1ull << 40)) return CHECL_ERR_BAD_IMAGE;
+  out->source_device = device;
+  out->L = L;
+  out->bufs = std::move(bufs);
+  return CHECL_SUCCESS;
+}
+
+// -- checkpoint -------------------------------------------------------------------
+
+// Builds (or reuses) the plan of `device` under the context lock.
+Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
+  std::lock_guard<std::mutex> lk(ctx->mu);
+  Plan& P = ds.plan;
+  if (P.version == ctx->version[device] && P.slot_bytes == ctx->slot_bytes) return P;
+  P.bufs.clear();
+  for (auto& kv : ctx->entries)
+    if (kv.second.device == device)
+      P.bufs.push_back(BufRec{kv.first, kv.second.bytes, 0, 0, kv.second.flags, kv.second.ptr});
+  Layout L = layout_records(P.bufs);
+  if (L.payload_bytes > (1ull << 40)) throw std::bad_alloc();
+  P.n_chunks = L.n_chunks;
+  P.payload_bytes = L.payload_bytes;
+  P.crc_off = L.crc_off;
+  P.payload_off = L.payload_off;
+  P.image_bytes = L.image_bytes;
+  P.desc.resize(L.n_chunks);
+  build_desc(P.bufs, L.payload_bytes, [&](size_t b) { return P.bufs[b].ptr; }, P.desc.data());
+  P.stages = build_stages(P.desc.data(), L.n_chunks, ctx->slot_bytes);
+  P.meta.assign(L.crc_off, 0);
+  write_header(P.meta.data(), L, P.bufs.size(), device, 0);
+  write_manifest(P.meta.data() + kHeaderBytes, P.bufs, device);
+  P.d_desc.ensure(L.n_chunks);
+  if (L.n_chunks) ck(cudaMemcpy(P.d_desc.p, P.desc.data(), L.n_chunks * sizeof(ChunkDesc), cudaMemcpyHostToDevice));
+  P.version = ctx->version[device];
+  P.slot_bytes = ctx->slot_bytes;
+  return P;
+}
+
+LaunchParams base_params(DevState& ds) {
+  LaunchParams p{};
+  p.inv_z = ds.inv_z.p;
+  p.status = ds.status.p;
+  for (int k = 0; k < kFoldLevels; ++k) p.fold[k] = ds.fold[k];
+  return p;
+}
+
+void timed_launch(DevState& ds, KernelTimer& kt, bool verify, const LaunchParams& p, cudaStream_t s) {
+  cudaEvent_t a = ds.events.get(), b = ds.events.get();
+  ck(cudaEventRecord(a, s));
+  ck(launch_snapshot(verify, p, ds.n_sms, s));
+  ck(cudaEventRecord(b, s));
+  kt.spans.push_back({a, b});
+}
+
+// Writes header + manifest + meta_crc into the image's host bytes [0, payload_off);
+// the CRC table must already be there.
+void finalize_meta(uint8_t* host, const Plan& P, uint64_t epoch) {
+  std::memcpy(host, P.meta.data(), P.crc_off);
+  put_u64(host + 88, epoch);
+  std::memset(host + P.crc_off + 4 * P.n_chunks, 0, P.payload_off - P.crc_off - 4 * P.n_chunks);
+  put_u32(host + 124, meta_crc(host, P.payload_off));
+}
+
+checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t epoch, checl_image* img,
+                           bool to_device) {
+  (void)stream;
+  const double t0 = now_ms();
+  DeviceGuard g(device);
+  DevState& ds = ctx->dev(device);
+  ds.events.reset();
+  KernelTimer kt;
+  checl_timing tm{};
+
+  // a1: synchronise the host and every queue of the device (L16 step 1)
+  const double ts = now_ms();
+  ck(cudaDeviceSynchronize());
+  tm.sync_ms = now_ms() - ts;
+
+  // a2: database walk -> manifest + chunk list (L19), cached per registry version
+  const double tp = now_ms();
+  Plan& P = get_plan(ctx, ds, device);
+  LaunchParams lp = base_params(ds);
+  lp.desc = P.d_desc.p;
+  tm.plan_ms = now_ms() - tp;
+
+  cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
+  if (to_device) {
+    // device-resident image: payload and CRC table in HBM, meta mirrored on host
+    if (img->location != CHECL_IMAGE_DEVICE || img->device != device) {
+      img->free_device();
+      img->free_host();
+    }
+    img->location = CHECL_IMAGE_DEVICE;
+    img->device = device;
+    if (img->d_payload_cap < P.payload_bytes + kSlotSlack) {
+      if (img->d_payload) cudaFree(img->d_payload);
+      img->d_payload = nullptr;
+      img->d_payload_cap = 0;
+      ck(cudaMalloc(&img->d_payload, P.payload_bytes + kSlotSlack));
+      img->d_payload_cap = P.payload_bytes + kSlotSlack;
+    }
+    if (img->d_crc_cap < std::max<uint64_t>(P.n_chunks, 1)) {
+      if (img->d_crc) cudaFree(img->d_crc);
+      img->d_crc = nullptr;
+      img->d_crc_cap = 0;
+      ck(cudaMalloc(&img->d_crc, std::max<uint64_t>(P.n_chunks, 1) * 4));
+      img->d_crc_cap = std::max<uint64_t>(P.n_chunks, 1);
+    }
+    img->ensure_host(P.payload_off, true);
+    lp.c0 = 0;
+    lp.c1 = P.n_chunks;
+    lp.image = img->d_payload;
+    lp.image_base = 0;
+    lp.crc = img->d_crc;
+    if (P.n_chunks) timed_launch(ds, kt, false, lp, ds.compute);
+    ck(cudaEventRecord(c_begin, ds.compute));
+    if (P.n_chunks)
+      ck(cudaMemcpyAsync(img->host_mut + P.crc_off, img->d_crc, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.compute));
+    ck(cudaEventRecord(c_end, ds.compute));
+    tm.n_stages = 1;
+    ck(cudaStreamSynchronize(ds.compute));
+  } else {
+    // a3 + a4: pack stage s into slot s % n_slots on the compute stream while the
+    // copy engine drains the previous slot to the pinned image
+    if (img->location != CHECL_IMAGE_HOST) {
+      img->free_device();
+      img->free_host();
+      img->location = CHECL_IMAGE_HOST;
+      img->device = -1;
+    }
+    img->ensure_host(P.image_bytes, true);
+    ds.ensure_slots(ctx->slot_bytes, ctx->n_slots);
+    ds.crc_scratch.ensure(std::max<uint64_t>(P.n_chunks, 1));
+    lp.crc = ds.crc_scratch.p;
+    std::vector<cudaEvent_t> packed(ds.n_slots), drained(ds.n_slots);
+    for (uint32_t i = 0; i < ds.n_slots; ++i) {
+      packed[i] = ds.events.get();
+      drained[i] = ds.events.get();
+    }
+    ck(cudaEventRecord(c_begin, ds.copy));
+    for (size_t s = 0; s < P.stages.size(); ++s) {
+      const Stage& S = P.stages[s];
+      const uint32_t k = (uint32_t)(s % ds.n_slots);
+      if (s >= ds.n_slots) ck(cudaStreamWaitEvent(ds.compute, drained[k], 0));
+      lp.c0 = S.c0;
+      lp.c1 = S.c1;
+      lp.image = ds.slot(k);
+      lp.image_base = S.img_lo;
+      timed_launch(ds, kt, false, lp, ds.compute);
+      ck(cudaEventRecord(packed[k], ds.compute));
+      ck(cudaStreamWaitEvent(ds.copy, packed[k], 0));
+      ck(cudaMemcpyAsync(img->host_mut + P.payload_off + S.img_lo, ds.slot(k), S.img_hi - S.img_lo,
+                         cudaMemcpyDeviceToHost, ds.copy));
+      ck(cudaEventRecord(drained[k], ds.copy));
+    }
+    if (P.n_chunks)
+      ck(cudaMemcpyAsync(img->host_mut + P.crc_off, ds.crc_scratch.p, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.copy));
+    ck(cudaEventRecord(c_end, ds.copy));
+    tm.n_stages = P.stages.size();
+    ck(cudaStreamSynchronize(ds.copy));
+  }
+  // a5: header, manifest and meta CRC (the CRC table has landed)
+  finalize_meta(img->host_mut, P, epoch);
+  img->image_bytes = P.image_bytes;
+  img->payload_off = P.payload_off;
+  float cms = 0;
+  if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
+  tm.kernel_ms = kt.sum_ms();
+  tm.n_kernels = kt.spans.size();
+  tm.total_ms = now_ms() - t0;
+  ctx->last = tm;
+  return CHECL_SUCCESS;
+}
+
+// -- restore ----------------------------------------------------------------------
+
+void set_report(checl_report* rep, const Parsed& P, uint64_t n_bad, uint64_t first_bad) {
+  if (!rep) return;
+  rep->n_buffers = P.bufs.size();
+  rep->payload_bytes = P.L.payload_bytes;
+  rep->n_chunks = P.L.n_chunks;
+  rep->n_bad_chunks = n_bad;
+  rep->first_bad_chunk = n_bad ? first_bad : ~0ull;
+  rep->first_bad_handle = 0;
+  if (n_bad) {
+    for (auto& b : P.bufs)
+      if (first_bad >= b.first_chunk && first_bad < b.first_chunk + chunks_of(b.size)) rep->first_bad_handle = b.handle;
+  }
+}
+
+bool ensure_peer(int dev, int peer) {
+  if (dev == peer) return true;
+  int can = 0;
+  if (cudaDeviceCanAccessPeer(&can, dev, peer) != cudaSuccess || !can) {
+    cudaGetLastError();
+    return false;
+  }
+  cudaError_t e = cudaDeviceEnablePeerAccess(peer, 0);  // current device = dev
+  if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled) {
+    cudaGetLastError();
+    return false;
+  }
+  cudaGetLastError();
+  return true;
+}
+
+// Swaps every handle of the image to its new buffer (L15); frees library-owned
+// buffers previously bound to those handles (after their devices are idle).
+void commit(checl_ctx* ctx, const Parsed& P, int device, const std::shared_ptr<Arena>& arena) {
+  std::vector<std::shared_ptr<Arena>> dropped;
+  {
+    std::lock_guard<std::mutex> lk(ctx->mu);
+    uint64_t max_h = 0;
+    for (const BufRec& b : P.bufs) {
+      auto it = ctx->entries.find(b.handle);
+      if (it != ctx->entries.end()) {
+        Entry& old = it->second;
+        if (old.bytes) ctx->by_addr[old.device].erase(reinterpret_cast<uintptr_t>(old.ptr));
+        ctx->version[old.device]++;
+        if (old.arena) dropped.push_back(old.arena);
+        ctx->entries.erase(it);
+      }
+      Entry e;
+      e.device = device;
+      e.ptr = b.size ? static_cast<uint8_t*>(arena->base) + b.off : nullptr;
+      e.bytes = b.size;
+      e.flags = b.flags;
+      e.owned = true;
+      e.arena = b.size ? arena : nullptr;
+      if (b.size) ctx->by_addr[device][reinterpret_cast<uintptr_t>(e.ptr)] = b.handle;
+      ctx->entries.emplace(b.handle, std::move(e));
+      max_h = std::max(max_h, b.handle);
+    }
+    ctx->version[device]++;
+    ctx->next_id = std::max(ctx->next_id, max_h + 1);
+  }
+  // arenas whose last handle moved away are freed here, outside the lock, once
+  // their device is idle
+  for (auto& a : dropped) {
+    if (a.use_count() == 1) {
+      DeviceGuard g(a->device);
+      ck(cudaDeviceSynchronize());
+    }
+    a.reset();
+  }
+}
+
+checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void* stream, checl_report* rep,
+                        bool in_migrate) {
+  const double t0 = now_ms();
+  DeviceGuard g(device);
+  DevState& ds = ctx->dev(device);
+  ds.events.reset();
+  KernelTimer kt;
+  checl_timing tm{};
+  if (rep) std::memset(rep, 0, sizeof(*rep)), rep->first_bad_chunk = ~0ull;
+
+  // quiesce the target (its old buffers may be freed at commit)
+  const double ts = now_ms();
+  ck(cudaDeviceSynchronize());
+  tm.sync_ms = now_ms() - ts;
+
+  // r1: validate header + manifest (+ meta CRC over the CRC table)
+  const double tp = now_ms();
+  Parsed P;
+  const bool dev_img = img->location == CHECL_IMAGE_DEVICE;
+  checl_status st = parse_image(img->host, dev_img ? img->payload_off : img->image_bytes, dev_img, &P);
+  if (st) return st;
+  if (rep) set_report(rep, P, 0, 0);
+
+  // r2: re-create the buffers: one allocation laid out like the payload
+  auto arena = std::make_shared<Arena>();
+  arena->alloc = ctx->alloc;
+  arena->device = device;
+  arena->stream = stream;
+  if (P.L.payload_bytes) {
+    if (ctx->alloc.alloc)
+      arena->base = ctx->alloc.alloc(P.L.payload_bytes, device, stream, ctx->alloc.user);
+    else if (cudaMalloc(&arena->base, P.L.payload_bytes) != cudaSuccess) {
+      cudaGetLastError();
+      arena->base = nullptr;
+    }
+    if (!arena->base) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
+  }
+  const uint64_t nch = P.L.n_chunks;
+  ds.h_desc.ensure(std::max<uint64_t>(nch, 1));
+  uint8_t* abase = static_cast<uint8_t*>(arena->base);
+  build_desc(P.bufs, P.L.payload_bytes, [&](size_t b) { return abase + P.bufs[b].off; }, ds.h_desc.p);
+  ds.desc_scratch.ensure(std::max<uint64_t>(nch, 1));
+  LaunchParams lp = base_params(ds);
+  lp.desc = ds.desc_scratch.p;
+  tm.plan_ms = now_ms() - tp;
+
+  cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
+  ck(cudaEventRecord(c_begin, ds.copy));
+  if (nch) ck(cudaMemcpyAsync(ds.desc_scratch.p, ds.h_desc.p, nch * sizeof(ChunkDesc), cudaMemcpyHostToDevice, ds.copy));
+  ds.h_status.p[0] = ~0ull;
+  ds.h_status.p[1] = 0;
+  ck(cudaMemcpyAsync(ds.status.p, ds.h_status.p, 16, cudaMemcpyHostToDevice, ds.copy));
+  DevBuf<uint8_t> tmp_payload;  // only when the source device is not peer-reachable
+  DevBuf<uint32_t> tmp_crc;
+  if (dev_img) {
+    // device image (same GPU, or a peer GPU read over NVLink by the kernel)
+    const uint8_t* src = img->d_payload;
+    const uint32_t* crc = img->d_crc;
+    if (!ensure_peer(device, img->device)) {
+      tmp_payload.ensure(P.L.payload_bytes + kSlotSlack);
+      tmp_crc.ensure(std::max<uint64_t>(nch, 1));
+      if (P.L.payload_bytes)
+        ck(cudaMemcpyPeerAsync(tmp_payload.p, device, img->d_payload, img->device, P.L.payload_bytes, ds.copy));
+      if (nch) ck(cudaMemcpyPeerAsync(tmp_crc.p, device, img->d_crc, img->device, 4 * nch, ds.copy));
+      src = tmp_payload.p;
+      crc = tmp_crc.p;
+    }
+    ck(cudaEventRecord(c_end, ds.copy));
+    ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
+    lp.c0 = 0;
+    lp.c1 = nch;
+    lp.image = const_cast<uint8_t*>(src);
+    lp.image_base = 0;
+    lp.crc = const_cast<uint32_t*>(crc);
+    if (nch) timed_launch(ds, kt, true, lp, ds.compute);
+    tm.n_stages = 1;
+  } else {
+    // r3 + r4: fill slot s % n_slots over PCIe while the previous slot is verified
+    ds.ensure_slots(ctx->slot_bytes, ctx->n_slots);
+    ds.crc_scratch.ensure(std::max<uint64_t>(nch, 1));
+    if (nch) ck(cudaMemcpyAsync(ds.crc_scratch.p, img->host + P.L.crc_off, 4 * nch, cudaMemcpyHostToDevice, ds.copy));
+    lp.crc = ds.crc_scratch.p;
+    std::vector<Stage> stages = build_stages(ds.h_desc.p, nch, ctx->slot_bytes);
+    std::vector<cudaEvent_t> filled(ds.n_slots), verified(ds.n_slots);
+    for (uint32_t i = 0; i < ds.n_slots; ++i) {
+      filled[i] = ds.events.get();
+      verified[i] = ds.events.get();
+    }
+    for (size_t s = 0; s < stages.size(); ++s) {
+      const Stage& S = stages[s];
+      const uint32_t k = (uint32_t)(s % ds.n_slots);
+      if (s >= ds.n_slots) ck(cudaStreamWaitEvent(ds.copy, verified[k], 0));
+      ck(cudaMemcpyAsync(ds.slot(k), img->host + P.L.payload_off + S.img_lo, S.img_hi - S.img_lo,
+                         cudaMemcpyHostToDevice, ds.copy));
+      ck(cudaEventRecord(filled[k], ds.copy));
+      ck(cudaStreamWaitEvent(ds.compute, filled[k], 0));
+      lp.c0 = S.c0;
+      lp.c1 = S.c1;
+      lp.image = ds.slot(k);
+      lp.image_base = S.img_lo;
+      timed_launch(ds, kt, true, lp, ds.compute);
+      ck(cudaEventRecord(verified[k], ds.compute));
+    }
+    ck(cudaEventRecord(c_end, ds.copy));
+    if (stages.empty()) ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
+    tm.n_stages = stages.size();
+  }
+  ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
+  ck(cudaStreamSynchronize(ds.compute));
+  ck(cudaStreamSynchronize(ds.copy));
+  const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
+  float cms = 0;
+  if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
+  tm.kernel_ms = kt.sum_ms();
+  tm.n_kernels = kt.spans.size();
+  tmp_payload.release();
+  tmp_crc.release();
+  if (rep) set_report(rep, P, n_bad, first_bad);
+  if (n_bad) {
+    ctx->last = tm;
+    return CHECL_ERR_CRC_MISMATCH;  // arena freed by its destructor; nothing rebound
+  }
+  // r5: rebind every handle (all-or-nothing)
+  (void)in_migrate;
+  commit(ctx, P, device, arena);
+  tm.total_ms = now_ms() - t0;
+  ctx->last = tm;
+  return CHECL_SUCCESS;
+}
+
+}  // namespace
+
+// ============================== C ABI =========================================
+
+extern "C" {
+
+checl_status checl_create(const checl_allocator* a, checl_ctx** out) {
+  if (!out) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    auto* c = new checl_ctx();
+    if (a) c->alloc = *a;
+    if (const char* s = std::getenv("CHECL_STAGING_BYTES")) {
+      const unsigned long long v = std::strtoull(s, nullptr, 10);
+      if (v >= kChunkBytes + kBufferAlign && v % kChunkBytes == 0) c->slot_bytes = v;
+    }
+    *out = c;
+    return CHECL_SUCCESS;
+  });
+}
+
+checl_status checl_destroy(checl_ctx* ctx) {
+  if (!ctx) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    {
+      // delete in the reverse of creation order (L19-L20)
+      std::lock_guard<std::mutex> lk(ctx->mu);
+      std::vector<std::shared_ptr<Arena>> arenas;
+      for (auto it = ctx->entries.rbegin(); it != ctx->entries.rend(); ++it) {
+        if (it->second.arena) {
+          int prev = -1;
+          cudaGetDevice(&prev);
+          cudaSetDevice(it->second.device);
+          cudaDeviceSynchronize();
+          if (prev >= 0) cudaSetDevice(prev);
+          arenas.push_back(it->second.arena);
+        }
+      }
+      ctx->entries.clear();
+      arenas.clear();
+    }
+    for (auto*& d : ctx->devs) {
+      if (d) {
+        d->destroy();
+        delete d;
+        d = nullptr;
+      }
+    }
+    delete ctx;
+    return CHECL_SUCCESS;
+  });
+}
+
+checl_status checl_set_staging(checl_ctx* ctx, size_t slot_bytes, uint32_t n_slots) {
+  if (!ctx || slot_bytes < kChunkBytes + kBufferAlign || slot_bytes % kChunkBytes || n_slots < 1 ||
+      n_slots > kMaxSlots)
+    return CHECL_ERR_INVALID_VALUE;
+  std::lock_guard<std::mutex> lk(ctx->mu);
+  ctx->slot_bytes = slot_bytes;
+  ctx->n_slots = n_slots;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_register_buffer(checl_ctx* ctx, int device, void* dev_ptr, size_t bytes, uint32_t flags,
+                                   checl_handle* out) {
+  if (!ctx || !out || (bytes > 0 && !dev_ptr)) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  const uintptr_t lo = reinterpret_cast<uintptr_t>(dev_ptr);
+  if (bytes && lo > ~(uintptr_t)0 - bytes) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    std::lock_guard<std::mutex> lk(ctx->mu);
+    if (bytes) {
+      auto& m = ctx->by_addr[device];
+      auto it = m.upper_bound(lo);  // first start > lo
+      if (it != m.end() && it->first < lo + bytes) return CHECL_ERR_INVALID_VALUE;
+      if (it != m.begin()) {
+        --it;  // start <= lo
+        const Entry& e = ctx->entries.at(it->second);
+        if (it->first + e.bytes > lo) return CHECL_ERR_INVALID_VALUE;
+      }
+    }
+    const uint64_t h = ctx->next_id++;
+    Entry e;
+    e.device = device;
+    e.ptr = static_cast<uint8_t*>(dev_ptr);
+    e.bytes = bytes;
+    e.flags = flags;
+    e.owned = false;
+    ctx->entries.emplace(h, std::move(e));
+    if (bytes) ctx->by_addr[device][lo] = h;
+    ctx->version[device]++;
+    *out = h;
+    return CHECL_SUCCESS;
+  });
+}
+
+checl_status checl_release(checl_ctx* ctx, checl_handle h) {
+  if (!ctx) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    std::shared_ptr<Arena> drop;
+    int dev = -1;
+    {
+      std::lock_guard<std::mutex> lk(ctx->mu);
+      auto it = ctx->entries.find(h);
+      if (it == ctx->entries.end()) return CHECL_ERR_INVALID_HANDLE;
+      Entry& e = it->second;
+      dev = e.device;
+      if (e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
+      drop = std::move(e.arena);
+      ctx->version[e.device]++;
+      ctx->entries.erase(it);
+    }
+    if (drop && drop.use_count() == 1) {
+      DeviceGuard g(dev);
+      ck(cudaDeviceSynchronize());
+    }
+    drop.reset();
+    return CHECL_SUCCESS;
+  });
+}
+
+checl_status checl_translate(const checl_ctx* ctx, checl_handle h, void** dev_ptr, size_t* bytes, int* device) {
+  if (!ctx) return CHECL_ERR_INVALID_VALUE;
+  std::lock_guard<std::mutex> lk(ctx->mu);
+  auto it = ctx->entries.find(h);
+  if (it == ctx->entries.end()) return CHECL_ERR_INVALID_HANDLE;
+  if (dev_ptr) *dev_ptr = it->second.ptr;
+  if (bytes) *bytes = it->second.bytes;
+  if (device) *device = it->second.device;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_count(const checl_ctx* ctx, int device, uint64_t* n_buffers, uint64_t* total_bytes) {
+  if (!ctx) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  std::lock_guard<std::mutex> lk(ctx->mu);
+  uint64_t n = 0, t = 0;
+  for (auto& kv : ctx->entries)
+    if (kv.second.device == device) ++n, t += kv.second.bytes;
+  if (n_buffers) *n_buffers = n;
+  if (total_bytes) *total_bytes = t;
+  return CHECL_SUCCESS;
+}
+
+static checl_status checkpoint_common(checl_ctx* ctx, int device, void* stream, uint64_t epoch, checl_image* img,
+                                      bool to_device) {
+  BusyGuard b(ctx);
+  if (!b.ok) return CHECL_ERR_BUSY;
+  return guarded([&]() { return do_checkpoint(ctx, device, stream, epoch, img, to_device); });
+}
+
+checl_status checl_checkpoint(checl_ctx* ctx, int device, void* cuda_stream, uint64_t epoch, checl_image** out) {
+  if (!ctx || !out) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  checl_image* img = new (std::nothrow) checl_image();
+  if (!img) return CHECL_ERR_OUT_OF_HOST_MEMORY;
+  checl_status st = checkpoint_common(ctx, device, cuda_stream, epoch, img, false);
+  if (st) {
+    checl_image_free(img);
+    return st;
+  }
+  *out = img;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_checkpoint_device(checl_ctx* ctx, int device, void* cuda_stream, uint64_t epoch,
+                                     checl_image** out) {
+  if (!ctx || !out) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  checl_image* img = new (std::nothrow) checl_image();
+  if (!img) return CHECL_ERR_OUT_OF_HOST_MEMORY;
+  checl_status st = checkpoint_common(ctx, device, cuda_stream, epoch, img, true);
+  if (st) {
+    checl_image_free(img);
+    return st;
+  }
+  *out = img;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_checkpoint_into(checl_ctx* ctx, int device, void* cuda_stream, uint64_t epoch,
+                                   checl_image* reuse) {
+  if (!ctx || !reuse || !reuse->owned) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  return checkpoint_common(ctx, device, cuda_stream, epoch, reuse, reuse->location == CHECL_IMAGE_DEVICE);
+}
+
+checl_status checl_image_view(const checl_image* img, const void** bytes, size_t* nbytes) {
+  if (!img || !bytes || !nbytes) return CHECL_ERR_INVALID_VALUE;
+  *bytes = img->host;
+  *nbytes = img->location == CHECL_IMAGE_DEVICE ? img->payload_off : img->image_bytes;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_image_info(const checl_image* img, int* location, int* device, uint64_t* image_bytes,
+                              void** device_payload) {
+  if (!img) return CHECL_ERR_INVALID_VALUE;
+  if (location) *location = img->location;
+  if (device) *device = img->location == CHECL_IMAGE_DEVICE ? img->device : -1;
+  if (image_bytes) *image_bytes = img->image_bytes;
+  if (device_payload) *device_payload = img->d_payload;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_image_wrap(const void* bytes, size_t nbytes, checl_image** out) {
+  if (!out || (!bytes && nbytes)) return CHECL_ERR_INVALID_VALUE;
+  checl_image* img = new (std::nothrow) checl_image();
+  if (!img) return CHECL_ERR_OUT_OF_HOST_MEMORY;
+  img->owned = false;
+  img->host = static_cast<const uint8_t*>(bytes);
+  img->host_cap = nbytes;
+  img->image_bytes = nbytes;  // validated against the header at restore
+  img->payload_off = nbytes >= 64 ? get_u64(static_cast<const uint8_t*>(bytes) + 56) : 0;
+  *out = img;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_image_to_host(const checl_image* img, checl_image** out) {
+  if (!img || !out) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    checl_image* h = new checl_image();
+    try {
+      if (img->location == CHECL_IMAGE_HOST) {
+        h->ensure_host(img->image_bytes, false);
+        std::memcpy(h->host_mut, img->host, img->image_bytes);
+      } else {
+        DeviceGuard g(img->device);
+        h->ensure_host(img->image_bytes, true);
+        std::memcpy(h->host_mut, img->host, img->payload_off);
+        if (img->image_bytes > img->payload_off)
+          ck(cudaMemcpy(h->host_mut + img->payload_off, img->d_payload, img->image_bytes - img->payload_off,
+                        cudaMemcpyDeviceToHost));
+      }
+    } catch (...) {
+      h->free_host();
+      delete h;
+      throw;
+    }
+    h->image_bytes = img->image_bytes;
+    h->payload_off = img->payload_off;
+    *out = h;
+    return CHECL_SUCCESS;
+  });
+}
+
+checl_status checl_image_free(checl_image* img) {
+  if (!img) return CHECL_SUCCESS;
+  img->free_device();
+  img->free_host();
+  delete img;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_restore(checl_ctx* ctx, const checl_image* img, int device, void* cuda_stream, checl_report* rep) {
+  if (!ctx || !img) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  if (img->location == CHECL_IMAGE_DEVICE && !valid_device(img->device)) return CHECL_ERR_INVALID_DEVICE;
+  BusyGuard b(ctx);
+  if (!b.ok) return CHECL_ERR_BUSY;
+  return guarded([&]() { return do_restore(ctx, img, device, cuda_stream, rep, false); });
+}
+
+checl_status checl_migrate(checl_ctx* ctx, int src_device, int dst_device, void* cuda_stream, checl_report* rep) {
+  if (!ctx) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(src_device) || !valid_device(dst_device)) return CHECL_ERR_INVALID_DEVICE;
+  BusyGuard b(ctx);
+  if (!b.ok) return CHECL_ERR_BUSY;
+  return guarded([&]() -> checl_status {
+    const double t0 = now_ms();
+    checl_image img;
+    checl_status st = do_checkpoint(ctx, src_device, cuda_stream, 0, &img, true);
+    checl_timing ck_t = ctx->last;
+    if (st == CHECL_SUCCESS) st = do_restore(ctx, &img, dst_device, cuda_stream, rep, true);
+    img.free_device();
+    img.free_host();
+    checl_timing& t = ctx->last;
+    t.sync_ms += ck_t.sync_ms;
+    t.plan_ms += ck_t.plan_ms;
+    t.kernel_ms += ck_t.kernel_ms;
+    t.copy_ms += ck_t.copy_ms;
+    t.n_kernels += ck_t.n_kernels;
+    t.n_stages += ck_t.n_stages;
+    t.total_ms = now_ms() - t0;
+    return st;
+  });
+}
+
+checl_status checl_last_timing(const checl_ctx* ctx, checl_timing* out) {
+  if (!ctx || !out) return CHECL_ERR_INVALID_VALUE;
+  *out = ctx->last;
+  return CHECL_SUCCESS;
+}
+
+const char* checl_status_string(checl_status s) {
+  switch (s) {
+    case CHECL_SUCCESS: return "CHECL_SUCCESS";
+    case CHECL_ERR_INVALID_VALUE: return "CHECL_ERR_INVALID_VALUE";
+    case CHECL_ERR_INVALID_HANDLE: return "CHECL_ERR_INVALID_HANDLE";
+    case CHECL_ERR_INVALID_DEVICE: return "CHECL_ERR_INVALID_DEVICE";
+    case CHECL_ERR_OUT_OF_DEVICE_MEMORY: return "CHECL_ERR_OUT_OF_DEVICE_MEMORY";
+    case CHECL_ERR_OUT_OF_HOST_MEMORY: return "CHECL_ERR_OUT_OF_HOST_MEMORY";
+    case CHECL_ERR_BAD_IMAGE: return "CHECL_ERR_BAD_IMAGE";
+    case CHECL_ERR_CRC_MISMATCH: return "CHECL_ERR_CRC_MISMATCH";
+    case CHECL_ERR_CUDA: return "CHECL_ERR_CUDA";
+    case CHECL_ERR_PEER_ACCESS: return "CHECL_ERR_PEER_ACCESS";
+    case CHECL_ERR_BUSY: return "CHECL_ERR_BUSY";
+    default: return "CHECL_ERR_UNKNOWN";
+  }
+}
+
+const char* checl_last_cuda_error(void) { return t_last_cuda_error.c_str(); }
+
+uint32_t checl_version(void) { return 0x00010000u; }
+
+checl_status checl_debug_fill(int device, void* dev_ptr, size_t bytes, uint64_t seed, uint64_t stream_id, int kind,
+                              void* cuda_stream) {
+  if ((!dev_ptr && bytes) || kind < 0 || kind > 2) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  return guarded([&]() -> checl_status {
+    DeviceGuard g(device);
+    int sms = 0;
+    ck(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
+    auto mix = [](uint64_t z) {
+      z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+      z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+      return z ^ (z >> 31);
+    };
+    const uint64_t key = mix((seed * 0x9E3779B97F4A7C15ull) ^ ((stream_id + 1) * 0xD1B54A32D192ED03ull));
+    ck(launch_fill(static_cast<uint8_t*>(dev_ptr), bytes, key, kind, sms, static_cast<cudaStream_t>(cuda_stream)));
+    return CHECL_SUCCESS;
+  });
+}
+
+checl_status checl_debug_compare(int device, const void* a, const void* b, size_t bytes, uint64_t* n_diff) {
+  if (!n_diff || ((!a || !b) && bytes)) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  return guarded([&]() -> checl_status {
+    DeviceGuard g(device);
+    int sms = 0;
+    ck(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, device));
+    unsigned long long* d = nullptr;
+    ck(cudaMalloc(&d, 8));
+    unsigned long long h = 0;
+    cudaError_t e = cudaMemset(d, 0, 8);
+    if (e == cudaSuccess)
+      e = launch_compare(static_cast<const uint8_t*>(a), static_cast<const uint8_t*>(b), bytes, d, sms, nullptr);
+    if (e == cudaSuccess) e = cudaMemcpy(&h, d, 8, cudaMemcpyDeviceToHost);
+    cudaFree(d);
+    ck(e);
+    *n_diff = h;
+    return CHECL_SUCCESS;
+  });
+}
+
+checl_status checl_debug_corrupt(checl_image* img, uint64_t image_offset, uint8_t mask) {
+  if (!img) return CHECL_ERR_INVALID_VALUE;
+  if (image_offset >= img->image_bytes) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    if (img->location == CHECL_IMAGE_DEVICE && image_offset >= img->payload_off) {
+      DeviceGuard g(img->device);
+      uint8_t* p = img->d_payload + (image_offset - img->payload_off);
+      uint8_t v = 0;
+      ck(cudaMemcpy(&v, p, 1, cudaMemcpyDeviceToHost));
+      v ^= mask;
+      ck(cudaMemcpy(p, &v, 1, cudaMemcpyHostToDevice));
+      return CHECL_SUCCESS;
+    }
+    if (!img->owned) return CHECL_ERR_INVALID_VALUE;  // wrapped bytes are the caller's
+    img->host_mut[image_offset] ^= mask;
+    return CHECL_SUCCESS;
+  });
+}
+
+}  // extern "C"

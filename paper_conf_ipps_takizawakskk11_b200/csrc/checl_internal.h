@@ -1,0 +1,108 @@
+// checl_internal.h — internal types of libchecl (product code; no oracle code).
+//
+// Format constants are FORMAT.md's; the CRC32C arithmetic is GF(2)[x] modulo the
+// Castagnoli polynomial in the reflected bit order CRC registers use (bit 31 of a
+// 32-bit value is the coefficient of x^0, bit 0 that of x^31).
+#pragma once
+
+#include <cstddef>
+#include <cstdint>
+
+#ifdef __CUDACC__
+#define CHECL_HD __host__ __device__ __forceinline__
+#else
+#define CHECL_HD inline
+#endif
+
+namespace checl {
+
+constexpr uint32_t kChunkBytes = 65536;     // FORMAT.md chunk_bytes
+constexpr uint32_t kBufferAlign = 256;      // payload_align
+constexpr uint32_t kHeaderBytes = 128;      // header_bytes
+constexpr uint32_t kRecordBytes = 48;       // manifest record
+constexpr uint32_t kPayloadAlign = 4096;    // payload_off alignment
+constexpr uint32_t kPolyRefl = 0x82F63B78u; // x^32 + ... (Castagnoli), low terms, reflected
+constexpr uint32_t kOne = 0x80000000u;      // the polynomial 1 (x^0) in reflected order
+constexpr uint32_t kX = 0x40000000u;        // the polynomial x
+
+// One chunk of the flat work list (16 bytes). `ptr` is the registered buffer's
+// address of the chunk (pack: source; restore: destination). The chunk's payload
+// offset is img_off_256 * 256 (chunks start on 256-byte boundaries: buffers are
+// 256-aligned and chunks are 64 KiB apart inside a buffer). len in [1, 65536];
+// pad = zero bytes owned after the chunk (< 256, non-zero only for a buffer's
+// last chunk).
+struct ChunkDesc {
+  uint64_t ptr;
+  uint32_t img_off_256;
+  uint32_t len_pad;  // len | pad << 24
+};
+static_assert(sizeof(ChunkDesc) == 16, "ChunkDesc is 16 bytes");
+
+CHECL_HD uint32_t desc_len(const ChunkDesc& d) { return d.len_pad & 0x1FFFFu; }
+CHECL_HD uint32_t desc_pad(const ChunkDesc& d) { return d.len_pad >> 24; }
+CHECL_HD uint32_t make_len_pad(uint32_t len, uint32_t pad) { return len | (pad << 24); }
+
+// a * x mod P: one zero bit through the CRC register.
+CHECL_HD uint32_t gf_mulx(uint32_t a) { return (a >> 1) ^ ((a & 1u) ? kPolyRefl : 0u); }
+
+// a * x^-1 mod P (x is invertible: P has a constant term). Inverse of gf_mulx:
+// bit 31 of gf_mulx(a) equals bit 0 of a because kPolyRefl has bit 31 set.
+CHECL_HD uint32_t gf_divx(uint32_t r) {
+  uint32_t b = r >> 31;
+  return ((r ^ (b ? kPolyRefl : 0u)) << 1) | b;
+}
+
+// a * b mod P.
+CHECL_HD uint32_t gf_mul(uint32_t a, uint32_t b) {
+  uint32_t p = 0;
+  for (int i = 0; i < 32; ++i) {
+    if (a & (kOne >> i)) p ^= b;
+    b = gf_mulx(b);
+  }
+  return p;
+}
+
+// x^(2^k) mod P.
+CHECL_HD uint32_t gf_x_pow2k(int k) {
+  uint32_t r = kX;
+  for (int i = 0; i < k; ++i) r = gf_mul(r, r);
+  return r;
+}
+
+// x^(8n) mod P (shift of a CRC register over n zero bytes), square-and-multiply.
+CHECL_HD uint32_t gf_x8n(uint64_t n) {
+  uint32_t r = kOne, sq = gf_mul(kX, kX);  // x^2
+  sq = gf_mul(sq, sq);                     // x^4
+  sq = gf_mul(sq, sq);                     // x^8
+  while (n) {
+    if (n & 1u) r = gf_mul(r, sq);
+    sq = gf_mul(sq, sq);
+    n >>= 1;
+  }
+  return r;
+}
+
+// Kernel geometry: one warp per chunk, 32 stripes of 2 KiB,
+// moved in rounds of 32 x 128 B.
+constexpr int kStripeBytes = kChunkBytes / 32;   // 2048
+constexpr int kSegBytes = 128;                   // per stripe per round
+constexpr int kRowPitch = kSegBytes + 16;        // padded smem row: conflict-free LDS.128
+constexpr int kWarpsPerCta = 16;
+constexpr int kThreadsPerCta = kWarpsPerCta * 32;
+constexpr int kFoldLevels = 5;                   // log2(32 stripes)
+
+// Parameters of one pack (checkpoint) or verify (restore) launch over the chunk
+// range [c0, c1) of `desc`. Payload byte o of the image lives at
+// image + o - image_base for the chunks of this launch.
+struct LaunchParams {
+  const ChunkDesc* desc;
+  uint64_t c0, c1;
+  uint8_t* image;           // pack: destination slot; verify: source (may be a peer address)
+  uint64_t image_base;      // payload offset that maps to image[0]
+  uint32_t* crc;            // pack: output table (global chunk index); verify: reference table
+  const uint32_t* inv_z;    // 65536 entries, x^(-8z) mod P
+  unsigned long long* status;  // verify: [0] = first bad chunk (atomicMin), [1] = bad count
+  uint32_t fold[kFoldLevels];  // x^(8 * 2048 * 2^k) mod P
+};
+
+}  // namespace checl
