@@ -1,0 +1,381 @@
+"""Benchmark of the CheCL snapshot hot path (checkpoint -> coordinate -> restore).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config C2] [--kind random]
+    python bench.py --impl reference ...     # the CPU oracle on the same workload
+
+One step = one pass of every SURVEY.md §8(a) row over the workload's buffers:
+a1 sync, a2 plan, a3 pack+CRC (K1), a4 drain, a5 finalize, a6 coordination
+all-reduce (N > 1), r1 validate, r2 re-create, r3 fill, r4 verify+scatter (K2),
+r5 rebind. `value` keeps the image resident in HBM (a4/r3 are HBM-resident, the
+path `checl_migrate` uses); `e2e` is the same step through the C ABI with the
+image in pinned HOST memory (PCIe D2H drain + H2D fill inside the timed region).
+Metric: payload GB/s of checkpoint + restore = bytes / (t_checkpoint + t_restore),
+summed over ranks, timed with CUDA events, max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "checkpoint & restore GB/s per GPU and box (1/2/4/8), % of HBM/PCIe roofline"
+L2_BYTES = 126 * 2**20
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", default="C2", choices=["C1", "C2", "C3", "C4", "C5"])
+    ap.add_argument("--kind", default="random", choices=["random", "float", "zeros"])
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--c4-scale", type=float, default=1.0)
+    return ap.parse_args()
+
+
+def workload(cfg: str, rank: int, c4_scale: float):
+    import synth
+    if cfg == "C4":
+        return synth.c4_md_rank(rank, c4_scale)
+    w = synth.CONFIGS[cfg]()
+    w.seed += 1000 * rank
+    return w
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.rows = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.index}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) == 7:
+                self.rows.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc:
+            time.sleep(0.25)
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=2)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[3 + i].lower().startswith("active")})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows)}
+
+
+def pcie_probe(dev: int, nbytes: int = 256 << 20):
+    """Pinned D2H / H2D copy bandwidth (torch plumbing, untimed region): the PCIe roofline."""
+    import torch
+    h = torch.empty(nbytes, dtype=torch.uint8, pin_memory=True)
+    d = torch.empty(nbytes, dtype=torch.uint8, device=dev)
+    out = {}
+    s = torch.cuda.Stream(dev)
+    for name, fn in (("d2h", lambda: h.copy_(d, non_blocking=True)), ("h2d", lambda: d.copy_(h, non_blocking=True))):
+        with torch.cuda.stream(s):
+            fn()
+            fn()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(s)
+            for _ in range(5):
+                fn()
+            e1.record(s)
+        e1.synchronize()
+        out[name] = nbytes * 5 / (e0.elapsed_time(e1) * 1e-3) / 1e9
+    del h, d
+    return out
+
+
+def cpu_baseline(w, max_seconds: float = 20.0):
+    """The oracle (oracle/, as it stands) on the same workload: checkpoint + restore."""
+    import numpy as np
+    import synth
+    from oracle import oracle as O
+    total = w.total_bytes
+    # bounded sample: whole buffers in order until ~1.5 GB (C2 fits whole)
+    picked, acc = [], 0
+    for b in w.buffers:
+        if picked and acc + b.size > 1_500_000_000:
+            break
+        picked.append(b)
+        acc += b.size
+    ents = [O.Entry(i + 1, synth.fill_bytes(b.size, w.seed, b.stream), b.flags) for i, b in enumerate(picked)]
+    times = []
+    t_start = time.perf_counter()
+    while True:
+        t0 = time.perf_counter()
+        img = O.checkpoint(ents, device=0, epoch=1)
+        st, rep, back = O.restore(img)
+        t = time.perf_counter() - t0
+        assert st == 0
+        times.append(t)
+        del img, back
+        if time.perf_counter() - t_start > max_seconds or len(times) >= 3:
+            break
+    t = statistics.median(times)
+    sample = (f"{len(picked)}/{len(w.buffers)} buffers of {w.name} ({acc} of {total} B), "
+              f"oracle checkpoint+restore, median of {len(times)}")
+    return {"value": acc / t / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample,
+            "ms_per_roundtrip": t * 1e3}
+
+
+def run_reference(a):
+    """--impl reference: the oracle, as it stands, on the host cores (rank 0 only)."""
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import numpy as np
+    import synth
+    from oracle import oracle as O
+    w = workload(a.config, 0, a.c4_scale)
+    picked, acc = [], 0
+    budget = 600_000_000  # bounded sample per step so K steps end within minutes
+    for b in w.buffers:
+        if picked and acc + b.size > budget:
+            break
+        picked.append(b)
+        acc += b.size
+    ents = [O.Entry(i + 1, synth.fill_bytes(b.size, w.seed, b.stream), b.flags) for i, b in enumerate(picked)]
+    for _ in range(a.warmup):
+        O.restore(O.checkpoint(ents, 0, 1))
+    t0 = time.perf_counter()
+    for _ in range(a.steps):
+        img = O.checkpoint(ents, 0, 1)
+        st, _, _ = O.restore(img)
+        assert st == 0
+    dt = time.perf_counter() - t0
+    value = acc * a.steps / dt / 1e9
+    sample = f"{len(picked)}/{len(w.buffers)} buffers of {w.name}, {acc} B per step (oracle pack+CRC+restore, 1 thread)"
+    print(json.dumps({
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": a.gpus, "steps": a.steps,
+        "warmup": a.warmup, "ms_per_step": dt / a.steps * 1e3, "higher_is_better": True, "scaling": "weak",
+        "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": w.name, "payload_bytes_per_gpu": w.total_bytes, "n_buffers": len(w.buffers)},
+        "cpu_baseline": {"value": value, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }))
+
+
+def main():
+    a = parse()
+    if a.impl == "reference":
+        run_reference(a)
+        return
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ipps_takizawakskk11_b200 import checl
+    from paper_conf_ipps_takizawakskk11_b200.coordination import agree
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    dev = local
+    torch.cuda.set_device(dev)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+    w = workload(a.config, rank, a.c4_scale)
+    kind = {"random": checl.FILL_RANDOM, "float": checl.FILL_FLOAT, "zeros": checl.FILL_ZEROS}[a.kind]
+
+    # the application's buffers (user-owned), filled on the device by the synth/ generator
+    tensors = [torch.empty(b.size, dtype=torch.uint8, device=dev) for b in w.buffers]
+    for t, b in zip(tensors, w.buffers):
+        checl.debug_fill(t, w.seed, b.stream, kind)
+    torch.cuda.synchronize()
+    ctx = checl.Context()
+    handles = [ctx.register(t, b.flags) for t, b in zip(tensors, w.buffers)]
+    S = w.total_bytes
+    n_chunks = sum((b.size + 65535) // 65536 for b in w.buffers)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    def coordinate(ok: bool, epoch: int):
+        if world > 1:
+            f, _, _, same, _ = agree(not ok, len(handles), S, epoch, None, dev)
+            assert f == 0 and same
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    def sum_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.SUM)
+        return float(t.item())
+
+    def run(img, steps, collect):
+        """steps x (checkpoint_into img -> coordinate -> restore img); returns device ms."""
+        cur = torch.cuda.current_stream(dev)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(cur)
+        for i in range(steps):
+            ctx.checkpoint(dev, epoch=i + 1, into=img)
+            tc = ctx.last_timing()
+            coordinate(True, i + 1)
+            ctx.restore(img, dev)
+            tr = ctx.last_timing()
+            if collect is not None:
+                collect.append((tc, tr))
+        e1.record(cur)
+        e1.synchronize()
+        return e0.elapsed_time(e1)
+
+    # -- value: device-resident image (HBM) --------------------------------------
+    dimg = ctx.checkpoint_device(dev, epoch=0)
+    run(dimg, a.warmup, None)
+    phases = []
+    barrier()
+    with ClockSampler(dev) as clk:
+        ms = run(dimg, a.steps, phases)
+    barrier()
+    ms_max = max_over_ranks(ms)
+    value = sum_over_ranks(S * a.steps) / (ms_max * 1e-3) / 1e9
+    # correctness of the last restore: every handle's new buffer == the application's bytes
+    n_diff = 0
+    for h, t in zip(handles, tensors):
+        ptr, nb, d = ctx.translate(h)
+        n_diff += checl.debug_compare(dev, ptr, t.data_ptr(), nb) if nb else 0
+    pack_ms = statistics.mean(p[0]["kernel_ms"] for p in phases)
+    verify_ms = statistics.mean(p[1]["kernel_ms"] for p in phases)
+    ck_ms = statistics.mean(p[0]["total_ms"] for p in phases)
+    rs_ms = statistics.mean(p[1]["total_ms"] for p in phases)
+    launches = sum(p[0]["n_kernels"] + p[1]["n_kernels"] for p in phases)
+    pk = peaks()
+    hbm_peak = pk.get("hbm_gbs")
+    peak_src = "MEASURED_PEAKS.json hbm_gbs (measured copy)" if hbm_peak else "fallback 6650 GB/s (B200_PROFILING.md)"
+    hbm_peak = hbm_peak or 6650.0
+    alg = 2 * S + 4 * n_chunks  # K1: read S + write S + CRC table; K2: read S + write S + read table
+    dom_ms, dom_name = (pack_ms, "pack_gather_crc (K1)") if pack_ms >= verify_ms else (verify_ms, "verify_scatter (K2)")
+    achieved = alg / (dom_ms * 1e-3) / 1e9
+    traffic = None
+    tf = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tf):
+        try:
+            traffic = json.load(open(tf)).get(a.config, {}).get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    dimg.free()
+
+    # -- e2e: pinned host image through the C ABI (PCIe inside the timed region) ----
+    e2e = None
+    if not a.no_e2e:
+        pcie = pcie_probe(dev)
+        himg = ctx.checkpoint(dev, epoch=0)
+        payload_span = himg.info()["image_bytes"]
+        run(himg, a.warmup, None)
+        ph2 = []
+        barrier()
+        ms2 = run(himg, a.steps, ph2)
+        barrier()
+        ms2_max = max_over_ranks(ms2)
+        E = sum_over_ranks(S * a.steps) / (ms2_max * 1e-3) / 1e9
+        ck2 = statistics.mean(p[0]["total_ms"] for p in ph2)
+        rs2 = statistics.mean(p[1]["total_ms"] for p in ph2)
+        drain = statistics.mean(p[0]["copy_ms"] for p in ph2)
+        fill = statistics.mean(p[1]["copy_ms"] for p in ph2)
+        himg.free()
+        pay = S  # payload bytes carried each way (+ padding, tables below)
+        e2e = {
+            "value": E, "unit": "GB/s",
+            "h2d_bytes_per_step": payload_span + 20 * n_chunks + 16,  # image payload + CRC table + descriptors + status
+            "d2h_bytes_per_step": payload_span + 4 * n_chunks + 16,   # payload + CRC table + status word
+            "checkpoint_ms": ck2, "restore_ms": rs2,
+            "checkpoint_GBs": pay / (ck2 * 1e-3) / 1e9, "restore_GBs": pay / (rs2 * 1e-3) / 1e9,
+            "drain_GBs": pay / (drain * 1e-3) / 1e9, "fill_GBs": pay / (fill * 1e-3) / 1e9,
+            "pcie_measured_GBs": pcie,
+            "drain_frac_of_pcie": (pay / (drain * 1e-3) / 1e9) / pcie["d2h"],
+            "fill_frac_of_pcie": (pay / (fill * 1e-3) / 1e9) / pcie["h2d"],
+            "gpu_launches": sum(p[0]["n_kernels"] + p[1]["n_kernels"] for p in ph2),
+            "image": "pinned host memory (cudaHostAlloc), reused across steps",
+        }
+
+    cpu = None
+    if rank == 0 and world == 1 and not a.no_cpu_baseline:
+        cpu = cpu_baseline(w)
+        cpu["cores_available"] = os.cpu_count()
+
+    if rank == 0:
+        out = {
+            "metric": METRIC, "value": value, "unit": "GB/s", "n_gpus": world, "steps": a.steps,
+            "warmup": a.warmup, "ms_per_step": ms_max / a.steps, "higher_is_better": True, "scaling": "weak",
+            "vs_baseline": None, "dtype": "u8", "data": "synthetic",
+            "config": {"workload": w.name, "payload_bytes_per_gpu": S, "n_buffers": len(w.buffers),
+                       "n_chunks": n_chunks, "fill": a.kind,
+                       "image": "device-resident (HBM), reused across steps",
+                       "l2": ("inputs larger than L2" if S > L2_BYTES else "inputs smaller than L2 (not flushed)"),
+                       "parallelism": f"independent snapshot per rank, {world} rank(s)"},
+            "roofline": {"bound": "hbm", "kernel": dom_name, "achieved": achieved, "peak": hbm_peak,
+                         "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic,
+                         "peak_source": peak_src, "algorithmic_bytes_per_launch": alg,
+                         "pack_ms": pack_ms, "verify_ms": verify_ms},
+            "phases": {"checkpoint_ms": ck_ms, "restore_ms": rs_ms, "checkpoint_GBs": S / (ck_ms * 1e-3) / 1e9,
+                       "restore_GBs": S / (rs_ms * 1e-3) / 1e9,
+                       "pack_GBs_2S": 2 * S / (pack_ms * 1e-3) / 1e9, "verify_GBs_2S": 2 * S / (verify_ms * 1e-3) / 1e9,
+                       "checkpoint_detail": phases[-1][0], "restore_detail": phases[-1][1]},
+            "verified": n_diff == 0,
+            "gpu_launches": launches,
+            "clocks": clk.summary(),
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+        }
+        print(json.dumps(out))
+    for h in handles:
+        ctx.release(h)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,106 @@
+"""-m "not gpu": the C-ABI library loads, exports every symbol include/checl.h
+declares, and its host logic (handle table, overlap checks, ids, wrapped images,
+status strings) works from C and from Python without a GPU."""
+import os
+import re
+import subprocess
+import sys
+
+import pytest
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+HEADER = os.path.join(ROOT, "include", "checl.h")
+PKG = os.path.join(ROOT, "paper_conf_ipps_takizawakskk11_b200")
+LIB = os.path.join(PKG, "libchecl.so")
+
+
+@pytest.fixture(scope="module")
+def built():
+    from paper_conf_ipps_takizawakskk11_b200 import build
+    build.build()
+    return LIB
+
+
+def declared_symbols():
+    text = open(HEADER).read()
+    text = re.sub(r"/\*.*?\*/", "", text, flags=re.S)
+    return sorted(set(re.findall(r"\b(checl_[a-z_]+)\s*\(", text)))
+
+
+def test_header_declares_the_north_star_calls():
+    syms = declared_symbols()
+    for s in ("checl_register_buffer", "checl_release", "checl_checkpoint", "checl_restore", "checl_translate",
+              "checl_migrate", "checl_image_free"):
+        assert s in syms
+
+
+def test_library_exports_every_declared_symbol(built):
+    out = subprocess.run(["nm", "-D", "--defined-only", built], capture_output=True, text=True, check=True).stdout
+    exported = set(re.findall(r"\bT (checl_\w+)", out))
+    missing = [s for s in declared_symbols() if s not in exported]
+    assert not missing, missing
+
+
+def test_library_is_sm100a(built):
+    out = subprocess.run(["cuobjdump", "--list-elf", built], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def test_python_binding_declares_every_export(built):
+    from paper_conf_ipps_takizawakskk11_b200 import checl
+    assert sorted(checl.EXPORTS) == declared_symbols()
+    for s in checl.EXPORTS:
+        assert hasattr(checl.lib, s)
+
+
+def test_c_client_registry_without_gpu(built, tmp_path):
+    exe = tmp_path / "abi_registry"
+    subprocess.check_call(["gcc", "-std=c99", "-Wall", "-Werror", f"-I{ROOT}/include",
+                           os.path.join(ROOT, "tests", "c", "abi_registry.c"), f"-L{PKG}", "-lchecl",
+                           f"-Wl,-rpath,{PKG}", "-o", str(exe)])
+    env = dict(os.environ, CHECL_FAKE_DEVICES="2")
+    r = subprocess.run([str(exe)], capture_output=True, text=True, env=env)
+    assert r.returncode == 0, r.stderr
+    assert "abi_registry ok" in r.stdout
+
+
+PY_REGISTRY = r"""
+import os, sys
+sys.path.insert(0, %r)
+from paper_conf_ipps_takizawakskk11_b200 import checl
+c = checl.Context(allocator="cuda")
+hs = [c.register_ptr(0, 0x10000 + 0x1000 * i, 0x800 + i, flags=i) for i in range(100)]
+assert hs == list(range(1, 101))
+assert c.count(0) == (100, sum(0x800 + i for i in range(100)))
+for h in hs[::2]:
+    c.release(h)
+assert c.count(0)[0] == 50
+assert c.translate(hs[1]) == (0x11000, 0x801, 0)
+try:
+    c.register_ptr(0, 0x11000 + 0x800, 4)
+    raise SystemExit("overlap not detected")
+except checl.CheclError as e:
+    assert e.status == checl.ERR_INVALID_VALUE
+assert c.register_ptr(0, 0x10000, 0x1000) == 101   # released range reusable, id fresh
+img = checl.Image.wrap(bytes(4096))
+assert img.view().size == 4096 and img.info()["location"] == checl.IMAGE_HOST
+img.free()
+c.close()
+print("ok")
+"""
+
+
+def test_python_registry_without_gpu(built):
+    env = dict(os.environ, CHECL_FAKE_DEVICES="1")
+    r = subprocess.run([sys.executable, "-c", PY_REGISTRY % ROOT], capture_output=True, text=True, env=env)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stderr
+
+
+def test_missing_library_fails_loudly(tmp_path):
+    # a copy of the package without libchecl.so must refuse to import (no CPU fallback)
+    import shutil
+    dst = tmp_path / "paper_conf_ipps_takizawakskk11_b200"
+    shutil.copytree(PKG, dst, ignore=shutil.ignore_patterns("*.so", "build_obj", "__pycache__"))
+    r = subprocess.run([sys.executable, "-c", "import paper_conf_ipps_takizawakskk11_b200"], cwd=tmp_path,
+                       capture_output=True, text=True)
+    assert r.returncode != 0 and "ImportError" in r.stderr and "no CPU fallback" in r.stderr

@@ -1,0 +1,79 @@
+"""-m "not gpu": the coordinated (global) snapshot protocol over torch.distributed
+gloo on CPU, world_size 2 and 8. Local snapshots are mocked;
+the commit rule is PAPER.md L40's global snapshot read as a two-phase commit
+(reading 16): commit iff no rank failed and all epochs agree."""
+import os
+import socket
+
+import pytest
+import torch.multiprocessing as mp
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+class FakeImage:
+    def __init__(self):
+        self.freed = False
+
+    def free(self):
+        self.freed = True
+
+
+def _worker(rank, world, port, scenario, q):
+    import torch.distributed as dist
+    from paper_conf_ipps_takizawakskk11_b200.coordination import coordinated
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    img = FakeImage()
+
+    def local():
+        if scenario == "fail" and rank == world - 1:
+            raise RuntimeError("injected local checkpoint failure")
+        return img, 3 + rank, 1000 * (rank + 1)
+
+    epoch = 7 if not (scenario == "epoch" and rank == 0) else 8
+    g = coordinated(local, epoch)
+    q.put((rank, g.committed, g.failures, g.n_buffers, g.total_bytes, g.epochs_agree, img.freed, g.image is None))
+    dist.destroy_process_group()
+
+
+def _run(world, scenario):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_worker, args=(r, world, port, scenario, q)) for r in range(world)]
+    for p in ps:
+        p.start()
+    out = [q.get(timeout=120) for _ in range(world)]
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    return sorted(out)
+
+
+@pytest.mark.parametrize("world", [2, 8])
+def test_commit_sums_closed_form(world):
+    for rank, ok, f, nb, tb, same, freed, none in _run(world, "ok"):
+        assert ok and f == 0 and same and not freed and not none
+        assert nb == sum(3 + r for r in range(world))           # closed form of the SUM
+        assert tb == sum(1000 * (r + 1) for r in range(world))
+
+
+@pytest.mark.parametrize("world", [2, 8])
+def test_one_failing_rank_aborts_everyone(world):
+    res = _run(world, "fail")
+    for rank, ok, f, nb, tb, same, freed, none in res:
+        assert not ok and f == 1 and none
+        if rank != world - 1:
+            assert freed  # surviving ranks free their local images
+
+
+def test_epoch_disagreement_aborts():
+    for rank, ok, f, nb, tb, same, freed, none in _run(2, "epoch"):
+        assert not ok and f == 0 and not same and none
