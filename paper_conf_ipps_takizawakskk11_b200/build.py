@@ -11,8 +11,9 @@ import sys
 PKG = os.path.dirname(os.path.abspath(__file__))
 ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
-LIB = os.path.join(PKG, "libchecl.so")
-OBJ = os.path.join(PKG, "build_obj")
+LIB = os.environ.get("CHECL_LIB_OUT", os.path.join(PKG, "libchecl.so"))
+OBJ = os.path.join(os.path.dirname(LIB), "build_obj" + os.environ.get("CHECL_OBJ_SUFFIX", ""))
+EXTRA = os.environ.get("CHECL_EXTRA_FLAGS", "").split()  # experiments only (e.g. -DCHECL_WARPS=8)
 SOURCES = ["checl_kernels.cu", "checl_engine.cpp", "checl_hostcrc.cpp"]
 HEADERS = [os.path.join(CSRC, "checl_internal.h"), os.path.join(ROOT, "include", "checl.h")]
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
@@ -35,7 +36,7 @@ def build(force: bool = False, verbose: bool = False) -> str:
         obj = os.path.join(OBJ, src + ".o")
         objs.append(obj)
         if force or _stale(obj, [path] + HEADERS):
-            cmd = [NVCC, *ARCH, *COMMON, "-c", path, "-o", obj]
+            cmd = [NVCC, *ARCH, *COMMON, *EXTRA, "-c", path, "-o", obj]
             if verbose and src.endswith(".cu"):
                 cmd[1:1] = ["-Xptxas", "-v"]
             if verbose:

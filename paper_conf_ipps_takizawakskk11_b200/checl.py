@@ -20,7 +20,7 @@ from typing import Optional, Tuple
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libchecl.so")
+LIB_PATH = os.environ.get("CHECL_LIB", os.path.join(_HERE, "libchecl.so"))  # override: experiments only
 
 SUCCESS = 0
 ERR_INVALID_VALUE = -1

@@ -112,12 +112,12 @@ struct DeviceGuard {
   }
 };
 
-// x^(-8z) mod P for z in [0, 65536): the short-chunk correction of the kernels.
+// x^(-8z) mod P for z in [0, 4096): the zero-padding correction of the kernels.
 const std::vector<uint32_t>& inv_z_table() {
   static const std::vector<uint32_t> t = [] {
-    std::vector<uint32_t> v(kChunkBytes);
+    std::vector<uint32_t> v(kRoundBytes);
     uint32_t r = kOne;
-    for (uint32_t z = 0; z < kChunkBytes; ++z) {
+    for (uint32_t z = 0; z < (uint32_t)kRoundBytes; ++z) {
       v[z] = r;
       for (int b = 0; b < 8; ++b) r = gf_divx(r);
     }
@@ -127,7 +127,7 @@ const std::vector<uint32_t>& inv_z_table() {
 }
 
 void fill_fold(uint32_t fold[kFoldLevels]) {
-  for (int k = 0; k < kFoldLevels; ++k) fold[k] = gf_x_pow2k(14 + k);  // x^(8*2048*2^k)
+  for (int k = 0; k < kFoldLevels; ++k) fold[k] = gf_x_pow2k(10 + k);  // x^(8*128*2^k)
 }
 
 // ---- per-device resources ---------------------------------------------------
@@ -232,8 +232,8 @@ struct DevState {
     ck(cudaStreamCreateWithFlags(&compute, cudaStreamNonBlocking));
     ck(cudaStreamCreateWithFlags(&copy, cudaStreamNonBlocking));
     ck(snapshot_configure());
-    inv_z.ensure(kChunkBytes);
-    ck(cudaMemcpy(inv_z.p, inv_z_table().data(), kChunkBytes * 4, cudaMemcpyHostToDevice));
+    inv_z.ensure(kRoundBytes);
+    ck(cudaMemcpy(inv_z.p, inv_z_table().data(), kRoundBytes * 4, cudaMemcpyHostToDevice));
     status.ensure(2);
     h_status.ensure(2);
     fill_fold(fold);
@@ -633,6 +633,7 @@ LaunchParams base_params(DevState& ds) {
   p.inv_z = ds.inv_z.p;
   p.status = ds.status.p;
   for (int k = 0; k < kFoldLevels; ++k) p.fold[k] = ds.fold[k];
+  p.horner = gf_x8n(kRoundBytes - kSegBytes);
   return p;
 }
 

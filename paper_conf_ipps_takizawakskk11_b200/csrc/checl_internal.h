@@ -82,12 +82,15 @@ CHECL_HD uint32_t gf_x8n(uint64_t n) {
   return r;
 }
 
-// Kernel geometry: one warp per chunk, 32 stripes of 2 KiB,
-// moved in rounds of 32 x 128 B.
-constexpr int kStripeBytes = kChunkBytes / 32;   // 2048
-constexpr int kSegBytes = 128;                   // per stripe per round
+// Kernel geometry: one warp per chunk, rounds of 4 KiB of
+// contiguous bytes, lane l CRCs the 128-byte segment 32r + l of round r.
+constexpr int kRoundBytes = 4096;
+constexpr int kSegBytes = 128;                   // per lane per round
 constexpr int kRowPitch = kSegBytes + 16;        // padded smem row: conflict-free LDS.128
-constexpr int kWarpsPerCta = 16;
+#ifndef CHECL_WARPS
+#define CHECL_WARPS 16
+#endif
+constexpr int kWarpsPerCta = CHECL_WARPS;
 constexpr int kThreadsPerCta = kWarpsPerCta * 32;
 constexpr int kFoldLevels = 5;                   // log2(32 stripes)
 
@@ -100,9 +103,10 @@ struct LaunchParams {
   uint8_t* image;           // pack: destination slot; verify: source (may be a peer address)
   uint64_t image_base;      // payload offset that maps to image[0]
   uint32_t* crc;            // pack: output table (global chunk index); verify: reference table
-  const uint32_t* inv_z;    // 65536 entries, x^(-8z) mod P
+  const uint32_t* inv_z;    // kRoundBytes entries, x^(-8z) mod P
   unsigned long long* status;  // verify: [0] = first bad chunk (atomicMin), [1] = bad count
-  uint32_t fold[kFoldLevels];  // x^(8 * 2048 * 2^k) mod P
+  uint32_t fold[kFoldLevels];  // x^(8 * 128 * 2^k) mod P
+  uint32_t horner;             // x^(8 * (kRoundBytes - kSegBytes)) mod P
 };
 
 }  // namespace checl

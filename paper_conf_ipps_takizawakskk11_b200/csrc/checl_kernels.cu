@@ -7,19 +7,21 @@
 //  K6 debug fill / compare (test tooling: synth/ generator on the device)
 //
 // Both K1 and K2 are one template (snapshot_kernel<kVerify>): a persistent grid,
-// one warp per 64 KiB chunk of a flat chunk list. The chunk is cut into 32
-// contiguous 2 KiB stripes, one per lane; each lane runs a slicing-by-4 CRC over
-// its stripe with lane-private lookup tables in shared memory (entry e of table k
-// for lane l sits at word (k*256 + e)*32 + l, so every lane always reads its own
-// bank: conflict-free lookups on random data). Data moves in rounds of 32 x 128 B:
-// coalesced 16-byte global loads (each warp instruction covers four full 128-byte
-// lines), a coalesced 16-byte store of the same registers to the destination, and
-// a transposition through a padded 32 x 144 B shared-memory tile so that each lane
-// then reads its own stripe segment with conflict-free 16-byte shared loads.
-// The 32 stripe registers are folded with a 5-level warp-shuffle tree (multiply by
-// x^(8*2048*2^k) mod P through nibble tables); a short chunk (the last chunk of a
-// buffer) is corrected with one multiply by x^(-8z), z = 65536 - len.
-// DESIGN.md §5 derives the resource budget.
+// one warp per chunk (<= 64 KiB) of a flat chunk list. A chunk is moved in rounds
+// of 4 KiB of contiguous bytes: eight coalesced 16-byte global loads per lane
+// (each warp instruction = 512 contiguous bytes), a coalesced 16-byte store of the
+// same registers to the destination, and a transposition through a padded
+// 32 x 144 B shared tile so that lane l then reads "its" 128-byte segment (segment
+// 32r + l of the chunk) with conflict-free 16-byte shared loads. Each lane runs a
+// slicing-by-4 CRC over its segments, carrying its register from round to round
+// with a Horner step (multiply by x^(8*3968) mod P: skip the other 31 lanes'
+// segments). Lookup tables are lane-private in shared memory (every lane reads its
+// own bank: conflict-free on any data). At the end the 32 lane registers are folded
+// with a 5-level warp-shuffle tree (multiply by x^(8*128*2^k)); a chunk whose length
+// is not a multiple of 4 KiB was CRC'd zero-padded and is corrected with one
+// multiply by x^(-8 zp). The next round's loads are issued before the current
+// round's CRC so that HBM latency hides under the table lookups.
+// DESIGN.md §5 derives the resource budget and the GF(2) identities.
 #include <cuda_runtime.h>
 
 #include "checl_internal.h"
@@ -27,9 +29,10 @@
 namespace checl {
 
 constexpr int kTabWords = 4 * 256 * 32;          // 128 KiB, lane-private slicing-by-4
+constexpr int kHornerWords = 8 * 16 * 32;       // 16 KiB lane-private nibble tables
 constexpr int kFoldWords = kFoldLevels * 8 * 16; // 2.5 KiB nibble tables
 constexpr int kStageBytes = 32 * kRowPitch;      // per warp
-constexpr size_t kSmemBytes = (size_t)(kTabWords + kFoldWords) * 4 + (size_t)kWarpsPerCta * kStageBytes;
+constexpr size_t kSmemBytes = (size_t)(kTabWords + kHornerWords + kFoldWords) * 4 + (size_t)kWarpsPerCta * kStageBytes;
 
 __device__ __forceinline__ uint4 ld_stream_v4(const void* p) {
   uint4 r;
@@ -70,25 +73,35 @@ __device__ __forceinline__ void st_partial(uint8_t* p, uint4 v, uint32_t n) {
     if ((uint32_t)i < n) p[i] = (uint8_t)(w[i >> 2] >> (8 * (i & 3)));
 }
 
-// One slicing-by-4 step over the little-endian word w (tl = this lane's column).
-__device__ __forceinline__ uint32_t crc_step4(uint32_t crc, uint32_t w, const uint32_t* tl) {
+// Lane-private slicing-by-4 tables, laid out as two "super-tables" of 256 rows x
+// 256 B: row e of A = [T3[e] x 32 lanes | T2[e] x 32 lanes], row e of B = [T1[e] |
+// T0[e]]. The byte address of T_k[e] for lane l is base + e*256 + half*128 + 4l, so
+// one PRMT builds the whole in-table offset from the data word and l4 = 4l:
+// result byte 0 = l4, byte 1 = the selected data byte, bytes 2-3 = 0. Every lane
+// reads its own bank (bank = l): conflict-free on any data.
+__device__ __forceinline__ uint32_t tab_ld(const uint8_t* tb, uint32_t off) {
+  return *reinterpret_cast<const uint32_t*>(tb + off);
+}
+
+// One slicing-by-4 step over the little-endian word w.
+__device__ __forceinline__ uint32_t crc_step4(uint32_t crc, uint32_t w, const uint8_t* tb, uint32_t l4) {
   const uint32_t x = crc ^ w;
-  return tl[(768u + (x & 0xFFu)) << 5] ^ tl[(512u + ((x >> 8) & 0xFFu)) << 5] ^
-         tl[(256u + ((x >> 16) & 0xFFu)) << 5] ^ tl[(x >> 24) << 5];
+  return tab_ld(tb, __byte_perm(x, l4, 0x5504)) ^ tab_ld(tb + 128, __byte_perm(x, l4, 0x5514)) ^
+         tab_ld(tb + 65536, __byte_perm(x, l4, 0x5524)) ^ tab_ld(tb + 65536 + 128, __byte_perm(x, l4, 0x5534));
 }
 
-__device__ __forceinline__ uint32_t crc_step1(uint32_t crc, uint32_t b, const uint32_t* tl) {
-  return (crc >> 8) ^ tl[((crc ^ b) & 0xFFu) << 5];
+__device__ __forceinline__ uint32_t crc_step1(uint32_t crc, uint32_t b, const uint8_t* tb, uint32_t l4) {
+  return (crc >> 8) ^ tab_ld(tb + 65536 + 128, __byte_perm(crc ^ b, l4, 0x5504));
 }
 
-__device__ __forceinline__ uint32_t crc_step16(uint32_t crc, uint4 q, const uint32_t* tl) {
-  crc = crc_step4(crc, q.x, tl);
-  crc = crc_step4(crc, q.y, tl);
-  crc = crc_step4(crc, q.z, tl);
-  return crc_step4(crc, q.w, tl);
+__device__ __forceinline__ uint32_t crc_step16(uint32_t crc, uint4 q, const uint8_t* tb, uint32_t l4) {
+  crc = crc_step4(crc, q.x, tb, l4);
+  crc = crc_step4(crc, q.y, tb, l4);
+  crc = crc_step4(crc, q.z, tb, l4);
+  return crc_step4(crc, q.w, tb, l4);
 }
 
-// f * x^(8*2048*2^level) mod P via 8 nibble lookups.
+// f * x^(8*128*2^level) mod P via 8 nibble lookups (shared table, once per chunk).
 __device__ __forceinline__ uint32_t fold_mul(uint32_t f, const uint32_t* ft) {
   uint32_t r = 0;
 #pragma unroll
@@ -96,23 +109,44 @@ __device__ __forceinline__ uint32_t fold_mul(uint32_t f, const uint32_t* ft) {
   return r;
 }
 
+// s * x^(8*3968) mod P (advance a lane's register over the 31 segments of the
+// other lanes) via 8 lane-private nibble lookups: entry (j, v) of lane l at byte
+// j*2048 + v*128 + 4l, bank = l.
+__device__ __forceinline__ uint32_t horner_mul(uint32_t s, const uint8_t* hb, uint32_t l4) {
+  uint32_t r = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) r ^= tab_ld(hb + j * 2048, (((s >> (4 * j)) & 15u) << 7) | l4);
+  return r;
+}
+
 template <bool kVerify>
 __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const LaunchParams p) {
   extern __shared__ __align__(16) uint32_t smem[];
   uint32_t* tab = smem;
-  uint32_t* ftab = smem + kTabWords;
-  uint8_t* stage_all = reinterpret_cast<uint8_t*>(smem + kTabWords + kFoldWords);
+  uint32_t* htab = smem + kTabWords;
+  uint32_t* ftab = htab + kHornerWords;
+  uint8_t* stage_all = reinterpret_cast<uint8_t*>(ftab + kFoldWords);
 
-  // Tables: T_k[e] = CRC register of byte e followed by k zero bytes (zero init),
-  // replicated once per lane; fold nibble tables N_l[j][v] = (v << 4j) * C_l.
-  for (int i = threadIdx.x; i < 1024; i += blockDim.x) {
-    const int k = i >> 8;
-    uint32_t r = (uint32_t)(i & 255);
-    for (int b = 0; b < 8 * (k + 1); ++b) r = gf_mulx(r);
-    uint4* dstv = reinterpret_cast<uint4*>(tab + (i << 5));
-    const uint4 rv = make_uint4(r, r, r, r);
-#pragma unroll
-    for (int j = 0; j < 8; ++j) dstv[j] = rv;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  // Tables. T_k[e] = CRC register of byte e followed by k zero bytes (zero init):
+  // T_0 by bit steps into a scratch (the warp tiles, unused yet), T_1..T_3 from
+  // it; H[j][v] = (v << 4j) * x^(8*3968); then one warp store per 32 words
+  // replicates an entry across the lanes (conflict-free).
+  uint32_t* scratch = reinterpret_cast<uint32_t*>(stage_all);
+  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
+    uint32_t r = (uint32_t)e;
+    for (int b = 0; b < 8; ++b) r = gf_mulx(r);
+    scratch[e] = r;
+  }
+  for (int i = threadIdx.x; i < 128; i += blockDim.x)
+    scratch[1024 + i] = gf_mul((uint32_t)(i & 15) << (4 * (i >> 4)), p.horner);
+  __syncthreads();
+  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
+    uint32_t r = scratch[e];
+    for (int k = 1; k < 4; ++k) {
+      r = (r >> 8) ^ scratch[r & 0xFFu];
+      scratch[k * 256 + e] = r;
+    }
   }
   for (int i = threadIdx.x; i < kFoldWords; i += blockDim.x) {
     const int lvl = i >> 7, j = (i >> 4) & 7, v = i & 15;
@@ -121,13 +155,22 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     ftab[i] = gf_mul((uint32_t)v << (4 * j), cl);
   }
   __syncthreads();
+  for (int h = warp; h < 1024; h += kWarpsPerCta) {  // h = row-half: super-table, row, half
+    const int st = h >> 9, e = (h >> 1) & 255, half = h & 1;
+    const int k = 3 - (2 * st + half);  // A = [T3|T2], B = [T1|T0]
+    tab[h * 32 + lane] = scratch[k * 256 + e];
+  }
+  for (int h = warp; h < 128; h += kWarpsPerCta) htab[h * 32 + lane] = scratch[1024 + h];
+  __syncthreads();
 
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   uint8_t* stage = stage_all + warp * kStageBytes;
-  const uint32_t* tl = tab + lane;
+  const uint8_t* tb = reinterpret_cast<const uint8_t*>(tab);
+  const uint8_t* hb = reinterpret_cast<const uint8_t*>(htab);
+  const uint32_t l4 = (uint32_t)lane * 4u;
   const uint64_t nwarps = (uint64_t)gridDim.x * kWarpsPerCta;
   const unsigned full = 0xFFFFFFFFu;
-  // this lane's slot for the transposition stores / its own row for the CRC
+  // instruction i of a round: lane l moves granule l%8 of segment 4i + l/8 (each
+  // warp instruction = 512 contiguous bytes = four full 128-byte lines)
   const int g_lane = lane & 7, s_lane = lane >> 3;
 
   for (uint64_t c = p.c0 + (uint64_t)blockIdx.x * kWarpsPerCta + warp; c < p.c1; c += nwarps) {
@@ -137,50 +180,45 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     const uint8_t* src = kVerify ? img : reinterpret_cast<const uint8_t*>(d.ptr);
     uint8_t* dst = kVerify ? reinterpret_cast<uint8_t*>(d.ptr) : img;
     const int mode = kVerify ? 0 : ((d.ptr & 15u) == 0 ? 0 : ((d.ptr & 3u) == 0 ? 1 : 2));
-
-    const int my_len = min(max((int)len - lane * kStripeBytes, 0), kStripeBytes);
+    const int nrounds = (int)((len + kRoundBytes - 1) / kRoundBytes);
     uint32_t crc = lane == 0 ? 0xFFFFFFFFu : 0u;
-    const uint32_t longest = len < (uint32_t)kStripeBytes ? len : (uint32_t)kStripeBytes;
-    const int nrounds = (int)((longest + kSegBytes - 1) / kSegBytes);
 
-    for (int r = 0; r < nrounds; ++r) {
-      uint4 v[8];
-      uint32_t off[8];
+    uint4 v[8];
+    auto load_round = [&](int r) {
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
-        off[i] = (uint32_t)(4 * i + s_lane) * kStripeBytes + (uint32_t)r * kSegBytes + (uint32_t)g_lane * 16;
-        if (off[i] + 16 <= len)
-          v[i] = ld_granule(src + off[i], mode);
-        else if (off[i] < len)
-          v[i] = ld_partial(src + off[i], len - off[i]);
+        const uint32_t o = (uint32_t)r * kRoundBytes + (uint32_t)(4 * i + s_lane) * kSegBytes + (uint32_t)g_lane * 16;
+        if (o + 16 <= len)
+          v[i] = ld_granule(src + o, mode);
+        else if (o < len)
+          v[i] = ld_partial(src + o, len - o);
         else
-          v[i] = make_uint4(0u, 0u, 0u, 0u);
+          v[i] = make_uint4(0u, 0u, 0u, 0u);  // past the chunk: CRC'd as zeros, corrected below
       }
+    };
+    load_round(0);
+    for (int r = 0; r < nrounds; ++r) {
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
-        if (off[i] < len) {
-          if (!kVerify || off[i] + 16 <= len)
-            *reinterpret_cast<uint4*>(dst + off[i]) = v[i];  // pack: zeros past len are owned padding
+        const uint32_t o = (uint32_t)r * kRoundBytes + (uint32_t)(4 * i + s_lane) * kSegBytes + (uint32_t)g_lane * 16;
+        if (o < len) {
+          if (!kVerify || o + 16 <= len)
+            *reinterpret_cast<uint4*>(dst + o) = v[i];  // pack: zeros past len are owned padding
           else
-            st_partial(dst + off[i], v[i], len - off[i]);
+            st_partial(dst + o, v[i], len - o);
         }
         *reinterpret_cast<uint4*>(stage + (4 * i + s_lane) * kRowPitch + g_lane * 16) = v[i];
       }
       __syncwarp();
-      const int vb = min(max(my_len - r * kSegBytes, 0), kSegBytes);
+      // next round's loads stay in flight while this round's CRC runs
+      if (r + 1 < nrounds) load_round(r + 1);
+#ifndef CHECL_EXP_SKIP_CRC
+      // lane l: segment 32r + l; Horner step over the other lanes' 31 segments
+      if (r > 0) crc = horner_mul(crc, hb, l4);
       const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
-      if (vb == kSegBytes) {
 #pragma unroll
-        for (int g = 0; g < 8; ++g) crc = crc_step16(crc, row[g], tl);
-      } else if (vb > 0) {
-        const int nw = vb >> 2;
-        const uint32_t* roww = reinterpret_cast<const uint32_t*>(row);
-        for (int w = 0; w < nw; ++w) crc = crc_step4(crc, roww[w], tl);
-        if (vb & 3) {
-          const uint32_t w = roww[nw];
-          for (int b = 0; b < (vb & 3); ++b) crc = crc_step1(crc, (w >> (8 * b)) & 0xFFu, tl);
-        }
-      }
+      for (int g = 0; g < 8; ++g) crc = crc_step16(crc, row[g], tb, l4);
+#endif
       __syncwarp();
     }
 
@@ -196,20 +234,19 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     }
     if (kVerify) pad_bad = __any_sync(full, pad_bad != 0);
 
-    // Fold the full stripes: at level k lane l (l % 2^(k+1) == 0) combines its
-    // group with the one 2^k stripes to the right: shift left group by 2048*2^k B.
-    const uint32_t q = len / kStripeBytes;
-    uint32_t f = ((uint32_t)lane < q) ? crc : 0u;
+    // Fold the lanes: at level k, lane l (l % 2^(k+1) == 0) shifts its group past
+    // the 128*2^k bytes of the group to its right and adds it. The result is the
+    // register of the chunk zero-padded to nrounds*4096 bytes; undo the zp padding
+    // bytes with one multiply by x^(-8 zp).
+    uint32_t f = crc;
 #pragma unroll
     for (int k = 0; k < kFoldLevels; ++k) {
       const uint32_t o = __shfl_down_sync(full, f, 1 << k);
       if ((lane & ((2 << k) - 1)) == 0) f = fold_mul(f, ftab + k * 128) ^ o;
     }
-    const uint32_t rq = __shfl_sync(full, crc, (int)(q & 31u));
     if (lane == 0) {
-      uint32_t t = f;
-      if (len < kChunkBytes) t = gf_mul(t, p.inv_z[kChunkBytes - len]) ^ rq;
-      const uint32_t out = ~t;
+      const uint32_t zp = (uint32_t)nrounds * kRoundBytes - len;
+      const uint32_t out = ~(zp ? gf_mul(f, p.inv_z[zp]) : f);
       if (!kVerify) {
         p.crc[c] = out;
       } else if (out != p.crc[c] || pad_bad) {

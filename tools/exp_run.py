@@ -1,0 +1,39 @@
+"""Time pack / verify kernels (device-resident image) for one library variant.
+CHECL_LIB=<path> python tools/exp_run.py [--config C2] [--reps 10]"""
+import argparse
+import os
+import statistics
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import torch  # noqa: E402
+
+import synth  # noqa: E402
+from paper_conf_ipps_takizawakskk11_b200 import checl  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--config", default="C2")
+ap.add_argument("--reps", type=int, default=10)
+ap.add_argument("--kind", type=int, default=0)
+a = ap.parse_args()
+w = synth.CONFIGS[a.config]()
+ts = [torch.empty(b.size, dtype=torch.uint8, device=0) for b in w.buffers]
+for t, b in zip(ts, w.buffers):
+    checl.debug_fill(t, w.seed, b.stream, a.kind)
+torch.cuda.synchronize()
+ctx = checl.Context()
+hs = [ctx.register(t) for t in ts]
+img = ctx.checkpoint_device(0)
+pk, vf = [], []
+for i in range(a.reps + 2):
+    ctx.checkpoint(0, epoch=i, into=img)
+    tp = ctx.last_timing()["kernel_ms"]
+    ctx.restore(img, 0)
+    tv = ctx.last_timing()["kernel_ms"]
+    if i >= 2:
+        pk.append(tp)
+        vf.append(tv)
+S = w.total_bytes
+p, v = statistics.median(pk), statistics.median(vf)
+print(f"{os.path.basename(os.path.dirname(os.environ.get('CHECL_LIB', 'default/x')))}: pack {p*1e3:.1f} us "
+      f"({2*S/p/1e6:.0f} GB/s 2S), verify {v*1e3:.1f} us ({2*S/v/1e6:.0f} GB/s 2S)")
