@@ -42,6 +42,8 @@ __device__ __forceinline__ uint4 ld_stream_v4(const void* p) {
   return r;
 }
 
+__device__ __forceinline__ void st_stream_v4(void* p, uint4 v) { *reinterpret_cast<uint4*>(p) = v; }
+
 __device__ __forceinline__ uint32_t ld_stream_u32(const void* p) {
   uint32_t r;
   asm("ld.global.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
@@ -185,11 +187,12 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
 
     uint4 v[8];
     auto load_round = [&](int r) {
+      const bool whole = mode == 0 && (uint32_t)(r + 1) * kRoundBytes <= len;  // warp-uniform fast path
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         const uint32_t o = (uint32_t)r * kRoundBytes + (uint32_t)(4 * i + s_lane) * kSegBytes + (uint32_t)g_lane * 16;
-        if (o + 16 <= len)
-          v[i] = ld_granule(src + o, mode);
+        if (whole || o + 16 <= len)
+          v[i] = ld_granule(src + o, whole ? 0 : mode);
         else if (o < len)
           v[i] = ld_partial(src + o, len - o);
         else
@@ -198,12 +201,13 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     };
     load_round(0);
     for (int r = 0; r < nrounds; ++r) {
+      const bool whole = (uint32_t)(r + 1) * kRoundBytes <= len;
 #pragma unroll
       for (int i = 0; i < 8; ++i) {
         const uint32_t o = (uint32_t)r * kRoundBytes + (uint32_t)(4 * i + s_lane) * kSegBytes + (uint32_t)g_lane * 16;
-        if (o < len) {
-          if (!kVerify || o + 16 <= len)
-            *reinterpret_cast<uint4*>(dst + o) = v[i];  // pack: zeros past len are owned padding
+        if (whole || o < len) {
+          if (whole || !kVerify || o + 16 <= len)
+            st_stream_v4(dst + o, v[i]);  // pack: zeros past len are owned padding
           else
             st_partial(dst + o, v[i], len - o);
         }
