@@ -302,7 +302,8 @@ def main():
     tf = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tf):
         try:
-            traffic = json.load(open(tf)).get(a.config, {}).get("dram_bytes_per_launch")
+            t = json.load(open(tf)).get(a.config, {})
+            traffic = t.get("K1" if dom_name.startswith("pack") else "K2", t.get("dram_bytes_per_launch"))
         except Exception:
             traffic = None
     dimg.free()

@@ -58,9 +58,9 @@ class _Report(C.Structure):
 
 
 class _Timing(C.Structure):
-    _fields_ = [("sync_ms", C.c_double), ("plan_ms", C.c_double), ("kernel_ms", C.c_double),
-                ("copy_ms", C.c_double), ("total_ms", C.c_double), ("n_stages", C.c_uint64),
-                ("n_kernels", C.c_uint64)]
+    _fields_ = [("sync_ms", C.c_double), ("plan_ms", C.c_double), ("alloc_ms", C.c_double),
+                ("kernel_ms", C.c_double), ("copy_ms", C.c_double), ("commit_ms", C.c_double),
+                ("total_ms", C.c_double), ("n_stages", C.c_uint64), ("n_kernels", C.c_uint64)]
 
 
 def _load() -> C.CDLL:

@@ -276,6 +276,7 @@ struct Arena {  // one allocation holding every buffer of one restore (payload l
   int device;
   void* stream;
   void* base = nullptr;
+  uint64_t bytes = 0;
   ~Arena() {
     if (!base) return;
     if (alloc.free)
@@ -374,7 +375,12 @@ struct checl_ctx {
   mutable std::mutex mu;
   checl_allocator alloc{nullptr, nullptr, nullptr};
   std::map<uint64_t, Entry> entries;                  // ascending handle = database order (L19)
-  std::map<uintptr_t, uint64_t> by_addr[kMaxDevices];  // start address -> handle (overlap checks)
+  // live address ranges per device for overlap checks: user registrations (handle)
+  // and restore arenas (handle 0, one range per arena)
+  struct Range {
+    uint64_t bytes, handle;
+  };
+  std::map<uintptr_t, Range> by_addr[kMaxDevices];
   uint64_t version[kMaxDevices] = {};
   uint64_t next_id = 1;
   std::atomic<bool> busy{false};
@@ -753,7 +759,9 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
     ck(cudaStreamSynchronize(ds.copy));
   }
   // a5: header, manifest and meta CRC (the CRC table has landed)
+  const double tf = now_ms();
   finalize_meta(img->host_mut, P, epoch);
+  tm.commit_ms = now_ms() - tf;
   img->image_bytes = P.image_bytes;
   img->payload_off = P.payload_off;
   float cms = 0;
@@ -800,32 +808,35 @@ bool ensure_peer(int dev, int peer) {
 // Swaps every handle of the image to its new buffer (L15); frees library-owned
 // buffers previously bound to those handles (after their devices are idle).
 void commit(checl_ctx* ctx, const Parsed& P, int device, const std::shared_ptr<Arena>& arena) {
-  std::vector<std::shared_ptr<Arena>> dropped;
+  std::vector<std::shared_ptr<Arena>> dropped;  // distinct arenas that lost handles
   {
     std::lock_guard<std::mutex> lk(ctx->mu);
+    if (arena->base) ctx->by_addr[device][reinterpret_cast<uintptr_t>(arena->base)] = {arena->bytes, 0};
     uint64_t max_h = 0;
     for (const BufRec& b : P.bufs) {
-      auto it = ctx->entries.find(b.handle);
-      if (it != ctx->entries.end()) {
-        Entry& old = it->second;
-        if (old.bytes) ctx->by_addr[old.device].erase(reinterpret_cast<uintptr_t>(old.ptr));
-        ctx->version[old.device]++;
-        if (old.arena) dropped.push_back(old.arena);
-        ctx->entries.erase(it);
+      auto ins = ctx->entries.try_emplace(b.handle);
+      Entry& e = ins.first->second;
+      if (!ins.second) {  // rebind an existing handle in place
+        if (!e.arena && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
+        ctx->version[e.device]++;
+        if (e.arena) {
+          if (dropped.empty() || dropped.back().get() != e.arena.get())
+            dropped.push_back(std::move(e.arena));
+          e.arena.reset();
+        }
       }
-      Entry e;
       e.device = device;
       e.ptr = b.size ? static_cast<uint8_t*>(arena->base) + b.off : nullptr;
       e.bytes = b.size;
       e.flags = b.flags;
       e.owned = true;
       e.arena = b.size ? arena : nullptr;
-      if (b.size) ctx->by_addr[device][reinterpret_cast<uintptr_t>(e.ptr)] = b.handle;
-      ctx->entries.emplace(b.handle, std::move(e));
       max_h = std::max(max_h, b.handle);
     }
     ctx->version[device]++;
     ctx->next_id = std::max(ctx->next_id, max_h + 1);
+    for (auto& a : dropped)
+      if (a.use_count() == 1 && a->base) ctx->by_addr[a->device].erase(reinterpret_cast<uintptr_t>(a->base));
   }
   // arenas whose last handle moved away are freed here, outside the lock, once
   // their device is idle
@@ -866,6 +877,8 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   arena->alloc = ctx->alloc;
   arena->device = device;
   arena->stream = stream;
+  const double ta = now_ms();
+  arena->bytes = P.L.payload_bytes;
   if (P.L.payload_bytes) {
     if (ctx->alloc.alloc)
       arena->base = ctx->alloc.alloc(P.L.payload_bytes, device, stream, ctx->alloc.user);
@@ -875,6 +888,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     }
     if (!arena->base) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
   }
+  tm.alloc_ms = now_ms() - ta;
   const uint64_t nch = P.L.n_chunks;
   ds.h_desc.ensure(std::max<uint64_t>(nch, 1));
   uint8_t* abase = static_cast<uint8_t*>(arena->base);
@@ -962,7 +976,9 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   }
   // r5: rebind every handle (all-or-nothing)
   (void)in_migrate;
+  const double tc = now_ms();
   commit(ctx, P, device, arena);
+  tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
   ctx->last = tm;
   return CHECL_SUCCESS;
@@ -1040,12 +1056,11 @@ checl_status checl_register_buffer(checl_ctx* ctx, int device, void* dev_ptr, si
     std::lock_guard<std::mutex> lk(ctx->mu);
     if (bytes) {
       auto& m = ctx->by_addr[device];
-      auto it = m.upper_bound(lo);  // first start > lo
+      auto it = m.upper_bound(lo);  // first range starting after lo
       if (it != m.end() && it->first < lo + bytes) return CHECL_ERR_INVALID_VALUE;
       if (it != m.begin()) {
-        --it;  // start <= lo
-        const Entry& e = ctx->entries.at(it->second);
-        if (it->first + e.bytes > lo) return CHECL_ERR_INVALID_VALUE;
+        --it;  // range starting at or before lo
+        if (it->first + it->second.bytes > lo) return CHECL_ERR_INVALID_VALUE;
       }
     }
     const uint64_t h = ctx->next_id++;
@@ -1056,7 +1071,7 @@ checl_status checl_register_buffer(checl_ctx* ctx, int device, void* dev_ptr, si
     e.flags = flags;
     e.owned = false;
     ctx->entries.emplace(h, std::move(e));
-    if (bytes) ctx->by_addr[device][lo] = h;
+    if (bytes) ctx->by_addr[device][lo] = {bytes, h};
     ctx->version[device]++;
     *out = h;
     return CHECL_SUCCESS;
@@ -1074,8 +1089,10 @@ checl_status checl_release(checl_ctx* ctx, checl_handle h) {
       if (it == ctx->entries.end()) return CHECL_ERR_INVALID_HANDLE;
       Entry& e = it->second;
       dev = e.device;
-      if (e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
+      if (!e.arena && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
       drop = std::move(e.arena);
+      if (drop && drop.use_count() == 1 && drop->base)
+        ctx->by_addr[drop->device].erase(reinterpret_cast<uintptr_t>(drop->base));
       ctx->version[e.device]++;
       ctx->entries.erase(it);
     }
