@@ -41,6 +41,7 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--c4-scale", type=float, default=1.0)
+    ap.add_argument("--c5-large", action="store_true", help="C5 with 16 x 1 GiB instead of the C2 set")
     return ap.parse_args()
 
 
@@ -200,10 +201,79 @@ def run_reference(a):
     }))
 
 
+def run_migration(a):
+    """configs[4] (C5): every rank migrates its buffers GPU i -> GPU (i+1) mod n
+    (m1-m3: K1 into an HBM image on i, K2 on the destination reading it over NVLink
+    peer memory). With one GPU the destination is the source (no NVLink crossing)."""
+    import torch
+    import torch.distributed as dist
+    import synth
+    from paper_conf_ipps_takizawakskk11_b200 import checl
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    dev = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(dev)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+    ndev = torch.cuda.device_count()
+    w = synth.c5_migration(large=a.c5_large)
+    tensors = [torch.empty(b.size, dtype=torch.uint8, device=dev) for b in w.buffers]
+    for t, b in zip(tensors, w.buffers):
+        checl.debug_fill(t, w.seed, b.stream)
+    torch.cuda.synchronize()
+    ctx = checl.Context()
+    handles = [ctx.register(t) for t in tensors]
+    S = w.total_bytes
+    cur = dev
+    for _ in range(a.warmup):
+        nxt = (cur + 1) % ndev if world > 1 else cur
+        ctx.migrate(cur, nxt)
+        cur = nxt
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    timings = []
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record()
+    for _ in range(a.steps):
+        nxt = (cur + 1) % ndev if world > 1 else cur
+        ctx.migrate(cur, nxt)
+        timings.append(ctx.last_timing())
+        cur = nxt
+    e1.record()
+    e1.synchronize()
+    ms = e0.elapsed_time(e1)
+    n_diff = 0
+    for h, t in zip(handles, tensors):
+        ptr, nb, d = ctx.translate(h)
+        if d == dev:
+            n_diff += checl.debug_compare(dev, ptr, t.data_ptr(), nb)
+    if world > 1:
+        t = torch.tensor([ms], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms = float(t.item())
+    if rank == 0:
+        kern = statistics.mean(t["kernel_ms"] for t in timings)
+        print(json.dumps({
+            "metric": "in-box migration GB/s (checl_migrate, GPU i -> GPU (i+1) mod n)", "value": S * world * a.steps / (ms * 1e-3) / 1e9,
+            "unit": "GB/s", "n_gpus": world, "steps": a.steps, "warmup": a.warmup, "ms_per_step": ms / a.steps,
+            "config": {"workload": w.name, "payload_bytes_per_gpu": S, "n_buffers": len(w.buffers),
+                       "route": "same GPU (1 device)" if world == 1 else "NVLink peer read"},
+            "kernel_ms_per_step": kern, "kernels_2S_GBs": 4 * S / (kern * 1e-3) / 1e9,
+            "verified": n_diff == 0, "last_timing": timings[-1]}))
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
 def main():
     a = parse()
     if a.impl == "reference":
         run_reference(a)
+        return
+    if a.config == "C5":
+        run_migration(a)
         return
     import torch
     import torch.distributed as dist

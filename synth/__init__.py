@@ -49,8 +49,19 @@ def _mix64_np(z: np.ndarray) -> np.ndarray:
     return z ^ (z >> np.uint64(31))
 
 
-def fill_bytes(size: int, seed: int, stream: int, kind: str = "random", out: np.ndarray | None = None) -> np.ndarray:
-    """Host copy of the bytes the device fill kernel writes (uint8[size])."""
+def fill_slice(offset: int, length: int, seed: int, stream: int, kind: str = "random") -> np.ndarray:
+    """Bytes [offset, offset + length) of a buffer filled by fill_bytes (counter-based:
+    no need to generate the prefix)."""
+    w0 = offset // 8
+    head = offset - 8 * w0
+    b = fill_bytes(head + length, seed, stream, kind, word0=w0)
+    return b[head:head + length]
+
+
+def fill_bytes(size: int, seed: int, stream: int, kind: str = "random", out: np.ndarray | None = None,
+               word0: int = 0) -> np.ndarray:
+    """Host copy of the bytes the device fill kernel writes (uint8[size]); with
+    word0 > 0, the bytes starting at word word0 of the buffer."""
     if out is None:
         out = np.empty(size, dtype=np.uint8)
     if size == 0:
@@ -64,7 +75,7 @@ def fill_bytes(size: int, seed: int, stream: int, kind: str = "random", out: np.
     for w0 in range(0, nwords, step):
         w1 = min(nwords, w0 + step)
         with np.errstate(over="ignore"):
-            st = key + (np.arange(w0 + 1, w1 + 1, dtype=np.uint64) * np.uint64(GOLDEN))
+            st = key + (np.arange(word0 + w0 + 1, word0 + w1 + 1, dtype=np.uint64) * np.uint64(GOLDEN))
             words = _mix64_np(st)
         if kind == "float":
             lo = (words & np.uint64(0xFFFFFFFF)).astype(np.uint32) >> np.uint32(8)

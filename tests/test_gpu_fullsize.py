@@ -1,0 +1,72 @@
+"""-m gpu: configs[3] (C4, SHOC-MD-shaped rank, 64 GiB) at full size on one B200.
+
+Checkpoint to a pinned host image, then restore into re-created buffers; the image
+header/manifest/CRC table are checked against the oracle's layout and meta CRC, and
+sampled chunks (random ones plus every buffer's short tail chunk) against the
+oracle's CRC32C and the synth generator's bytes; restored buffers are compared on
+the same samples (full sizes are checked on samples
+the oracle computes one by one).
+"""
+import struct
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import oracle as O
+
+pytestmark = pytest.mark.gpu
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+from paper_conf_ipps_takizawakskk11_b200 import checl  # noqa: E402
+
+
+def test_c4_md_rank_full_size_sampled():
+    w = synth.c4_md_rank(0)
+    S = w.total_bytes
+    free, _ = torch.cuda.mem_get_info(0)
+    if free < S + (8 << 30):
+        pytest.skip(f"needs {S >> 30} GiB free on the device")
+    ctx = checl.Context()
+    tensors = [torch.empty(b.size, dtype=torch.uint8, device=0) for b in w.buffers]
+    for t, b in zip(tensors, w.buffers):
+        checl.debug_fill(t, w.seed, b.stream, checl.FILL_FLOAT if b.name != "md.neigh" else checl.FILL_RANDOM)
+    kinds = ["float" if b.name != "md.neigh" else "random" for b in w.buffers]
+    torch.cuda.synchronize()
+    handles = [ctx.register(t, 0x40 + i) for i, t in enumerate(tensors)]
+    img = ctx.checkpoint(0, epoch=4)
+    got = img.view()
+    L = O.layout(list(zip(handles, [b.size for b in w.buffers])))
+    assert got.size == L["image_bytes"] and L["payload_bytes"] == S + 288  # two 144-B alignment gaps
+    assert L["n_chunks"] == 1048578
+    st, rep = O.validate(got)  # header, manifest, meta CRC over the 4 MiB CRC table
+    assert st == 0 and rep["n_chunks"] == 1048578
+    recs = [struct.unpack_from("<QQQQIiQ", got, 128 + 48 * i) for i in range(3)]
+    crcs = np.frombuffer(got, dtype="<u4", count=L["n_chunks"], offset=L["crc_off"])
+    rng = np.random.default_rng(44)
+    samples = []
+    for bi, (h, size, off, first, fl, dv, _) in enumerate(recs):
+        nch = (size + 65535) // 65536
+        ks = list(rng.integers(0, nch, 12)) + [nch - 1]
+        samples += [(bi, int(k)) for k in ks]
+    for bi, k in samples:
+        h, size, off, first, fl, dv, _ = recs[bi]
+        lo = k * 65536
+        n = min(65536, size - lo)
+        data = synth.fill_slice(lo, n, w.seed, w.buffers[bi].stream, kinds[bi])
+        p0 = L["payload_off"] + off + lo
+        assert np.array_equal(got[p0:p0 + n], data), (bi, k)
+        assert int(crcs[first + k]) == O.crc32c(data), (bi, k)
+    del tensors
+    torch.cuda.empty_cache()
+    rep = ctx.restore(img, 0)
+    assert rep.n_bad_chunks == 0 and rep.n_chunks == 1048578
+    for bi, k in samples:
+        lo = k * 65536
+        n = min(65536, w.buffers[bi].size - lo)
+        back = ctx.tensor(handles[bi])[lo:lo + n].cpu().numpy()
+        assert np.array_equal(back, synth.fill_slice(lo, n, w.seed, w.buffers[bi].stream, kinds[bi])), (bi, k)
+    img.free()
+    ctx.close()

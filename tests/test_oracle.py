@@ -265,3 +265,10 @@ def test_invalid_registries_rejected():
         O.checkpoint([O.Entry(0, np.zeros(3, np.uint8))])
     with pytest.raises(ValueError):
         O.checkpoint([O.Entry(4, np.zeros(3, np.uint8)), O.Entry(4, np.zeros(1, np.uint8))])
+
+
+def test_synth_slices_match_whole_buffer():
+    import synth
+    full = synth.fill_bytes(70001, 9, 4)
+    for off, n in [(0, 1), (7, 33), (8, 8), (12345, 999), (69990, 11)]:
+        assert np.array_equal(synth.fill_slice(off, n, 9, 4), full[off:off + n])
