@@ -31,6 +31,8 @@ cudaError_t launch_snapshot(bool verify, const LaunchParams& p, int n_sms, cudaS
 cudaError_t launch_fill(uint8_t* ptr, uint64_t bytes, uint64_t key, int kind, int n_sms, cudaStream_t s);
 cudaError_t launch_compare(const uint8_t* a, const uint8_t* b, uint64_t bytes, unsigned long long* n_diff, int n_sms,
                            cudaStream_t s);
+cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload_bytes, uint64_t n_chunks,
+                          ChunkDesc* out, int n_sms, cudaStream_t s);
 uint32_t host_crc32c_update(uint32_t crc, const void* data, size_t n);
 uint32_t host_crc32c(const void* data, size_t n);
 }  // namespace checl
@@ -204,10 +206,11 @@ struct Plan {
   size_t slot_bytes = 0;
   std::vector<BufRec> bufs;
   uint64_t n_chunks = 0, payload_bytes = 0, crc_off = 0, payload_off = 0, image_bytes = 0;
-  std::vector<ChunkDesc> desc;
+  std::vector<BufferRecord> recs;
   std::vector<Stage> stages;
   std::vector<uint8_t> meta;  // header (meta_crc = 0, epoch = 0) + manifest
   DevBuf<ChunkDesc> d_desc;
+  DevBuf<BufferRecord> d_recs;
 };
 
 struct DevState {
@@ -218,9 +221,10 @@ struct DevState {
   uint32_t n_slots = 0;
   DevBuf<uint32_t> inv_z, crc_scratch;
   DevBuf<ChunkDesc> desc_scratch;
+  DevBuf<BufferRecord> recs_scratch;
   DevBuf<unsigned long long> status;
   PinnedBuf<unsigned long long> h_status;
-  PinnedBuf<ChunkDesc> h_desc;
+  PinnedBuf<BufferRecord> h_recs;
   EventPool events;
   Plan plan;
   uint32_t fold[kFoldLevels];
@@ -256,10 +260,12 @@ struct DevState {
     inv_z.release();
     crc_scratch.release();
     desc_scratch.release();
+    recs_scratch.release();
+    plan.d_recs.release();
     status.release();
     plan.d_desc.release();
     h_status.release();
-    h_desc.release();
+    h_recs.release();
     for (auto e : events.ev) cudaEventDestroy(e);
     events.ev.clear();
     if (compute) cudaStreamDestroy(compute);
@@ -388,6 +394,7 @@ struct checl_ctx {
   size_t slot_bytes = kDefaultSlotBytes;
   uint32_t n_slots = 2;
   checl_timing last{};
+  checl_image* mig_img[kMaxDevices] = {};  // migration images, reused (HBM of the source)
 
   DevState& dev(int d) {
     if (!devs[d]) {
@@ -455,46 +462,56 @@ Layout layout_records(std::vector<BufRec>& bufs) {
   return L;
 }
 
-// Flat chunk list; ptr(b) is the device address chunk k of record b is read from
-// (pack) or written to (restore).
+// Per-buffer records for the GPU chunk-list expansion (expand_plan_kernel);
+// ptr(b) is the device address of record b (pack: source; restore: destination).
 template <typename PtrOf>
-void build_desc(const std::vector<BufRec>& bufs, uint64_t payload_bytes, PtrOf ptr_of, ChunkDesc* out) {
-  size_t c = 0;
-  for (size_t b = 0; b < bufs.size(); ++b) {
-    const uint64_t nch = chunks_of(bufs[b].size);
-    const uint64_t pad_end = b + 1 < bufs.size() ? bufs[b + 1].off : payload_bytes;
-    uint8_t* base = ptr_of(b);
-    for (uint64_t k = 0; k < nch; ++k) {
-      const uint64_t lo = k * kChunkBytes;
-      const uint32_t len = (uint32_t)std::min<uint64_t>(kChunkBytes, bufs[b].size - lo);
-      const uint32_t pad = k + 1 == nch ? (uint32_t)(pad_end - (bufs[b].off + bufs[b].size)) : 0u;
-      ChunkDesc d;
-      d.ptr = reinterpret_cast<uint64_t>(base + lo);
-      d.img_off_256 = (uint32_t)((bufs[b].off + lo) / kBufferAlign);
-      d.len_pad = make_len_pad(len, pad);
-      out[c++] = d;
-    }
-  }
+void build_records(const std::vector<BufRec>& bufs, PtrOf ptr_of, BufferRecord* out) {
+  for (size_t b = 0; b < bufs.size(); ++b)
+    out[b] = BufferRecord{reinterpret_cast<uint64_t>(ptr_of(b)), bufs[b].size, bufs[b].off, bufs[b].first_chunk};
 }
 
-// Consecutive chunks whose image span fits in one staging slot.
-std::vector<Stage> build_stages(const ChunkDesc* desc, uint64_t n, size_t slot_bytes) {
+// Stages = maximal runs of consecutive chunks whose image span (chunk bytes plus
+// owned padding) fits in one staging slot; a stage always takes at least one
+// chunk. Computed per buffer in O(#buffers + #stages): inside a buffer, chunk j
+// (not the last) ends at off + (j+1)*64K, the last one at the next buffer's offset.
+std::vector<Stage> build_stages(const std::vector<BufRec>& bufs, uint64_t payload_bytes, size_t slot) {
   std::vector<Stage> st;
-  uint64_t c = 0;
-  while (c < n) {
-    Stage s;
-    s.c0 = c;
-    s.img_lo = (uint64_t)desc[c].img_off_256 * kBufferAlign;
-    s.img_hi = s.img_lo;
-    while (c < n) {
-      const uint64_t hi = (uint64_t)desc[c].img_off_256 * kBufferAlign + desc_len(desc[c]) + desc_pad(desc[c]);
-      if (c > s.c0 && hi - s.img_lo > slot_bytes) break;
-      s.img_hi = hi;
-      ++c;
+  bool open = false;
+  Stage cur{0, 0, 0, 0};
+  for (size_t b = 0; b < bufs.size(); ++b) {
+    const uint64_t nch = chunks_of(bufs[b].size);
+    if (!nch) continue;
+    const uint64_t off = bufs[b].off, first = bufs[b].first_chunk;
+    const uint64_t end_last = b + 1 < bufs.size() ? bufs[b + 1].off : payload_bytes;
+    uint64_t j = 0;
+    while (j < nch) {
+      if (!open) {
+        cur = Stage{first + j, first + j, off + j * kChunkBytes, off + j * kChunkBytes};
+        open = true;
+      }
+      if (end_last - cur.img_lo <= slot) {  // the rest of the buffer fits
+        cur.c1 = first + nch;
+        cur.img_hi = end_last;
+        j = nch;
+        continue;
+      }
+      // non-last chunks jj < fit end inside the slot: off + fit*64K <= img_lo + slot
+      uint64_t fit = cur.img_lo + slot >= off ? (cur.img_lo + slot - off) / kChunkBytes : 0;
+      fit = std::min(fit, nch - 1);
+      if (fit > j) {
+        cur.c1 = first + fit;
+        cur.img_hi = off + fit * kChunkBytes;
+        j = fit;
+      } else if (cur.c1 == cur.c0) {  // empty stage: take one chunk regardless
+        cur.c1 = first + j + 1;
+        cur.img_hi = j + 1 < nch ? off + (j + 1) * kChunkBytes : end_last;
+        ++j;
+      }
+      st.push_back(cur);
+      open = false;
     }
-    s.c1 = c;
-    st.push_back(s);
   }
+  if (open) st.push_back(cur);
   return st;
 }
 
@@ -621,14 +638,21 @@ Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
   P.crc_off = L.crc_off;
   P.payload_off = L.payload_off;
   P.image_bytes = L.image_bytes;
-  P.desc.resize(L.n_chunks);
-  build_desc(P.bufs, L.payload_bytes, [&](size_t b) { return P.bufs[b].ptr; }, P.desc.data());
-  P.stages = build_stages(P.desc.data(), L.n_chunks, ctx->slot_bytes);
+  P.recs.resize(P.bufs.size());
+  build_records(P.bufs, [&](size_t b) { return P.bufs[b].ptr; }, P.recs.data());
+  P.stages = build_stages(P.bufs, L.payload_bytes, ctx->slot_bytes);
   P.meta.assign(L.crc_off, 0);
   write_header(P.meta.data(), L, P.bufs.size(), device, 0);
   write_manifest(P.meta.data() + kHeaderBytes, P.bufs, device);
-  P.d_desc.ensure(L.n_chunks);
-  if (L.n_chunks) ck(cudaMemcpy(P.d_desc.p, P.desc.data(), L.n_chunks * sizeof(ChunkDesc), cudaMemcpyHostToDevice));
+  P.d_desc.ensure(std::max<uint64_t>(L.n_chunks, 1));
+  P.d_recs.ensure(std::max<size_t>(P.recs.size(), 1));
+  if (L.n_chunks) {  // chunk list expanded on the GPU from one record per buffer
+    ck(cudaMemcpyAsync(P.d_recs.p, P.recs.data(), P.recs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
+                       ds.compute));
+    ck(launch_expand(P.d_recs.p, (uint32_t)P.recs.size(), L.payload_bytes, L.n_chunks, P.d_desc.p, ds.n_sms,
+                     ds.compute));
+    ck(cudaStreamSynchronize(ds.compute));  // P.recs may be rebuilt by the next plan
+  }
   P.version = ctx->version[device];
   P.slot_bytes = ctx->slot_bytes;
   return P;
@@ -890,17 +914,23 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   }
   tm.alloc_ms = now_ms() - ta;
   const uint64_t nch = P.L.n_chunks;
-  ds.h_desc.ensure(std::max<uint64_t>(nch, 1));
+  ds.h_recs.ensure(std::max<size_t>(P.bufs.size(), 1));
   uint8_t* abase = static_cast<uint8_t*>(arena->base);
-  build_desc(P.bufs, P.L.payload_bytes, [&](size_t b) { return abase + P.bufs[b].off; }, ds.h_desc.p);
+  build_records(P.bufs, [&](size_t b) { return abase + P.bufs[b].off; }, ds.h_recs.p);
   ds.desc_scratch.ensure(std::max<uint64_t>(nch, 1));
+  ds.recs_scratch.ensure(std::max<size_t>(P.bufs.size(), 1));
   LaunchParams lp = base_params(ds);
   lp.desc = ds.desc_scratch.p;
   tm.plan_ms = now_ms() - tp;
 
   cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
   ck(cudaEventRecord(c_begin, ds.copy));
-  if (nch) ck(cudaMemcpyAsync(ds.desc_scratch.p, ds.h_desc.p, nch * sizeof(ChunkDesc), cudaMemcpyHostToDevice, ds.copy));
+  if (nch) {  // chunk list expanded on the GPU (compute stream, ahead of the verify launches)
+    ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, P.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
+                       ds.compute));
+    ck(launch_expand(ds.recs_scratch.p, (uint32_t)P.bufs.size(), P.L.payload_bytes, nch, ds.desc_scratch.p, ds.n_sms,
+                     ds.compute));
+  }
   ds.h_status.p[0] = ~0ull;
   ds.h_status.p[1] = 0;
   ck(cudaMemcpyAsync(ds.status.p, ds.h_status.p, 16, cudaMemcpyHostToDevice, ds.copy));
@@ -934,7 +964,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     ds.crc_scratch.ensure(std::max<uint64_t>(nch, 1));
     if (nch) ck(cudaMemcpyAsync(ds.crc_scratch.p, img->host + P.L.crc_off, 4 * nch, cudaMemcpyHostToDevice, ds.copy));
     lp.crc = ds.crc_scratch.p;
-    std::vector<Stage> stages = build_stages(ds.h_desc.p, nch, ctx->slot_bytes);
+    std::vector<Stage> stages = build_stages(P.bufs, P.L.payload_bytes, ctx->slot_bytes);
     std::vector<cudaEvent_t> filled(ds.n_slots), verified(ds.n_slots);
     for (uint32_t i = 0; i < ds.n_slots; ++i) {
       filled[i] = ds.events.get();
@@ -1029,6 +1059,14 @@ checl_status checl_destroy(checl_ctx* ctx) {
         d->destroy();
         delete d;
         d = nullptr;
+      }
+    }
+    for (auto*& m : ctx->mig_img) {
+      if (m) {
+        m->free_device();
+        m->free_host();
+        delete m;
+        m = nullptr;
       }
     }
     delete ctx;
@@ -1253,12 +1291,11 @@ checl_status checl_migrate(checl_ctx* ctx, int src_device, int dst_device, void*
   if (!b.ok) return CHECL_ERR_BUSY;
   return guarded([&]() -> checl_status {
     const double t0 = now_ms();
-    checl_image img;
+    if (!ctx->mig_img[src_device]) ctx->mig_img[src_device] = new checl_image();
+    checl_image& img = *ctx->mig_img[src_device];
     checl_status st = do_checkpoint(ctx, src_device, cuda_stream, 0, &img, true);
     checl_timing ck_t = ctx->last;
     if (st == CHECL_SUCCESS) st = do_restore(ctx, &img, dst_device, cuda_stream, rep, true);
-    img.free_device();
-    img.free_host();
     checl_timing& t = ctx->last;
     t.sync_ms += ck_t.sync_ms;
     t.plan_ms += ck_t.plan_ms;

@@ -38,6 +38,14 @@ struct ChunkDesc {
 };
 static_assert(sizeof(ChunkDesc) == 16, "ChunkDesc is 16 bytes");
 
+// One buffer of a plan (32 bytes); the GPU expands records into ChunkDescs.
+// ptr = the buffer's device address (pack: source; restore: destination),
+// off = payload offset (256-aligned), first_chunk = global index of its chunk 0.
+struct BufferRecord {
+  uint64_t ptr, size, off, first_chunk;
+};
+static_assert(sizeof(BufferRecord) == 32, "BufferRecord is 32 bytes");
+
 CHECL_HD uint32_t desc_len(const ChunkDesc& d) { return d.len_pad & 0x1FFFFu; }
 CHECL_HD uint32_t desc_pad(const ChunkDesc& d) { return d.len_pad >> 24; }
 CHECL_HD uint32_t make_len_pad(uint32_t len, uint32_t pad) { return len | (pad << 24); }

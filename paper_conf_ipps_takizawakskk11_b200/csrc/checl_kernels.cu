@@ -312,7 +312,45 @@ __global__ void compare_kernel(const uint8_t* a, const uint8_t* b, uint64_t byte
   if (local) atomicAdd(n_diff, local);
 }
 
+// ---- plan expansion: buffer records -> flat chunk list (a2 / r2) -------------
+// One thread per chunk: find the buffer (largest record index whose first_chunk
+// <= c: zero-size records share first_chunk with the next record, so the search
+// lands on the non-empty one), then emit {ptr + k*64K, off + k*64K, len, pad}.
+// The pad of a buffer's last chunk runs to the next record's offset (or to
+// payload_bytes): FORMAT.md "Chunk ownership of padding".
+__global__ void expand_plan_kernel(const BufferRecord* __restrict__ recs, uint32_t n, uint64_t payload_bytes,
+                                   uint64_t n_chunks, ChunkDesc* __restrict__ out) {
+  for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < n_chunks;
+       c += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t lo = 0, hi = n - 1;
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi + 1) >> 1;
+      if (recs[mid].first_chunk <= c) lo = mid; else hi = mid - 1;
+    }
+    const BufferRecord r = recs[lo];
+    const uint64_t k = c - r.first_chunk, base = k * kChunkBytes;
+    const uint64_t nch = (r.size + kChunkBytes - 1) / kChunkBytes;
+    const uint32_t len = (uint32_t)(r.size - base < kChunkBytes ? r.size - base : kChunkBytes);
+    uint32_t pad = 0;
+    if (k + 1 == nch) pad = (uint32_t)((lo + 1 < n ? recs[lo + 1].off : payload_bytes) - (r.off + r.size));
+    ChunkDesc d;
+    d.ptr = r.ptr + base;
+    d.img_off_256 = (uint32_t)((r.off + base) / kBufferAlign);
+    d.len_pad = make_len_pad(len, pad);
+    out[c] = d;
+  }
+}
+
 // ---- launchers (called from checl_engine.cpp) --------------------------------
+
+cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload_bytes, uint64_t n_chunks,
+                          ChunkDesc* out, int n_sms, cudaStream_t s) {
+  if (n_chunks == 0) return cudaSuccess;
+  uint64_t blocks = (n_chunks + 255) / 256;
+  if (blocks > (uint64_t)n_sms * 8) blocks = (uint64_t)n_sms * 8;
+  expand_plan_kernel<<<(unsigned)blocks, 256, 0, s>>>(recs, n, payload_bytes, n_chunks, out);
+  return cudaGetLastError();
+}
 
 size_t snapshot_smem_bytes() { return kSmemBytes; }
 
