@@ -663,7 +663,8 @@ LaunchParams base_params(DevState& ds) {
   p.inv_z = ds.inv_z.p;
   p.status = ds.status.p;
   for (int k = 0; k < kFoldLevels; ++k) p.fold[k] = ds.fold[k];
-  p.horner = gf_x8n(kRoundBytes - kSegBytes);
+  p.horner = gf_x8n(kRoundBytes - kSegBytes / kChains);
+  p.chain_shift = gf_x8n(kSegBytes / kChains);
   return p;
 }
 

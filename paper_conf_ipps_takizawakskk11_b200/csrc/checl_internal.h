@@ -100,7 +100,12 @@ constexpr int kRowPitch = kSegBytes + 16;        // padded smem row: conflict-fr
 #endif
 constexpr int kWarpsPerCta = CHECL_WARPS;
 constexpr int kThreadsPerCta = kWarpsPerCta * 32;
-constexpr int kFoldLevels = 5;                   // log2(32 stripes)
+constexpr int kFoldLevels = 5;
+#ifndef CHECL_CHAINS
+#define CHECL_CHAINS 1
+#endif
+constexpr int kChains = CHECL_CHAINS;  // independent CRC chains per lane per segment (ILP)
+static_assert(kChains == 1 || kChains == 2 || kChains == 4 || kChains == 8, "chains divide the 8 granules");
 
 // Parameters of one pack (checkpoint) or verify (restore) launch over the chunk
 // range [c0, c1) of `desc`. Payload byte o of the image lives at
@@ -114,7 +119,8 @@ struct LaunchParams {
   const uint32_t* inv_z;    // kRoundBytes entries, x^(-8z) mod P
   unsigned long long* status;  // verify: [0] = first bad chunk (atomicMin), [1] = bad count
   uint32_t fold[kFoldLevels];  // x^(8 * 128 * 2^k) mod P
-  uint32_t horner;             // x^(8 * (kRoundBytes - kSegBytes)) mod P
+  uint32_t horner;             // x^(8 * (kRoundBytes - kSegBytes / kChains)) mod P
+  uint32_t chain_shift;        // x^(8 * kSegBytes / kChains) mod P
 };
 
 }  // namespace checl

@@ -183,45 +183,72 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     uint8_t* dst = kVerify ? reinterpret_cast<uint8_t*>(d.ptr) : img;
     const int mode = kVerify ? 0 : ((d.ptr & 15u) == 0 ? 0 : ((d.ptr & 3u) == 0 ? 1 : 2));
     const int nrounds = (int)((len + kRoundBytes - 1) / kRoundBytes);
-    uint32_t crc = lane == 0 ? 0xFFFFFFFFu : 0u;
+    uint32_t ch[kChains];
+#pragma unroll
+    for (int c = 0; c < kChains; ++c) ch[c] = (lane == 0 && c == 0) ? 0xFFFFFFFFu : 0u;
 
     uint4 v[8];
+    // lane's byte offset of granule i in round r: r*4096 + (4i + l/8)*128 + (l%8)*16
+    const uint32_t lane_off = (uint32_t)s_lane * kSegBytes + (uint32_t)g_lane * 16;
     auto load_round = [&](int r) {
-      const bool whole = mode == 0 && (uint32_t)(r + 1) * kRoundBytes <= len;  // warp-uniform fast path
+      const uint32_t base = (uint32_t)r * kRoundBytes + lane_off;
+      if (mode == 0 && (uint32_t)(r + 1) * kRoundBytes <= len) {  // warp-uniform fast path
+        const uint8_t* s = src + base;
 #pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        const uint32_t o = (uint32_t)r * kRoundBytes + (uint32_t)(4 * i + s_lane) * kSegBytes + (uint32_t)g_lane * 16;
-        if (whole || o + 16 <= len)
-          v[i] = ld_granule(src + o, whole ? 0 : mode);
-        else if (o < len)
-          v[i] = ld_partial(src + o, len - o);
-        else
-          v[i] = make_uint4(0u, 0u, 0u, 0u);  // past the chunk: CRC'd as zeros, corrected below
+        for (int i = 0; i < 8; ++i) v[i] = ld_stream_v4(s + i * 4 * kSegBytes);
+      } else {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
+          if (o + 16 <= len)
+            v[i] = ld_granule(src + o, mode);
+          else if (o < len)
+            v[i] = ld_partial(src + o, len - o);
+          else
+            v[i] = make_uint4(0u, 0u, 0u, 0u);  // past the chunk: CRC'd as zeros, corrected below
+        }
       }
     };
+    uint8_t* tile_w = stage + s_lane * kRowPitch + g_lane * 16;  // this lane's slot, instruction 0
     load_round(0);
     for (int r = 0; r < nrounds; ++r) {
-      const bool whole = (uint32_t)(r + 1) * kRoundBytes <= len;
+      const uint32_t base = (uint32_t)r * kRoundBytes + lane_off;
+      if ((uint32_t)(r + 1) * kRoundBytes <= len) {  // warp-uniform fast path
+        uint8_t* d = dst + base;
 #pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        const uint32_t o = (uint32_t)r * kRoundBytes + (uint32_t)(4 * i + s_lane) * kSegBytes + (uint32_t)g_lane * 16;
-        if (whole || o < len) {
-          if (whole || !kVerify || o + 16 <= len)
-            st_stream_v4(dst + o, v[i]);  // pack: zeros past len are owned padding
-          else
-            st_partial(dst + o, v[i], len - o);
+        for (int i = 0; i < 8; ++i) {
+          st_stream_v4(d + i * 4 * kSegBytes, v[i]);
+          *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
         }
-        *reinterpret_cast<uint4*>(stage + (4 * i + s_lane) * kRowPitch + g_lane * 16) = v[i];
+      } else {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
+          if (o < len) {
+            if (!kVerify || o + 16 <= len)
+              st_stream_v4(dst + o, v[i]);  // pack: zeros past len are owned padding
+            else
+              st_partial(dst + o, v[i], len - o);
+          }
+          *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
+        }
       }
       __syncwarp();
       // next round's loads stay in flight while this round's CRC runs
       if (r + 1 < nrounds) load_round(r + 1);
 #ifndef CHECL_EXP_SKIP_CRC
-      // lane l: segment 32r + l; Horner step over the other lanes' 31 segments
-      if (r > 0) crc = horner_mul(crc, hb, l4);
+      // lane l: segment 32r + l, as kChains independent chains of 128/kChains
+      // bytes (ILP); Horner step of each chain over the rest of the round
+      if (r > 0) {
+#pragma unroll
+        for (int c = 0; c < kChains; ++c) ch[c] = horner_mul(ch[c], hb, l4);
+      }
       const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
 #pragma unroll
-      for (int g = 0; g < 8; ++g) crc = crc_step16(crc, row[g], tb, l4);
+      for (int g = 0; g < 8 / kChains; ++g) {
+#pragma unroll
+        for (int c = 0; c < kChains; ++c) ch[c] = crc_step16(ch[c], row[c * (8 / kChains) + g], tb, l4);
+      }
 #endif
       __syncwarp();
     }
@@ -242,7 +269,10 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     // the 128*2^k bytes of the group to its right and adds it. The result is the
     // register of the chunk zero-padded to nrounds*4096 bytes; undo the zp padding
     // bytes with one multiply by x^(-8 zp).
-    uint32_t f = crc;
+    // the lane's register: chains joined in order (each shifted past the next chain's bytes)
+    uint32_t f = ch[0];
+#pragma unroll
+    for (int c = 1; c < kChains; ++c) f = gf_mul(f, p.chain_shift) ^ ch[c];
 #pragma unroll
     for (int k = 0; k < kFoldLevels; ++k) {
       const uint32_t o = __shfl_down_sync(full, f, 1 << k);
