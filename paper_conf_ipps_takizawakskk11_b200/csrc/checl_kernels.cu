@@ -185,7 +185,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     const int nrounds = (int)((len + kRoundBytes - 1) / kRoundBytes);
     uint32_t ch[kChains];
 #pragma unroll
-    for (int c = 0; c < kChains; ++c) ch[c] = (lane == 0 && c == 0) ? 0xFFFFFFFFu : 0u;
+    for (int cc = 0; cc < kChains; ++cc) ch[cc] = (lane == 0 && cc == 0) ? 0xFFFFFFFFu : 0u;
 
     uint4 v[8];
     // lane's byte offset of granule i in round r: r*4096 + (4i + l/8)*128 + (l%8)*16
@@ -241,13 +241,13 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
       // bytes (ILP); Horner step of each chain over the rest of the round
       if (r > 0) {
 #pragma unroll
-        for (int c = 0; c < kChains; ++c) ch[c] = horner_mul(ch[c], hb, l4);
+        for (int cc = 0; cc < kChains; ++cc) ch[cc] = horner_mul(ch[cc], hb, l4);
       }
       const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
 #pragma unroll
       for (int g = 0; g < 8 / kChains; ++g) {
 #pragma unroll
-        for (int c = 0; c < kChains; ++c) ch[c] = crc_step16(ch[c], row[c * (8 / kChains) + g], tb, l4);
+        for (int cc = 0; cc < kChains; ++cc) ch[cc] = crc_step16(ch[cc], row[cc * (8 / kChains) + g], tb, l4);
       }
 #endif
       __syncwarp();
@@ -272,7 +272,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     // the lane's register: chains joined in order (each shifted past the next chain's bytes)
     uint32_t f = ch[0];
 #pragma unroll
-    for (int c = 1; c < kChains; ++c) f = gf_mul(f, p.chain_shift) ^ ch[c];
+    for (int cc = 1; cc < kChains; ++cc) f = gf_mul(f, p.chain_shift) ^ ch[cc];
 #pragma unroll
     for (int k = 0; k < kFoldLevels; ++k) {
       const uint32_t o = __shfl_down_sync(full, f, 1 << k);
