@@ -27,7 +27,7 @@
 namespace checl {
 size_t snapshot_smem_bytes();
 cudaError_t snapshot_configure();
-cudaError_t launch_snapshot(bool verify, const LaunchParams& p, int n_sms, cudaStream_t s);
+cudaError_t launch_snapshot(bool verify, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel);
 cudaError_t launch_fill(uint8_t* ptr, uint64_t bytes, uint64_t key, int kind, int n_sms, cudaStream_t s);
 cudaError_t launch_compare(const uint8_t* a, const uint8_t* b, uint64_t bytes, unsigned long long* n_diff, int n_sms,
                            cudaStream_t s);
@@ -223,6 +223,11 @@ struct DevState {
   DevBuf<ChunkDesc> desc_scratch;
   DevBuf<BufferRecord> recs_scratch;
   DevBuf<unsigned long long> status;
+  DevBuf<uint32_t> lanepow, unitpow;  // sweep kernel
+  DevBuf<unsigned long long> unit_acc;
+  // 1 = warp per chunk (throughput), 2 = 4 KiB units swept by the grid (latency of
+  // small launches); 0 = by size; env CHECL_KERNEL=1|2 forces one
+  int kernel = 0;
   PinnedBuf<unsigned long long> h_status;
   PinnedBuf<BufferRecord> h_recs;
   EventPool events;
@@ -241,6 +246,14 @@ struct DevState {
     status.ensure(2);
     h_status.ensure(2);
     fill_fold(fold);
+    uint32_t lp[32], up[16];
+    for (int l = 0; l < 32; ++l) lp[l] = gf_x8n((uint64_t)kSegBytes * (31 - l));
+    for (int k = 0; k < 16; ++k) up[k] = gf_x8n((uint64_t)kRoundBytes * k);
+    lanepow.ensure(32);
+    unitpow.ensure(16);
+    ck(cudaMemcpy(lanepow.p, lp, sizeof lp, cudaMemcpyHostToDevice));
+    ck(cudaMemcpy(unitpow.p, up, sizeof up, cudaMemcpyHostToDevice));
+    if (const char* k = std::getenv("CHECL_KERNEL")) kernel = std::atoi(k) == 1 ? 1 : std::atoi(k) == 2 ? 2 : 0;
   }
   void ensure_slots(size_t bytes, uint32_t n) {
     if (slot_bytes == bytes && n_slots == n && slots.p) return;
@@ -263,6 +276,9 @@ struct DevState {
     recs_scratch.release();
     plan.d_recs.release();
     status.release();
+    unit_acc.release();
+    lanepow.release();
+    unitpow.release();
     plan.d_desc.release();
     h_status.release();
     h_recs.release();
@@ -665,13 +681,25 @@ LaunchParams base_params(DevState& ds) {
   for (int k = 0; k < kFoldLevels; ++k) p.fold[k] = ds.fold[k];
   p.horner = gf_x8n(kRoundBytes - kSegBytes / kChains);
   p.chain_shift = gf_x8n(kSegBytes / kChains);
+  p.lanepow = ds.lanepow.p;
+  p.unitpow = ds.unitpow.p;
   return p;
 }
 
-void timed_launch(DevState& ds, KernelTimer& kt, bool verify, const LaunchParams& p, cudaStream_t s) {
+void timed_launch(DevState& ds, KernelTimer& kt, bool verify, const LaunchParams& p0, cudaStream_t s) {
+  LaunchParams p = p0;
+  const uint64_t chunks = p.c1 - p.c0;
+  // a warp needs ~55 us per 64 KiB chunk in kernel 1: when chunks are fewer than
+  // half the warps, the 4 KiB-unit sweep finishes sooner (tools/size_scan.py)
+  const int kernel = ds.kernel ? ds.kernel : (chunks * 2 <= (uint64_t)ds.n_sms * kWarpsPerCta ? 2 : 1);
+  if (kernel == 2) {
+    ds.unit_acc.ensure(std::max<uint64_t>(chunks, 1));
+    p.unit_acc = ds.unit_acc.p;
+  }
   cudaEvent_t a = ds.events.get(), b = ds.events.get();
   ck(cudaEventRecord(a, s));
-  ck(launch_snapshot(verify, p, ds.n_sms, s));
+  if (kernel == 2 && chunks) ck(cudaMemsetAsync(p.unit_acc, 0, chunks * 8, s));
+  ck(launch_snapshot(verify, p, ds.n_sms, s, kernel));
   ck(cudaEventRecord(b, s));
   kt.spans.push_back({a, b});
 }

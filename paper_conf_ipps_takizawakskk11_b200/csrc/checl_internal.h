@@ -121,6 +121,10 @@ struct LaunchParams {
   uint32_t fold[kFoldLevels];  // x^(8 * 128 * 2^k) mod P
   uint32_t horner;             // x^(8 * (kRoundBytes - kSegBytes / kChains)) mod P
   uint32_t chain_shift;        // x^(8 * kSegBytes / kChains) mod P
+  // sweep kernel (one 4 KiB unit per warp-iteration)
+  unsigned long long* unit_acc;  // per chunk: low 32 = XOR of unit terms, high = finished-unit mask (zeroed)
+  const uint32_t* lanepow;     // 32 entries: x^(8 * 128 * (31 - l)) mod P
+  const uint32_t* unitpow;     // 16 entries: x^(8 * 4096 * k) mod P
 };
 
 }  // namespace checl

@@ -291,6 +291,229 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
   }
 }
 
+// ---- sweep kernel: one 4 KiB unit per warp-iteration ------------------------
+//
+// Same data path and CRC tables as snapshot_kernel, different work split: the
+// work units are the 4 KiB rounds of all chunks (unit u = round u%16 of chunk
+// u/16), taken grid-stride, so that at any time the warps of the whole GPU touch
+// neighbouring 4 KiB blocks of the payload (the access pattern a plain copy needs
+// to run near the HBM roofline) and a chunk's latency is one unit, not 16.
+// Lane l CRCs segment l of its unit (zero init; lane 0 of round 0 takes the CRC
+// init), then the unit register is  XOR_l  reg_l * x^(8*128*(31-l))  — one
+// lane-private nibble-table multiply per lane and a shuffle-XOR reduction. The
+// unit registers go to global memory; the last unit of a chunk to finish (atomic
+// counter) combines them: CRC = ~( XOR_u reg_u * x^(8*4096*(n-1-u)) * x^(-8 zp) ),
+// zp = 4096 n - len. The next unit's loads are issued before the current unit's CRC.
+
+// s * x^(8*128*(31-l)) mod P via 8 lane-private nibble lookups (lane l's constant).
+__device__ __forceinline__ uint32_t lanepos_mul(uint32_t s, const uint8_t* pb, uint32_t l4) {
+  uint32_t r = 0;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) r ^= tab_ld(pb + j * 2048, (((s >> (4 * j)) & 15u) << 7) | l4);
+  return r;
+}
+
+__device__ __forceinline__ uint32_t warp_xor(uint32_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v ^= __shfl_xor_sync(0xFFFFFFFFu, v, o);
+  return v;
+}
+
+template <bool kVerify>
+__global__ void __launch_bounds__(kThreadsPerCta, 1) sweep_kernel(const LaunchParams p) {
+  extern __shared__ __align__(16) uint32_t smem[];
+  uint32_t* tab = smem;
+  uint32_t* ptab = smem + kTabWords;  // lane-private position tables (kHornerWords words)
+  uint32_t* utab = ptab + kHornerWords;  // [16][32]: x^(8*4096*k) * x^i (within kFoldWords)
+  uint8_t* stage_all = reinterpret_cast<uint8_t*>(ptab + kHornerWords + kFoldWords);
+
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint32_t* scratch = reinterpret_cast<uint32_t*>(stage_all);
+  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
+    uint32_t r = (uint32_t)e;
+    for (int b = 0; b < 8; ++b) r = gf_mulx(r);
+    scratch[e] = r;
+  }
+  // position tables: entry (j, v) of lane l = (v << 4j) * C_l; from the four
+  // single-bit products C_l * x^(31-4j-t) (bit 4j+t of a reflected value is x^(31-4j-t))
+  for (int t = threadIdx.x; t < 8 * 32; t += blockDim.x) {
+    const int j = t >> 5, l = t & 31;
+    uint32_t b = p.lanepow[l];
+    for (int m = 0; m < 31 - 4 * j - 3; ++m) b = gf_mulx(b);  // b = C * x^(28-4j)
+    uint32_t bit[4];
+    bit[3] = b;  // v bit 3 sits at position 4j+3 -> x^(28-4j)
+    for (int q = 2; q >= 0; --q) bit[q] = gf_mulx(bit[q + 1]);
+    for (int v = 0; v < 16; ++v) {
+      uint32_t e = 0;
+      for (int q = 0; q < 4; ++q)
+        if (v & (1 << q)) e ^= bit[q];
+      ptab[(j * 16 + v) * 32 + l] = e;
+    }
+  }
+  for (int t = threadIdx.x; t < 16 * 32; t += blockDim.x) {
+    uint32_t b = p.unitpow[t >> 5];
+    for (int m = 0; m < (t & 31); ++m) b = gf_mulx(b);
+    utab[t] = b;
+  }
+  __syncthreads();
+  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
+    uint32_t r = scratch[e];
+    for (int k = 1; k < 4; ++k) {
+      r = (r >> 8) ^ scratch[r & 0xFFu];
+      scratch[k * 256 + e] = r;
+    }
+  }
+  __syncthreads();
+  for (int h = warp; h < 1024; h += kWarpsPerCta) {
+    const int st = h >> 9, e = (h >> 1) & 255, half = h & 1;
+    const int k = 3 - (2 * st + half);  // A = [T3|T2], B = [T1|T0]
+    tab[h * 32 + lane] = scratch[k * 256 + e];
+  }
+  __syncthreads();
+
+  uint8_t* stage = stage_all + warp * kStageBytes;
+  const uint8_t* tb = reinterpret_cast<const uint8_t*>(tab);
+  const uint8_t* pb = reinterpret_cast<const uint8_t*>(ptab);
+  const uint32_t l4 = (uint32_t)lane * 4u;
+  const int g_lane = lane & 7, s_lane = lane >> 3;
+  const uint32_t lane_off = (uint32_t)s_lane * kSegBytes + (uint32_t)g_lane * 16;
+  uint8_t* tile_w = stage + s_lane * kRowPitch + g_lane * 16;
+  const uint64_t nunits = (p.c1 - p.c0) * 16;
+  const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta;
+
+  struct Unit {
+    uint64_t c;
+    int r, nrounds, mode;
+    uint32_t len, pad;
+    const uint8_t* src;
+    uint8_t* dst;
+    bool on;
+  };
+  auto get_unit = [&](uint64_t u) {
+    Unit x;
+    x.on = false;
+    if (u >= nunits) return x;
+    x.c = p.c0 + (u >> 4);
+    x.r = (int)(u & 15);
+    const ChunkDesc d = p.desc[x.c];
+    x.len = desc_len(d);
+    x.pad = desc_pad(d);
+    x.nrounds = (int)((x.len + kRoundBytes - 1) / kRoundBytes);
+    if (x.r >= x.nrounds) return x;
+    uint8_t* img = p.image + ((uint64_t)d.img_off_256 * kBufferAlign - p.image_base);
+    x.src = kVerify ? img : reinterpret_cast<const uint8_t*>(d.ptr);
+    x.dst = kVerify ? reinterpret_cast<uint8_t*>(d.ptr) : img;
+    x.mode = kVerify ? 0 : ((d.ptr & 15u) == 0 ? 0 : ((d.ptr & 3u) == 0 ? 1 : 2));
+    x.on = true;
+    return x;
+  };
+  uint4 v[8];
+  auto load_unit = [&](const Unit& x) {
+    const uint32_t base = (uint32_t)x.r * kRoundBytes + lane_off;
+    if (x.mode == 0 && (uint32_t)(x.r + 1) * kRoundBytes <= x.len) {
+      const uint8_t* s = x.src + base;
+#pragma unroll
+      for (int i = 0; i < 8; ++i) v[i] = ld_stream_v4(s + i * 4 * kSegBytes);
+    } else {
+#pragma unroll
+      for (int i = 0; i < 8; ++i) {
+        const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
+        if (o + 16 <= x.len)
+          v[i] = ld_granule(x.src + o, x.mode);
+        else if (o < x.len)
+          v[i] = ld_partial(x.src + o, x.len - o);
+        else
+          v[i] = make_uint4(0u, 0u, 0u, 0u);
+      }
+    }
+  };
+
+  uint64_t u = (uint64_t)blockIdx.x * kWarpsPerCta + warp;
+  Unit cur = get_unit(u);
+  if (cur.on) load_unit(cur);
+  for (; u < nunits; u += nw) {
+    const Unit nxt = get_unit(u + nw);
+    if (cur.on) {
+      const uint32_t base = (uint32_t)cur.r * kRoundBytes + lane_off;
+      if ((uint32_t)(cur.r + 1) * kRoundBytes <= cur.len) {
+        uint8_t* d = cur.dst + base;
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          st_stream_v4(d + i * 4 * kSegBytes, v[i]);
+          *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
+        }
+      } else {
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+          const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
+          if (o < cur.len) {
+            if (!kVerify || o + 16 <= cur.len)
+              st_stream_v4(cur.dst + o, v[i]);  // pack: zeros past len are owned padding
+            else
+              st_partial(cur.dst + o, v[i], cur.len - o);
+          }
+          *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
+        }
+      }
+    }
+    __syncwarp();
+    if (nxt.on) load_unit(nxt);  // in flight during this unit's CRC
+    if (cur.on) {
+#ifndef CHECL_EXP_SKIP_CRC
+      uint32_t crc = (lane == 0 && cur.r == 0) ? 0xFFFFFFFFu : 0u;
+      const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
+#pragma unroll
+      for (int g = 0; g < 8; ++g) crc = crc_step16(crc, row[g], tb, l4);
+      const uint32_t reg = warp_xor(lanepos_mul(crc, pb, l4));
+      // the unit's term in the chunk register: reg * x^(8*4096*(n-1-r)), lane i
+      // adding the x^i coefficient of reg times utab[k][i] = x^(8*4096*k) * x^i
+      const int k = cur.nrounds - 1 - cur.r;
+      const uint32_t term = warp_xor(((reg >> (31 - lane)) & 1u) ? utab[k * 32 + lane] : 0u);
+#else
+      const uint32_t term = 0;
+#endif
+      // one 64-bit atomicXor carries the term (low half) and this unit's bit in the
+      // finished-unit mask (high half): the unit that completes the mask holds the
+      // chunk register — no fence, no second pass
+      const unsigned long long mine = (unsigned long long)term | (1ull << (32 + cur.r));
+      unsigned long long old = 0;
+#ifdef CHECL_EXP_SKIP_ATOMIC
+      if (lane == 0 && term == 0x12345678u) old = atomicXor(&p.unit_acc[cur.c - p.c0], mine);
+#else
+      if (lane == 0) old = atomicXor(&p.unit_acc[cur.c - p.c0], mine);
+#endif
+      const unsigned long long now = __shfl_sync(0xFFFFFFFFu, old, 0) ^ mine;
+      if ((now >> 32) == (1ull << cur.nrounds) - 1) {
+        // last unit of the chunk: zero-padding correction, padding, CRC table / check
+        const uint32_t t = (uint32_t)now;
+        const uint32_t zp = (uint32_t)cur.nrounds * kRoundBytes - cur.len;
+        const uint32_t out = ~(zp ? gf_mul(t, p.inv_z[zp]) : t);
+        uint32_t pad_bad = 0;
+        if (cur.pad) {
+          if (!kVerify) {
+            const uint32_t start = (cur.len + 15u) & ~15u, end = cur.len + cur.pad;
+            for (uint32_t o = start + lane * 16u; o < end; o += 512u)
+              *reinterpret_cast<uint4*>(cur.dst + o) = make_uint4(0u, 0u, 0u, 0u);
+          } else {
+            for (uint32_t o = cur.len + lane; o < cur.len + cur.pad; o += 32u) pad_bad |= cur.src[o];
+          }
+        }
+        if (kVerify) pad_bad = __any_sync(0xFFFFFFFFu, pad_bad != 0);
+        if (lane == 0) {
+          if (!kVerify) {
+            p.crc[cur.c] = out;
+          } else if (out != p.crc[cur.c] || pad_bad) {
+            atomicMin(&p.status[0], (unsigned long long)cur.c);
+            atomicAdd(&p.status[1], 1ull);
+          }
+        }
+      }
+    }
+    __syncwarp();
+    cur = nxt;
+  }
+}
+
 // ---- K6 test tooling -------------------------------------------------------
 
 __device__ __forceinline__ uint64_t mix64(uint64_t z) {
@@ -386,19 +609,34 @@ size_t snapshot_smem_bytes() { return kSmemBytes; }
 
 cudaError_t snapshot_configure() {
   cudaError_t e = cudaFuncSetAttribute(snapshot_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
-  if (e != cudaSuccess) return e;
-  return cudaFuncSetAttribute(snapshot_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(snapshot_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(sweep_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(sweep_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+  return e;
 }
 
-cudaError_t launch_snapshot(bool verify, const LaunchParams& p, int n_sms, cudaStream_t s) {
+// kernel 1 = warp per chunk (snapshot_kernel), 2 = 4 KiB units swept by the grid
+// (sweep_kernel; needs p.unit_reg / unit_cnt / lanepow / unitpow and a zeroed
+// unit_cnt for the chunk range)
+cudaError_t launch_snapshot(bool verify, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel) {
   const uint64_t chunks = p.c1 - p.c0;
   if (chunks == 0) return cudaSuccess;
-  uint64_t ctas = (chunks + kWarpsPerCta - 1) / kWarpsPerCta;
+  uint64_t ctas = kernel == 2 ? (chunks * 16 + kWarpsPerCta - 1) / kWarpsPerCta : (chunks + kWarpsPerCta - 1) / kWarpsPerCta;
   if (ctas > (uint64_t)n_sms) ctas = (uint64_t)n_sms;
-  if (verify)
-    snapshot_kernel<true><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
-  else
-    snapshot_kernel<false><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
+  if (kernel == 2) {
+    if (verify)
+      sweep_kernel<true><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
+    else
+      sweep_kernel<false><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
+  } else {
+    if (verify)
+      snapshot_kernel<true><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
+    else
+      snapshot_kernel<false><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
+  }
   return cudaGetLastError();
 }
 
