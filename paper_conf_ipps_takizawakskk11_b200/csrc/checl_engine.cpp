@@ -27,7 +27,8 @@
 namespace checl {
 size_t snapshot_smem_bytes();
 cudaError_t snapshot_configure();
-cudaError_t launch_snapshot(bool verify, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel);
+cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel);
+cudaError_t launch_build_tables(const TableParams& tp, uint32_t* out, cudaStream_t s);
 cudaError_t launch_fill(uint8_t* ptr, uint64_t bytes, uint64_t key, int kind, int n_sms, cudaStream_t s);
 cudaError_t launch_compare(const uint8_t* a, const uint8_t* b, uint64_t bytes, unsigned long long* n_diff, int n_sms,
                            cudaStream_t s);
@@ -128,8 +129,13 @@ const std::vector<uint32_t>& inv_z_table() {
   return t;
 }
 
-void fill_fold(uint32_t fold[kFoldLevels]) {
-  for (int k = 0; k < kFoldLevels; ++k) fold[k] = gf_x_pow2k(10 + k);  // x^(8*128*2^k)
+TableParams table_params() {
+  TableParams tp{};
+  for (int k = 0; k < kFoldLevels; ++k) tp.fold[k] = gf_x_pow2k(10 + k);  // x^(8*128*2^k)
+  tp.horner = gf_x8n(kRoundBytes - kSegBytes);
+  for (int l = 0; l < 32; ++l) tp.lanepow[l] = gf_x8n((uint64_t)kSegBytes * (31 - l));
+  for (int k = 0; k < 16; ++k) tp.unitpow[k] = gf_x8n((uint64_t)kRoundBytes * k);
+  return tp;
 }
 
 // ---- per-device resources ---------------------------------------------------
@@ -219,11 +225,10 @@ struct DevState {
   DevBuf<uint8_t> slots;
   size_t slot_bytes = 0;
   uint32_t n_slots = 0;
-  DevBuf<uint32_t> inv_z, crc_scratch;
+  DevBuf<uint32_t> inv_z, crc_scratch, tables;
   DevBuf<ChunkDesc> desc_scratch;
   DevBuf<BufferRecord> recs_scratch;
   DevBuf<unsigned long long> status;
-  DevBuf<uint32_t> lanepow, unitpow;  // sweep kernel
   DevBuf<unsigned long long> unit_acc;
   // 1 = warp per chunk (throughput), 2 = 4 KiB units swept by the grid (latency of
   // small launches); 0 = by size; env CHECL_KERNEL=1|2 forces one
@@ -232,7 +237,6 @@ struct DevState {
   PinnedBuf<BufferRecord> h_recs;
   EventPool events;
   Plan plan;
-  uint32_t fold[kFoldLevels];
 
   void init(int d) {
     dev = d;
@@ -245,14 +249,9 @@ struct DevState {
     ck(cudaMemcpy(inv_z.p, inv_z_table().data(), kRoundBytes * 4, cudaMemcpyHostToDevice));
     status.ensure(2);
     h_status.ensure(2);
-    fill_fold(fold);
-    uint32_t lp[32], up[16];
-    for (int l = 0; l < 32; ++l) lp[l] = gf_x8n((uint64_t)kSegBytes * (31 - l));
-    for (int k = 0; k < 16; ++k) up[k] = gf_x8n((uint64_t)kRoundBytes * k);
-    lanepow.ensure(32);
-    unitpow.ensure(16);
-    ck(cudaMemcpy(lanepow.p, lp, sizeof lp, cudaMemcpyHostToDevice));
-    ck(cudaMemcpy(unitpow.p, up, sizeof up, cudaMemcpyHostToDevice));
+    tables.ensure(kTableWords);
+    ck(launch_build_tables(table_params(), tables.p, compute));
+    ck(cudaStreamSynchronize(compute));
     if (const char* k = std::getenv("CHECL_KERNEL")) kernel = std::atoi(k) == 1 ? 1 : std::atoi(k) == 2 ? 2 : 0;
   }
   void ensure_slots(size_t bytes, uint32_t n) {
@@ -277,8 +276,7 @@ struct DevState {
     plan.d_recs.release();
     status.release();
     unit_acc.release();
-    lanepow.release();
-    unitpow.release();
+    tables.release();
     plan.d_desc.release();
     h_status.release();
     h_recs.release();
@@ -667,7 +665,7 @@ Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
                        ds.compute));
     ck(launch_expand(P.d_recs.p, (uint32_t)P.recs.size(), L.payload_bytes, L.n_chunks, P.d_desc.p, ds.n_sms,
                      ds.compute));
-    ck(cudaStreamSynchronize(ds.compute));  // P.recs may be rebuilt by the next plan
+    // no sync: a pageable-source cudaMemcpyAsync returns once P.recs has been staged
   }
   P.version = ctx->version[device];
   P.slot_bytes = ctx->slot_bytes;
@@ -678,28 +676,26 @@ LaunchParams base_params(DevState& ds) {
   LaunchParams p{};
   p.inv_z = ds.inv_z.p;
   p.status = ds.status.p;
-  for (int k = 0; k < kFoldLevels; ++k) p.fold[k] = ds.fold[k];
-  p.horner = gf_x8n(kRoundBytes - kSegBytes / kChains);
-  p.chain_shift = gf_x8n(kSegBytes / kChains);
-  p.lanepow = ds.lanepow.p;
-  p.unitpow = ds.unitpow.p;
+  p.tables = ds.tables.p;
   return p;
 }
 
-void timed_launch(DevState& ds, KernelTimer& kt, bool verify, const LaunchParams& p0, cudaStream_t s) {
+void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0, cudaStream_t s) {
   LaunchParams p = p0;
   const uint64_t chunks = p.c1 - p.c0;
   // a warp needs ~55 us per 64 KiB chunk in kernel 1: when chunks are fewer than
   // half the warps, the 4 KiB-unit sweep finishes sooner (tools/size_scan.py)
   const int kernel = ds.kernel ? ds.kernel : (chunks * 2 <= (uint64_t)ds.n_sms * kWarpsPerCta ? 2 : 1);
   if (kernel == 2) {
-    ds.unit_acc.ensure(std::max<uint64_t>(chunks, 1));
+    if (ds.unit_acc.cap < chunks) {  // zeroed once; every sweep launch leaves it zero
+      ds.unit_acc.ensure(chunks);
+      ck(cudaMemsetAsync(ds.unit_acc.p, 0, ds.unit_acc.cap * 8, s));
+    }
     p.unit_acc = ds.unit_acc.p;
   }
   cudaEvent_t a = ds.events.get(), b = ds.events.get();
   ck(cudaEventRecord(a, s));
-  if (kernel == 2 && chunks) ck(cudaMemsetAsync(p.unit_acc, 0, chunks * 8, s));
-  ck(launch_snapshot(verify, p, ds.n_sms, s, kernel));
+  ck(launch_snapshot(op, p, ds.n_sms, s, kernel));
   ck(cudaEventRecord(b, s));
   kt.spans.push_back({a, b});
 }
@@ -764,7 +760,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
     lp.image = img->d_payload;
     lp.image_base = 0;
     lp.crc = img->d_crc;
-    if (P.n_chunks) timed_launch(ds, kt, false, lp, ds.compute);
+    if (P.n_chunks) timed_launch(ds, kt, kOpPack, lp, ds.compute);
     ck(cudaEventRecord(c_begin, ds.compute));
     if (P.n_chunks)
       ck(cudaMemcpyAsync(img->host_mut + P.crc_off, img->d_crc, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.compute));
@@ -798,7 +794,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       lp.c1 = S.c1;
       lp.image = ds.slot(k);
       lp.image_base = S.img_lo;
-      timed_launch(ds, kt, false, lp, ds.compute);
+      timed_launch(ds, kt, kOpPack, lp, ds.compute);
       ck(cudaEventRecord(packed[k], ds.compute));
       ck(cudaStreamWaitEvent(ds.copy, packed[k], 0));
       ck(cudaMemcpyAsync(img->host_mut + P.payload_off + S.img_lo, ds.slot(k), S.img_hi - S.img_lo,
@@ -985,7 +981,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     lp.image = const_cast<uint8_t*>(src);
     lp.image_base = 0;
     lp.crc = const_cast<uint32_t*>(crc);
-    if (nch) timed_launch(ds, kt, true, lp, ds.compute);
+    if (nch) timed_launch(ds, kt, kOpVerify, lp, ds.compute);
     tm.n_stages = 1;
   } else {
     // r3 + r4: fill slot s % n_slots over PCIe while the previous slot is verified
@@ -1011,7 +1007,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
       lp.c1 = S.c1;
       lp.image = ds.slot(k);
       lp.image_base = S.img_lo;
-      timed_launch(ds, kt, true, lp, ds.compute);
+      timed_launch(ds, kt, kOpVerify, lp, ds.compute);
       ck(cudaEventRecord(verified[k], ds.compute));
     }
     ck(cudaEventRecord(c_end, ds.copy));

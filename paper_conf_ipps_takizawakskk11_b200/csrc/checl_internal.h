@@ -101,30 +101,52 @@ constexpr int kRowPitch = kSegBytes + 16;        // padded smem row: conflict-fr
 constexpr int kWarpsPerCta = CHECL_WARPS;
 constexpr int kThreadsPerCta = kWarpsPerCta * 32;
 constexpr int kFoldLevels = 5;
-#ifndef CHECL_CHAINS
-#define CHECL_CHAINS 1
-#endif
-constexpr int kChains = CHECL_CHAINS;  // independent CRC chains per lane per segment (ILP)
-static_assert(kChains == 1 || kChains == 2 || kChains == 4 || kChains == 8, "chains divide the 8 granules");
 
-// Parameters of one pack (checkpoint) or verify (restore) launch over the chunk
-// range [c0, c1) of `desc`. Payload byte o of the image lives at
-// image + o - image_base for the chunks of this launch.
+// What one launch does with each chunk of its list (the same data path serves
+// every step that streams chunks):
+//   kOpPack   a3  K1: buffer -> image, CRC -> table, zero the owned padding
+//   kOpVerify r4  K2: image -> buffer, CRC == table and owned padding zero
+//   kOpCrc    f1  CRC only (no copy): the table of the current contents
+//   kOpCheck  f1  CRC only, compared with the table (in-place verify of a restore)
+//   kOpCopy   f1  buffer -> image without CRC (gather of an incremental image)
+enum : int { kOpPack = 0, kOpVerify = 1, kOpCrc = 2, kOpCheck = 3, kOpCopy = 4 };
+
+// Lane-private lookup tables, computed once per device into global memory and
+// bulk-copied (cp.async.bulk) into shared memory by every CTA. Word offsets:
+constexpr int kTabWords = 4 * 256 * 32;          // slicing-by-4, 128 KiB
+constexpr int kHornerWords = 8 * 16 * 32;       // x^(8*3968) nibble tables, 16 KiB
+constexpr int kFoldWords = kFoldLevels * 8 * 16; // fold nibble tables, 2.5 KiB
+constexpr int kPosWords = 8 * 16 * 32;          // sweep: lane-position nibble tables, 16 KiB
+constexpr int kUnitWords = 16 * 32;             // sweep: x^(8*4096*k) * x^i, 2 KiB
+constexpr int kTabOff = 0;
+constexpr int kHornerOff = kTabOff + kTabWords;
+constexpr int kFoldOff = kHornerOff + kHornerWords;
+constexpr int kPosOff = kFoldOff + kFoldWords;
+constexpr int kUnitOff = kPosOff + kPosWords;
+constexpr int kTableWords = kUnitOff + kUnitWords;
+static_assert((kPosOff * 4) % 16 == 0 && (kFoldOff * 4 + kFoldWords * 4) % 16 == 0, "bulk-copy alignment");
+
+// Constants the table builder needs (computed on the host).
+struct TableParams {
+  uint32_t fold[kFoldLevels];  // x^(8 * 128 * 2^k) mod P
+  uint32_t horner;             // x^(8 * (kRoundBytes - kSegBytes)) mod P
+  uint32_t lanepow[32];        // x^(8 * 128 * (31 - l)) mod P
+  uint32_t unitpow[16];        // x^(8 * 4096 * k) mod P
+};
+
+// Parameters of one launch over the chunk range [c0, c1) of `desc`. Payload byte
+// o of the image lives at image + o - image_base for the chunks of this launch.
 struct LaunchParams {
   const ChunkDesc* desc;
   uint64_t c0, c1;
-  uint8_t* image;           // pack: destination slot; verify: source (may be a peer address)
+  uint8_t* image;           // pack/copy: destination slot; verify: source (may be a peer address)
   uint64_t image_base;      // payload offset that maps to image[0]
-  uint32_t* crc;            // pack: output table (global chunk index); verify: reference table
+  uint32_t* crc;            // pack/crc: output table (global chunk index); verify/check: reference table
   const uint32_t* inv_z;    // kRoundBytes entries, x^(-8z) mod P
-  unsigned long long* status;  // verify: [0] = first bad chunk (atomicMin), [1] = bad count
-  uint32_t fold[kFoldLevels];  // x^(8 * 128 * 2^k) mod P
-  uint32_t horner;             // x^(8 * (kRoundBytes - kSegBytes / kChains)) mod P
-  uint32_t chain_shift;        // x^(8 * kSegBytes / kChains) mod P
+  const uint32_t* tables;   // kTableWords words (build_tables)
+  unsigned long long* status;  // verify/check: [0] = first bad chunk (atomicMin), [1] = bad count
   // sweep kernel (one 4 KiB unit per warp-iteration)
   unsigned long long* unit_acc;  // per chunk: low 32 = XOR of unit terms, high = finished-unit mask (zeroed)
-  const uint32_t* lanepow;     // 32 entries: x^(8 * 128 * (31 - l)) mod P
-  const uint32_t* unitpow;     // 16 entries: x^(8 * 4096 * k) mod P
 };
 
 }  // namespace checl

@@ -6,7 +6,7 @@
 //     CRC-verified, and its bytes are scattered into freshly re-created buffers")
 //  K6 debug fill / compare (test tooling: synth/ generator on the device)
 //
-// Both K1 and K2 are one template (snapshot_kernel<kVerify>): a persistent grid,
+// Both K1 and K2 are one template (snapshot_kernel<kOp>): a persistent grid,
 // one warp per chunk (<= 64 KiB) of a flat chunk list. A chunk is moved in rounds
 // of 4 KiB of contiguous bytes: eight coalesced 16-byte global loads per lane
 // (each warp instruction = 512 contiguous bytes), a coalesced 16-byte store of the
@@ -28,11 +28,12 @@
 
 namespace checl {
 
-constexpr int kTabWords = 4 * 256 * 32;          // 128 KiB, lane-private slicing-by-4
-constexpr int kHornerWords = 8 * 16 * 32;       // 16 KiB lane-private nibble tables
-constexpr int kFoldWords = kFoldLevels * 8 * 16; // 2.5 KiB nibble tables
 constexpr int kStageBytes = 32 * kRowPitch;      // per warp
-constexpr size_t kSmemBytes = (size_t)(kTabWords + kHornerWords + kFoldWords) * 4 + (size_t)kWarpsPerCta * kStageBytes;
+constexpr int kSnapTabWords = kPosOff;           // snapshot kernel: tab | horner | fold
+constexpr size_t kTileOff = (size_t)kSnapTabWords * 4;
+constexpr size_t kMbarOff = kTileOff + (size_t)kWarpsPerCta * kStageBytes;
+constexpr size_t kSmemBytes = kMbarOff + 16;
+static_assert(kSmemBytes <= 232448, "fits the 227 KiB opt-in shared memory");
 
 __device__ __forceinline__ uint4 ld_stream_v4(const void* p) {
   uint4 r;
@@ -121,173 +122,211 @@ __device__ __forceinline__ uint32_t horner_mul(uint32_t s, const uint8_t* hb, ui
   return r;
 }
 
-template <bool kVerify>
-__global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const LaunchParams p) {
-  extern __shared__ __align__(16) uint32_t smem[];
-  uint32_t* tab = smem;
-  uint32_t* htab = smem + kTabWords;
-  uint32_t* ftab = htab + kHornerWords;
-  uint8_t* stage_all = reinterpret_cast<uint8_t*>(ftab + kFoldWords);
+// What each op does (kOp* in checl_internal.h).
+template <int kOp>
+struct OpT {
+  static constexpr bool kSrcImg = kOp == kOpVerify;   // read the image, write the buffer
+  static constexpr bool kStore = kOp == kOpPack || kOp == kOpVerify || kOp == kOpCopy;
+  static constexpr bool kCrc = kOp != kOpCopy;
+  static constexpr bool kCompare = kOp == kOpVerify || kOp == kOpCheck;  // vs table + owned padding zero
+  static constexpr bool kZeroPad = kOp == kOpPack || kOp == kOpCopy;     // destination is the image
+  static constexpr bool kExactTail = kOp == kOpVerify;                   // destination is a buffer
+};
 
-  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  // Tables. T_k[e] = CRC register of byte e followed by k zero bytes (zero init):
-  // T_0 by bit steps into a scratch (the warp tiles, unused yet), T_1..T_3 from
-  // it; H[j][v] = (v << 4j) * x^(8*3968); then one warp store per 32 words
-  // replicates an entry across the lanes (conflict-free).
-  uint32_t* scratch = reinterpret_cast<uint32_t*>(stage_all);
-  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
-    uint32_t r = (uint32_t)e;
-    for (int b = 0; b < 8; ++b) r = gf_mulx(r);
-    scratch[e] = r;
-  }
-  for (int i = threadIdx.x; i < 128; i += blockDim.x)
-    scratch[1024 + i] = gf_mul((uint32_t)(i & 15) << (4 * (i >> 4)), p.horner);
-  __syncthreads();
-  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
-    uint32_t r = scratch[e];
-    for (int k = 1; k < 4; ++k) {
-      r = (r >> 8) ^ scratch[r & 0xFFu];
-      scratch[k * 256 + e] = r;
+__device__ __forceinline__ uint32_t smem_addr(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+// Bulk-copies `n` regions of the global table image into shared memory (one
+// elected thread issues cp.async.bulk, everyone waits on one mbarrier). Sizes and
+// addresses are multiples of 16.
+struct TableCopy {
+  uint32_t dst_off, src_word, bytes;
+};
+template <int N>
+__device__ __forceinline__ void load_tables(uint8_t* smem, const uint32_t* gtab, const TableCopy (&cp)[N],
+                                            uint64_t* mbar) {
+  const uint32_t mb = smem_addr(mbar);
+  if (threadIdx.x == 0) {
+    uint32_t total = 0;
+#pragma unroll
+    for (int i = 0; i < N; ++i) total += cp[i].bytes;
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(total) : "memory");
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+      for (uint32_t o = 0; o < cp[i].bytes; o += 32768u) {
+        const uint32_t n = cp[i].bytes - o < 32768u ? cp[i].bytes - o : 32768u;
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                smem_addr(smem + cp[i].dst_off + o)),
+            "l"(reinterpret_cast<const uint8_t*>(gtab + cp[i].src_word) + o), "r"(n), "r"(mb)
+            : "memory");
+      }
     }
   }
-  for (int i = threadIdx.x; i < kFoldWords; i += blockDim.x) {
-    const int lvl = i >> 7, j = (i >> 4) & 7, v = i & 15;
-    // select, not p.fold[lvl]: a dynamic index into kernel parameters spills them to the stack
-    const uint32_t cl = lvl == 0 ? p.fold[0] : lvl == 1 ? p.fold[1] : lvl == 2 ? p.fold[2] : lvl == 3 ? p.fold[3] : p.fold[4];
-    ftab[i] = gf_mul((uint32_t)v << (4 * j), cl);
-  }
-  __syncthreads();
-  for (int h = warp; h < 1024; h += kWarpsPerCta) {  // h = row-half: super-table, row, half
-    const int st = h >> 9, e = (h >> 1) & 255, half = h & 1;
-    const int k = 3 - (2 * st + half);  // A = [T3|T2], B = [T1|T0]
-    tab[h * 32 + lane] = scratch[k * 256 + e];
-  }
-  for (int h = warp; h < 128; h += kWarpsPerCta) htab[h * 32 + lane] = scratch[1024 + h];
-  __syncthreads();
+  __syncthreads();  // the barrier is initialised before anyone waits on it
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], 0;\n"
+      " @!p bra WAIT_%=;\n}" ::"r"(mb)
+      : "memory");
+}
 
-  uint8_t* stage = stage_all + warp * kStageBytes;
-  const uint8_t* tb = reinterpret_cast<const uint8_t*>(tab);
-  const uint8_t* hb = reinterpret_cast<const uint8_t*>(htab);
+// Loads granule set of round `r` (8 x 16 B per lane) of a chunk of `len` bytes.
+__device__ __forceinline__ void load_round(uint4 (&v)[8], const uint8_t* src, uint32_t len, int mode, int r,
+                                           uint32_t lane_off) {
+  const uint32_t base = (uint32_t)r * kRoundBytes + lane_off;
+  if (mode == 0 && (uint32_t)(r + 1) * kRoundBytes <= len) {  // warp-uniform fast path
+    const uint8_t* s = src + base;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) v[i] = ld_stream_v4(s + i * 4 * kSegBytes);
+  } else {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
+      if (o + 16 <= len)
+        v[i] = ld_granule(src + o, mode);
+      else if (o < len)
+        v[i] = ld_partial(src + o, len - o);
+      else
+        v[i] = make_uint4(0u, 0u, 0u, 0u);  // past the chunk: CRC'd as zeros, corrected at the end
+    }
+  }
+}
+
+// Stores round r to the destination (if the op stores) and into the warp's tile.
+template <int kOp>
+__device__ __forceinline__ void store_round(const uint4 (&v)[8], uint8_t* dst, uint32_t len, int r, uint32_t lane_off,
+                                            uint8_t* tile_w) {
+  using O = OpT<kOp>;
+  const uint32_t base = (uint32_t)r * kRoundBytes + lane_off;
+  if ((uint32_t)(r + 1) * kRoundBytes <= len) {  // warp-uniform fast path
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      if (O::kStore) st_stream_v4(dst + base + i * 4 * kSegBytes, v[i]);
+      if (O::kCrc) *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
+    }
+  } else {
+#pragma unroll
+    for (int i = 0; i < 8; ++i) {
+      const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
+      if (O::kStore && o < len) {
+        if (!O::kExactTail || o + 16 <= len)
+          st_stream_v4(dst + o, v[i]);  // image destination: zeros past len are owned padding
+        else
+          st_partial(dst + o, v[i], len - o);
+      }
+      if (O::kCrc) *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
+    }
+  }
+}
+
+// End of a chunk: the owned padding (zeroed in the image, or checked), and the CRC
+// word (written to the table, or compared). `f` = the chunk register before the
+// zero-padding correction, valid in lane 0.
+template <int kOp>
+__device__ __forceinline__ void finish_chunk(const LaunchParams& p, uint64_t c, const uint8_t* src, uint8_t* dst,
+                                             uint32_t len, uint32_t pad, int nrounds, uint32_t f, int lane) {
+  using O = OpT<kOp>;
+  uint32_t pad_bad = 0;
+  if (pad) {
+    if (O::kZeroPad) {
+      const uint32_t start = (len + 15u) & ~15u, end = len + pad;
+      for (uint32_t o = start + lane * 16u; o < end; o += 512u)
+        *reinterpret_cast<uint4*>(dst + o) = make_uint4(0u, 0u, 0u, 0u);
+    } else if (O::kCompare) {
+      for (uint32_t o = len + lane; o < len + pad; o += 32u) pad_bad |= src[o];
+    }
+  }
+  if (O::kCompare) pad_bad = __any_sync(0xFFFFFFFFu, pad_bad != 0);
+  if (O::kCrc && lane == 0) {
+    const uint32_t zp = (uint32_t)nrounds * kRoundBytes - len;
+    const uint32_t out = ~(zp ? gf_mul(f, p.inv_z[zp]) : f);
+    if (!O::kCompare) {
+      p.crc[c] = out;
+    } else if (out != p.crc[c] || pad_bad) {
+      atomicMin(&p.status[0], (unsigned long long)c);
+      atomicAdd(&p.status[1], 1ull);
+    }
+  }
+}
+
+template <int kOp>
+__device__ __forceinline__ void chunk_ptrs(const LaunchParams& p, const ChunkDesc& d, const uint8_t*& src,
+                                           uint8_t*& dst, int& mode) {
+  using O = OpT<kOp>;
+  uint8_t* img = p.image + ((uint64_t)d.img_off_256 * kBufferAlign - p.image_base);
+  uint8_t* buf = reinterpret_cast<uint8_t*>(d.ptr);
+  src = O::kSrcImg ? img : buf;
+  dst = O::kSrcImg ? buf : img;
+  mode = O::kSrcImg ? 0 : ((d.ptr & 15u) == 0 ? 0 : ((d.ptr & 3u) == 0 ? 1 : 2));
+}
+
+template <int kOp>
+__global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const LaunchParams p) {
+  using O = OpT<kOp>;
+  extern __shared__ __align__(128) uint8_t smem[];
+  if (O::kCrc) {
+    const TableCopy cp[1] = {{0u, (uint32_t)kTabOff, (uint32_t)kSnapTabWords * 4u}};
+    load_tables(smem, p.tables, cp, reinterpret_cast<uint64_t*>(smem + kMbarOff));
+  }
+  const uint8_t* tb = smem + kTabOff * 4;
+  const uint8_t* hb = smem + kHornerOff * 4;
+  const uint32_t* ftab = reinterpret_cast<const uint32_t*>(smem + kFoldOff * 4);
+
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint8_t* stage = smem + kTileOff + warp * kStageBytes;
   const uint32_t l4 = (uint32_t)lane * 4u;
   const uint64_t nwarps = (uint64_t)gridDim.x * kWarpsPerCta;
   const unsigned full = 0xFFFFFFFFu;
   // instruction i of a round: lane l moves granule l%8 of segment 4i + l/8 (each
   // warp instruction = 512 contiguous bytes = four full 128-byte lines)
   const int g_lane = lane & 7, s_lane = lane >> 3;
+  const uint32_t lane_off = (uint32_t)s_lane * kSegBytes + (uint32_t)g_lane * 16;
+  uint8_t* tile_w = stage + s_lane * kRowPitch + g_lane * 16;  // this lane's slot, instruction 0
 
   for (uint64_t c = p.c0 + (uint64_t)blockIdx.x * kWarpsPerCta + warp; c < p.c1; c += nwarps) {
     const ChunkDesc d = p.desc[c];
     const uint32_t len = desc_len(d), pad = desc_pad(d);
-    uint8_t* img = p.image + ((uint64_t)d.img_off_256 * kBufferAlign - p.image_base);
-    const uint8_t* src = kVerify ? img : reinterpret_cast<const uint8_t*>(d.ptr);
-    uint8_t* dst = kVerify ? reinterpret_cast<uint8_t*>(d.ptr) : img;
-    const int mode = kVerify ? 0 : ((d.ptr & 15u) == 0 ? 0 : ((d.ptr & 3u) == 0 ? 1 : 2));
+    const uint8_t* src;
+    uint8_t* dst;
+    int mode;
+    chunk_ptrs<kOp>(p, d, src, dst, mode);
     const int nrounds = (int)((len + kRoundBytes - 1) / kRoundBytes);
-    uint32_t ch[kChains];
-#pragma unroll
-    for (int cc = 0; cc < kChains; ++cc) ch[cc] = (lane == 0 && cc == 0) ? 0xFFFFFFFFu : 0u;
+    uint32_t ch = lane == 0 ? 0xFFFFFFFFu : 0u;
 
     uint4 v[8];
-    // lane's byte offset of granule i in round r: r*4096 + (4i + l/8)*128 + (l%8)*16
-    const uint32_t lane_off = (uint32_t)s_lane * kSegBytes + (uint32_t)g_lane * 16;
-    auto load_round = [&](int r) {
-      const uint32_t base = (uint32_t)r * kRoundBytes + lane_off;
-      if (mode == 0 && (uint32_t)(r + 1) * kRoundBytes <= len) {  // warp-uniform fast path
-        const uint8_t* s = src + base;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) v[i] = ld_stream_v4(s + i * 4 * kSegBytes);
-      } else {
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
-          if (o + 16 <= len)
-            v[i] = ld_granule(src + o, mode);
-          else if (o < len)
-            v[i] = ld_partial(src + o, len - o);
-          else
-            v[i] = make_uint4(0u, 0u, 0u, 0u);  // past the chunk: CRC'd as zeros, corrected below
-        }
-      }
-    };
-    uint8_t* tile_w = stage + s_lane * kRowPitch + g_lane * 16;  // this lane's slot, instruction 0
-    load_round(0);
+    load_round(v, src, len, mode, 0, lane_off);
     for (int r = 0; r < nrounds; ++r) {
-      const uint32_t base = (uint32_t)r * kRoundBytes + lane_off;
-      if ((uint32_t)(r + 1) * kRoundBytes <= len) {  // warp-uniform fast path
-        uint8_t* d = dst + base;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          st_stream_v4(d + i * 4 * kSegBytes, v[i]);
-          *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
-        }
-      } else {
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
-          if (o < len) {
-            if (!kVerify || o + 16 <= len)
-              st_stream_v4(dst + o, v[i]);  // pack: zeros past len are owned padding
-            else
-              st_partial(dst + o, v[i], len - o);
-          }
-          *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
-        }
-      }
+      store_round<kOp>(v, dst, len, r, lane_off, tile_w);
       __syncwarp();
       // next round's loads stay in flight while this round's CRC runs
-      if (r + 1 < nrounds) load_round(r + 1);
-#ifndef CHECL_EXP_SKIP_CRC
-      // lane l: segment 32r + l, as kChains independent chains of 128/kChains
-      // bytes (ILP); Horner step of each chain over the rest of the round
-      if (r > 0) {
+      if (r + 1 < nrounds) load_round(v, src, len, mode, r + 1, lane_off);
+      if (O::kCrc) {
+        // lane l: segment 32r + l; Horner step over the rest of the round first
+        if (r > 0) ch = horner_mul(ch, hb, l4);
+        const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
 #pragma unroll
-        for (int cc = 0; cc < kChains; ++cc) ch[cc] = horner_mul(ch[cc], hb, l4);
+        for (int g = 0; g < 8; ++g) ch = crc_step16(ch, row[g], tb, l4);
       }
-      const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
-#pragma unroll
-      for (int g = 0; g < 8 / kChains; ++g) {
-#pragma unroll
-        for (int cc = 0; cc < kChains; ++cc) ch[cc] = crc_step16(ch[cc], row[cc * (8 / kChains) + g], tb, l4);
-      }
-#endif
       __syncwarp();
     }
-
-    uint32_t pad_bad = 0;
-    if (pad) {
-      if (!kVerify) {
-        const uint32_t start = (len + 15u) & ~15u, end = len + pad;
-        for (uint32_t o = start + lane * 16u; o < end; o += 512u)
-          *reinterpret_cast<uint4*>(dst + o) = make_uint4(0u, 0u, 0u, 0u);
-      } else {
-        for (uint32_t o = len + lane; o < len + pad; o += 32u) pad_bad |= src[o];
-      }
-    }
-    if (kVerify) pad_bad = __any_sync(full, pad_bad != 0);
 
     // Fold the lanes: at level k, lane l (l % 2^(k+1) == 0) shifts its group past
     // the 128*2^k bytes of the group to its right and adds it. The result is the
-    // register of the chunk zero-padded to nrounds*4096 bytes; undo the zp padding
-    // bytes with one multiply by x^(-8 zp).
-    // the lane's register: chains joined in order (each shifted past the next chain's bytes)
-    uint32_t f = ch[0];
+    // register of the chunk zero-padded to nrounds*4096 bytes (corrected in
+    // finish_chunk with one multiply by x^(-8 zp)).
+    uint32_t f = ch;
+    if (O::kCrc) {
 #pragma unroll
-    for (int cc = 1; cc < kChains; ++cc) f = gf_mul(f, p.chain_shift) ^ ch[cc];
-#pragma unroll
-    for (int k = 0; k < kFoldLevels; ++k) {
-      const uint32_t o = __shfl_down_sync(full, f, 1 << k);
-      if ((lane & ((2 << k) - 1)) == 0) f = fold_mul(f, ftab + k * 128) ^ o;
-    }
-    if (lane == 0) {
-      const uint32_t zp = (uint32_t)nrounds * kRoundBytes - len;
-      const uint32_t out = ~(zp ? gf_mul(f, p.inv_z[zp]) : f);
-      if (!kVerify) {
-        p.crc[c] = out;
-      } else if (out != p.crc[c] || pad_bad) {
-        atomicMin(&p.status[0], (unsigned long long)c);
-        atomicAdd(&p.status[1], 1ull);
+      for (int k = 0; k < kFoldLevels; ++k) {
+        const uint32_t o = __shfl_down_sync(full, f, 1 << k);
+        if ((lane & ((2 << k) - 1)) == 0) f = fold_mul(f, ftab + k * 128) ^ o;
       }
     }
+    finish_chunk<kOp>(p, c, src, dst, len, pad, nrounds, f, lane);
   }
 }
 
@@ -301,9 +340,10 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
 // Lane l CRCs segment l of its unit (zero init; lane 0 of round 0 takes the CRC
 // init), then the unit register is  XOR_l  reg_l * x^(8*128*(31-l))  — one
 // lane-private nibble-table multiply per lane and a shuffle-XOR reduction. The
-// unit registers go to global memory; the last unit of a chunk to finish (atomic
-// counter) combines them: CRC = ~( XOR_u reg_u * x^(8*4096*(n-1-u)) * x^(-8 zp) ),
-// zp = 4096 n - len. The next unit's loads are issued before the current unit's CRC.
+// unit's term reg * x^(8*4096*(n-1-r)) is XORed into a per-chunk 64-bit word
+// whose high half is a mask of finished units; the unit that completes the mask
+// holds the chunk register: CRC = ~( XOR_u term_u * x^(-8 zp) ), zp = 4096 n - len.
+// The next unit's loads are issued before the current unit's CRC.
 
 // s * x^(8*128*(31-l)) mod P via 8 lane-private nibble lookups (lane l's constant).
 __device__ __forceinline__ uint32_t lanepos_mul(uint32_t s, const uint8_t* pb, uint32_t l4) {
@@ -319,61 +359,25 @@ __device__ __forceinline__ uint32_t warp_xor(uint32_t v) {
   return v;
 }
 
-template <bool kVerify>
+template <int kOp>
 __global__ void __launch_bounds__(kThreadsPerCta, 1) sweep_kernel(const LaunchParams p) {
-  extern __shared__ __align__(16) uint32_t smem[];
-  uint32_t* tab = smem;
-  uint32_t* ptab = smem + kTabWords;  // lane-private position tables (kHornerWords words)
-  uint32_t* utab = ptab + kHornerWords;  // [16][32]: x^(8*4096*k) * x^i (within kFoldWords)
-  uint8_t* stage_all = reinterpret_cast<uint8_t*>(ptab + kHornerWords + kFoldWords);
+  using O = OpT<kOp>;
+  extern __shared__ __align__(128) uint8_t smem[];
+  // shared layout: tab | pos | unit | (unused) | tiles | mbarrier
+  constexpr uint32_t kPosSm = (uint32_t)kTabWords * 4u;
+  constexpr uint32_t kUnitSm = kPosSm + (uint32_t)kPosWords * 4u;
+  static_assert(kUnitSm + kUnitWords * 4u <= kTileOff, "sweep tables fit before the tiles");
+  if (O::kCrc) {
+    const TableCopy cp[2] = {{0u, (uint32_t)kTabOff, (uint32_t)kTabWords * 4u},
+                             {kPosSm, (uint32_t)kPosOff, (uint32_t)(kPosWords + kUnitWords) * 4u}};
+    load_tables(smem, p.tables, cp, reinterpret_cast<uint64_t*>(smem + kMbarOff));
+  }
+  const uint8_t* tb = smem;
+  const uint8_t* pb = smem + kPosSm;
+  const uint32_t* utab = reinterpret_cast<const uint32_t*>(smem + kUnitSm);
 
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
-  uint32_t* scratch = reinterpret_cast<uint32_t*>(stage_all);
-  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
-    uint32_t r = (uint32_t)e;
-    for (int b = 0; b < 8; ++b) r = gf_mulx(r);
-    scratch[e] = r;
-  }
-  // position tables: entry (j, v) of lane l = (v << 4j) * C_l; from the four
-  // single-bit products C_l * x^(31-4j-t) (bit 4j+t of a reflected value is x^(31-4j-t))
-  for (int t = threadIdx.x; t < 8 * 32; t += blockDim.x) {
-    const int j = t >> 5, l = t & 31;
-    uint32_t b = p.lanepow[l];
-    for (int m = 0; m < 31 - 4 * j - 3; ++m) b = gf_mulx(b);  // b = C * x^(28-4j)
-    uint32_t bit[4];
-    bit[3] = b;  // v bit 3 sits at position 4j+3 -> x^(28-4j)
-    for (int q = 2; q >= 0; --q) bit[q] = gf_mulx(bit[q + 1]);
-    for (int v = 0; v < 16; ++v) {
-      uint32_t e = 0;
-      for (int q = 0; q < 4; ++q)
-        if (v & (1 << q)) e ^= bit[q];
-      ptab[(j * 16 + v) * 32 + l] = e;
-    }
-  }
-  for (int t = threadIdx.x; t < 16 * 32; t += blockDim.x) {
-    uint32_t b = p.unitpow[t >> 5];
-    for (int m = 0; m < (t & 31); ++m) b = gf_mulx(b);
-    utab[t] = b;
-  }
-  __syncthreads();
-  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
-    uint32_t r = scratch[e];
-    for (int k = 1; k < 4; ++k) {
-      r = (r >> 8) ^ scratch[r & 0xFFu];
-      scratch[k * 256 + e] = r;
-    }
-  }
-  __syncthreads();
-  for (int h = warp; h < 1024; h += kWarpsPerCta) {
-    const int st = h >> 9, e = (h >> 1) & 255, half = h & 1;
-    const int k = 3 - (2 * st + half);  // A = [T3|T2], B = [T1|T0]
-    tab[h * 32 + lane] = scratch[k * 256 + e];
-  }
-  __syncthreads();
-
-  uint8_t* stage = stage_all + warp * kStageBytes;
-  const uint8_t* tb = reinterpret_cast<const uint8_t*>(tab);
-  const uint8_t* pb = reinterpret_cast<const uint8_t*>(ptab);
+  uint8_t* stage = smem + kTileOff + warp * kStageBytes;
   const uint32_t l4 = (uint32_t)lane * 4u;
   const int g_lane = lane & 7, s_lane = lane >> 3;
   const uint32_t lane_off = (uint32_t)s_lane * kSegBytes + (uint32_t)g_lane * 16;
@@ -400,117 +404,106 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) sweep_kernel(const LaunchPa
     x.pad = desc_pad(d);
     x.nrounds = (int)((x.len + kRoundBytes - 1) / kRoundBytes);
     if (x.r >= x.nrounds) return x;
-    uint8_t* img = p.image + ((uint64_t)d.img_off_256 * kBufferAlign - p.image_base);
-    x.src = kVerify ? img : reinterpret_cast<const uint8_t*>(d.ptr);
-    x.dst = kVerify ? reinterpret_cast<uint8_t*>(d.ptr) : img;
-    x.mode = kVerify ? 0 : ((d.ptr & 15u) == 0 ? 0 : ((d.ptr & 3u) == 0 ? 1 : 2));
+    chunk_ptrs<kOp>(p, d, x.src, x.dst, x.mode);
     x.on = true;
     return x;
   };
   uint4 v[8];
-  auto load_unit = [&](const Unit& x) {
-    const uint32_t base = (uint32_t)x.r * kRoundBytes + lane_off;
-    if (x.mode == 0 && (uint32_t)(x.r + 1) * kRoundBytes <= x.len) {
-      const uint8_t* s = x.src + base;
-#pragma unroll
-      for (int i = 0; i < 8; ++i) v[i] = ld_stream_v4(s + i * 4 * kSegBytes);
-    } else {
-#pragma unroll
-      for (int i = 0; i < 8; ++i) {
-        const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
-        if (o + 16 <= x.len)
-          v[i] = ld_granule(x.src + o, x.mode);
-        else if (o < x.len)
-          v[i] = ld_partial(x.src + o, x.len - o);
-        else
-          v[i] = make_uint4(0u, 0u, 0u, 0u);
-      }
-    }
-  };
 
   uint64_t u = (uint64_t)blockIdx.x * kWarpsPerCta + warp;
   Unit cur = get_unit(u);
-  if (cur.on) load_unit(cur);
+  if (cur.on) load_round(v, cur.src, cur.len, cur.mode, cur.r, lane_off);
   for (; u < nunits; u += nw) {
     const Unit nxt = get_unit(u + nw);
-    if (cur.on) {
-      const uint32_t base = (uint32_t)cur.r * kRoundBytes + lane_off;
-      if ((uint32_t)(cur.r + 1) * kRoundBytes <= cur.len) {
-        uint8_t* d = cur.dst + base;
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          st_stream_v4(d + i * 4 * kSegBytes, v[i]);
-          *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
-        }
-      } else {
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-          const uint32_t o = base + (uint32_t)i * 4 * kSegBytes;
-          if (o < cur.len) {
-            if (!kVerify || o + 16 <= cur.len)
-              st_stream_v4(cur.dst + o, v[i]);  // pack: zeros past len are owned padding
-            else
-              st_partial(cur.dst + o, v[i], cur.len - o);
-          }
-          *reinterpret_cast<uint4*>(tile_w + i * 4 * kRowPitch) = v[i];
-        }
-      }
-    }
+    if (cur.on) store_round<kOp>(v, cur.dst, cur.len, cur.r, lane_off, tile_w);
     __syncwarp();
-    if (nxt.on) load_unit(nxt);  // in flight during this unit's CRC
+    if (nxt.on) load_round(v, nxt.src, nxt.len, nxt.mode, nxt.r, lane_off);  // in flight during this unit's CRC
     if (cur.on) {
-#ifndef CHECL_EXP_SKIP_CRC
-      uint32_t crc = (lane == 0 && cur.r == 0) ? 0xFFFFFFFFu : 0u;
-      const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
+      if (!O::kCrc) {
+        if (cur.r == cur.nrounds - 1) finish_chunk<kOp>(p, cur.c, cur.src, cur.dst, cur.len, cur.pad, cur.nrounds, 0u, lane);
+      } else {
+        uint32_t crc = (lane == 0 && cur.r == 0) ? 0xFFFFFFFFu : 0u;
+        const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
 #pragma unroll
-      for (int g = 0; g < 8; ++g) crc = crc_step16(crc, row[g], tb, l4);
-      const uint32_t reg = warp_xor(lanepos_mul(crc, pb, l4));
-      // the unit's term in the chunk register: reg * x^(8*4096*(n-1-r)), lane i
-      // adding the x^i coefficient of reg times utab[k][i] = x^(8*4096*k) * x^i
-      const int k = cur.nrounds - 1 - cur.r;
-      const uint32_t term = warp_xor(((reg >> (31 - lane)) & 1u) ? utab[k * 32 + lane] : 0u);
-#else
-      const uint32_t term = 0;
-#endif
-      // one 64-bit atomicXor carries the term (low half) and this unit's bit in the
-      // finished-unit mask (high half): the unit that completes the mask holds the
-      // chunk register — no fence, no second pass
-      const unsigned long long mine = (unsigned long long)term | (1ull << (32 + cur.r));
-      unsigned long long old = 0;
-#ifdef CHECL_EXP_SKIP_ATOMIC
-      if (lane == 0 && term == 0x12345678u) old = atomicXor(&p.unit_acc[cur.c - p.c0], mine);
-#else
-      if (lane == 0) old = atomicXor(&p.unit_acc[cur.c - p.c0], mine);
-#endif
-      const unsigned long long now = __shfl_sync(0xFFFFFFFFu, old, 0) ^ mine;
-      if ((now >> 32) == (1ull << cur.nrounds) - 1) {
-        // last unit of the chunk: zero-padding correction, padding, CRC table / check
-        const uint32_t t = (uint32_t)now;
-        const uint32_t zp = (uint32_t)cur.nrounds * kRoundBytes - cur.len;
-        const uint32_t out = ~(zp ? gf_mul(t, p.inv_z[zp]) : t);
-        uint32_t pad_bad = 0;
-        if (cur.pad) {
-          if (!kVerify) {
-            const uint32_t start = (cur.len + 15u) & ~15u, end = cur.len + cur.pad;
-            for (uint32_t o = start + lane * 16u; o < end; o += 512u)
-              *reinterpret_cast<uint4*>(cur.dst + o) = make_uint4(0u, 0u, 0u, 0u);
-          } else {
-            for (uint32_t o = cur.len + lane; o < cur.len + cur.pad; o += 32u) pad_bad |= cur.src[o];
-          }
-        }
-        if (kVerify) pad_bad = __any_sync(0xFFFFFFFFu, pad_bad != 0);
-        if (lane == 0) {
-          if (!kVerify) {
-            p.crc[cur.c] = out;
-          } else if (out != p.crc[cur.c] || pad_bad) {
-            atomicMin(&p.status[0], (unsigned long long)cur.c);
-            atomicAdd(&p.status[1], 1ull);
-          }
+        for (int g = 0; g < 8; ++g) crc = crc_step16(crc, row[g], tb, l4);
+        const uint32_t reg = warp_xor(lanepos_mul(crc, pb, l4));
+        // the unit's term in the chunk register: reg * x^(8*4096*(n-1-r)), lane i
+        // adding the x^i coefficient of reg times utab[k][i] = x^(8*4096*k) * x^i
+        const int k = cur.nrounds - 1 - cur.r;
+        const uint32_t term = warp_xor(((reg >> (31 - lane)) & 1u) ? utab[k * 32 + lane] : 0u);
+        // one 64-bit atomicXor carries the term (low half) and this unit's bit in the
+        // finished-unit mask (high half): the unit that completes the mask holds the
+        // chunk register — no fence, no second pass
+        const unsigned long long mine = (unsigned long long)term | (1ull << (32 + cur.r));
+        unsigned long long old = 0;
+        if (lane == 0) old = atomicXor(&p.unit_acc[cur.c - p.c0], mine);
+        const unsigned long long now = __shfl_sync(0xFFFFFFFFu, old, 0) ^ mine;
+        if ((now >> 32) == (1ull << cur.nrounds) - 1) {
+          // every unit of the chunk has arrived: reset its word for the next launch
+          // (the accumulators are all zero between launches; no memset)
+          if (lane == 0) p.unit_acc[cur.c - p.c0] = 0ull;
+          finish_chunk<kOp>(p, cur.c, cur.src, cur.dst, cur.len, cur.pad, cur.nrounds, (uint32_t)now, lane);
         }
       }
     }
     __syncwarp();
     cur = nxt;
+  }
+}
+
+// ---- lookup tables: built once per device (DevState::init) -------------------
+// T_k[e] = CRC register of byte e followed by k zero bytes (zero init); H[j][v] =
+// (v << 4j) * x^(8*3968); fold[lvl][j][v] = (v << 4j) * x^(8*128*2^lvl); the sweep
+// kernel's position tables (v << 4j) * x^(8*128*(31-l)) and unit powers
+// x^(8*4096*k) * x^i. Lane-private copies: entry e of lane l at word e*32 + l.
+__global__ void build_tables_kernel(const TableParams tp, uint32_t* __restrict__ out) {
+  __shared__ uint32_t scratch[1024 + 128];
+  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
+    uint32_t r = (uint32_t)e;
+    for (int b = 0; b < 8; ++b) r = gf_mulx(r);
+    scratch[e] = r;
+  }
+  for (int i = threadIdx.x; i < 128; i += blockDim.x) scratch[1024 + i] = gf_mul((uint32_t)(i & 15) << (4 * (i >> 4)), tp.horner);
+  __syncthreads();
+  for (int e = threadIdx.x; e < 256; e += blockDim.x) {
+    uint32_t r = scratch[e];
+    for (int k = 1; k < 4; ++k) {
+      r = (r >> 8) ^ scratch[r & 0xFFu];
+      scratch[k * 256 + e] = r;
+    }
+  }
+  __syncthreads();
+  // slicing-by-4 super-tables: row-half h = (super-table, row e, half); A = [T3|T2], B = [T1|T0]
+  for (int i = threadIdx.x; i < 1024 * 32; i += blockDim.x) {
+    const int h = i >> 5, st = h >> 9, e = (h >> 1) & 255, half = h & 1;
+    const int k = 3 - (2 * st + half);
+    out[kTabOff + i] = scratch[k * 256 + e];
+  }
+  for (int i = threadIdx.x; i < 128 * 32; i += blockDim.x) out[kHornerOff + i] = scratch[1024 + (i >> 5)];
+  for (int i = threadIdx.x; i < kFoldWords; i += blockDim.x) {
+    const int lvl = i >> 7, j = (i >> 4) & 7, v = i & 15;
+    out[kFoldOff + i] = gf_mul((uint32_t)v << (4 * j), tp.fold[lvl]);
+  }
+  // position tables: entry (j, v) of lane l = (v << 4j) * C_l, from the four
+  // single-bit products C_l * x^(31-4j-t) (bit 4j+t of a reflected value is x^(31-4j-t))
+  for (int t = threadIdx.x; t < 8 * 32; t += blockDim.x) {
+    const int j = t >> 5, l = t & 31;
+    uint32_t b = tp.lanepow[l];
+    for (int m = 0; m < 31 - 4 * j - 3; ++m) b = gf_mulx(b);  // b = C * x^(28-4j)
+    uint32_t bit[4];
+    bit[3] = b;  // v bit 3 sits at position 4j+3 -> x^(28-4j)
+    for (int q = 2; q >= 0; --q) bit[q] = gf_mulx(bit[q + 1]);
+    for (int v = 0; v < 16; ++v) {
+      uint32_t e = 0;
+      for (int q = 0; q < 4; ++q)
+        if (v & (1 << q)) e ^= bit[q];
+      out[kPosOff + (j * 16 + v) * 32 + l] = e;
+    }
+  }
+  for (int t = threadIdx.x; t < kUnitWords; t += blockDim.x) {
+    uint32_t b = tp.unitpow[t >> 5];
+    for (int m = 0; m < (t & 31); ++m) b = gf_mulx(b);
+    out[kUnitOff + t] = b;
   }
 }
 
@@ -607,35 +600,51 @@ cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload
 
 size_t snapshot_smem_bytes() { return kSmemBytes; }
 
-cudaError_t snapshot_configure() {
-  cudaError_t e = cudaFuncSetAttribute(snapshot_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+template <int kOp>
+static cudaError_t configure_op() {
+  cudaError_t e = cudaFuncSetAttribute(snapshot_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(snapshot_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(sweep_kernel<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
-  if (e == cudaSuccess)
-    e = cudaFuncSetAttribute(sweep_kernel<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+    e = cudaFuncSetAttribute(sweep_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   return e;
 }
 
+cudaError_t snapshot_configure() {
+  cudaError_t e = configure_op<kOpPack>();
+  if (e == cudaSuccess) e = configure_op<kOpVerify>();
+  if (e == cudaSuccess) e = configure_op<kOpCrc>();
+  if (e == cudaSuccess) e = configure_op<kOpCheck>();
+  if (e == cudaSuccess) e = configure_op<kOpCopy>();
+  return e;
+}
+
+cudaError_t launch_build_tables(const TableParams& tp, uint32_t* out, cudaStream_t s) {
+  build_tables_kernel<<<1, 512, 0, s>>>(tp, out);
+  return cudaGetLastError();
+}
+
+template <int kOp>
+static void launch_op(const LaunchParams& p, unsigned ctas, cudaStream_t s, int kernel) {
+  if (kernel == 2)
+    sweep_kernel<kOp><<<ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
+  else
+    snapshot_kernel<kOp><<<ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
+}
+
 // kernel 1 = warp per chunk (snapshot_kernel), 2 = 4 KiB units swept by the grid
-// (sweep_kernel; needs p.unit_reg / unit_cnt / lanepow / unitpow and a zeroed
-// unit_cnt for the chunk range)
-cudaError_t launch_snapshot(bool verify, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel) {
+// (sweep_kernel; p.unit_acc must be zero for the chunk range when the op CRCs —
+// the kernel leaves it zero again)
+cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel) {
   const uint64_t chunks = p.c1 - p.c0;
   if (chunks == 0) return cudaSuccess;
   uint64_t ctas = kernel == 2 ? (chunks * 16 + kWarpsPerCta - 1) / kWarpsPerCta : (chunks + kWarpsPerCta - 1) / kWarpsPerCta;
   if (ctas > (uint64_t)n_sms) ctas = (uint64_t)n_sms;
-  if (kernel == 2) {
-    if (verify)
-      sweep_kernel<true><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
-    else
-      sweep_kernel<false><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
-  } else {
-    if (verify)
-      snapshot_kernel<true><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
-    else
-      snapshot_kernel<false><<<(unsigned)ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
+  switch (op) {
+    case kOpPack: launch_op<kOpPack>(p, (unsigned)ctas, s, kernel); break;
+    case kOpVerify: launch_op<kOpVerify>(p, (unsigned)ctas, s, kernel); break;
+    case kOpCrc: launch_op<kOpCrc>(p, (unsigned)ctas, s, kernel); break;
+    case kOpCheck: launch_op<kOpCheck>(p, (unsigned)ctas, s, kernel); break;
+    case kOpCopy: launch_op<kOpCopy>(p, (unsigned)ctas, s, kernel); break;
+    default: return cudaErrorInvalidValue;
   }
   return cudaGetLastError();
 }
