@@ -235,6 +235,19 @@ done:
   return st;
 }
 
+/* Span of chunk j of manifest record b (FORMAT.md "Span of a chunk"): its bytes
+ * plus, for a buffer's last chunk, the padding it owns, in full-payload offsets. */
+static void chunk_span(const uint8_t* img, uint64_t n, uint64_t b, uint64_t j, uint64_t full_payload,
+                       uint64_t* start, uint64_t* stop) {
+  const uint8_t* r = img + O_HEADER + O_RECORD * b;
+  uint64_t size = get_u64(r + 8), off = get_u64(r + 16);
+  *start = off + (uint64_t)O_CHUNK * j;
+  if (j + 1 < chunks_of(size))
+    *stop = *start + O_CHUNK;
+  else
+    *stop = b + 1 < n ? get_u64(r + O_RECORD + 16) : full_payload;
+}
+
 /* ------------------------------------------------------------------------ */
 /* Restart (L16 restart steps 2-3)                                           */
 /* ------------------------------------------------------------------------ */
@@ -250,11 +263,14 @@ int oracle_validate(const uint8_t* img, size_t len, oracle_report* rep) {
   report_init(rep);
   if (!img || len < O_HEADER) return ORACLE_BAD_IMAGE;
   if (memcmp(img, "CHECLIM1", 8) != 0) return ORACLE_BAD_IMAGE;
+  uint32_t flags = get_u32(img + 84); /* 0 = full, 1 = incremental */
   if (get_u32(img + 8) != 1 || get_u32(img + 12) != O_HEADER || get_u32(img + 16) != O_CHUNK ||
-      get_u32(img + 20) != O_ALIGN || get_u64(img + 40) != O_HEADER || get_u32(img + 84) != 0)
+      get_u32(img + 20) != O_ALIGN || get_u64(img + 40) != O_HEADER || flags > 1)
     return ORACLE_BAD_IMAGE;
-  for (int i = 96; i < 124; ++i)
-    if (img[i] != 0) return ORACLE_BAD_IMAGE;
+  for (int i = 96; i < 124; ++i) {
+    int used = flags == 1 && ((i >= 96 && i < 108) || (i >= 112 && i < 120)); /* base_epoch, base_table_crc, n_present */
+    if (!used && img[i] != 0) return ORACLE_BAD_IMAGE;
+  }
   uint64_t n = get_u64(img + 24), nch = get_u64(img + 32);
   uint64_t crc_off = get_u64(img + 48), payload_off = get_u64(img + 56);
   uint64_t payload_bytes = get_u64(img + 64), image_bytes = get_u64(img + 72);
@@ -263,14 +279,15 @@ int oracle_validate(const uint8_t* img, size_t len, oracle_report* rep) {
   if (n > (UINT64_MAX - O_HEADER) / O_RECORD) return ORACLE_BAD_IMAGE;
   if (crc_off != O_HEADER + O_RECORD * n) return ORACLE_BAD_IMAGE;
   if (nch > (UINT64_MAX - crc_off) / 4u) return ORACLE_BAD_IMAGE;
+  uint64_t map_bytes = flags == 1 ? nch / 8 + (nch % 8 ? 1 : 0) : 0; /* present bitmap */
   uint64_t want_payload_off;
-  if (!align_ok(crc_off + 4u * nch, O_PAYLOAD_ALIGN, &want_payload_off)) return ORACLE_BAD_IMAGE;
+  if (!align_ok(crc_off + 4u * nch + map_bytes, O_PAYLOAD_ALIGN, &want_payload_off)) return ORACLE_BAD_IMAGE;
   if (payload_off != want_payload_off) return ORACLE_BAD_IMAGE;
   uint64_t want_image;
   if (!add_ok(payload_off, payload_bytes, &want_image) || image_bytes != want_image) return ORACLE_BAD_IMAGE;
   if ((uint64_t)len < image_bytes) return ORACLE_BAD_IMAGE;
   if (get_u32(img + 124) != meta_crc_of(img, payload_off)) return ORACLE_BAD_IMAGE;
-  for (uint64_t i = crc_off + 4u * nch; i < payload_off; ++i)
+  for (uint64_t i = crc_off + 4u * nch + map_bytes; i < payload_off; ++i)
     if (img[i] != 0) return ORACLE_BAD_IMAGE;
   /* records */
   uint64_t off = 0, end = 0, chunk = 0, prev = 0;
@@ -286,7 +303,27 @@ int oracle_validate(const uint8_t* img, size_t len, oracle_report* rep) {
     prev = h;
   }
   if (chunk != nch) return ORACLE_BAD_IMAGE;
-  if (payload_bytes != (n ? end : 0)) return ORACLE_BAD_IMAGE;
+  uint64_t full_payload = n ? end : 0;
+  if (flags == 0 && payload_bytes != full_payload) return ORACLE_BAD_IMAGE;
+  if (flags == 1) {
+    /* present bitmap: unused bits zero, popcount = n_present, spans sum to payload_bytes */
+    const uint8_t* map = img + crc_off + 4u * nch;
+    for (uint64_t k = nch; k < map_bytes * 8; ++k)
+      if (map[k / 8] & (1u << (k % 8))) return ORACLE_BAD_IMAGE;
+    uint64_t n_present = 0, sum = 0;
+    for (uint64_t b = 0; b < n; ++b) {
+      uint64_t nb = chunks_of(get_u64(img + O_HEADER + O_RECORD * b + 8));
+      uint64_t first = get_u64(img + O_HEADER + O_RECORD * b + 24);
+      for (uint64_t j = 0; j < nb; ++j) {
+        if (!(map[(first + j) / 8] & (1u << ((first + j) % 8)))) continue;
+        uint64_t start, stop;
+        chunk_span(img, n, b, j, full_payload, &start, &stop);
+        n_present++;
+        sum += stop - start;
+      }
+    }
+    if (n_present != get_u64(img + 112) || sum != payload_bytes) return ORACLE_BAD_IMAGE;
+  }
   rep->n_buffers = n;
   rep->payload_bytes = payload_bytes;
   rep->n_chunks = nch;
@@ -301,6 +338,7 @@ int oracle_restore(const uint8_t* img, size_t len, uint8_t* out_bytes, size_t ou
   /* Step r1: header + manifest */
   int st = oracle_validate(img, len, rep);
   if (st) return st;
+  if (get_u32(img + 84) != 0) return ORACLE_BAD_IMAGE; /* a delta restores only through merge */
   uint64_t n = rep->n_buffers;
   uint64_t crc_off = get_u64(img + 48), payload_off = get_u64(img + 56);
   uint64_t payload_bytes = rep->payload_bytes;
@@ -346,5 +384,158 @@ int oracle_restore(const uint8_t* img, size_t len, uint8_t* out_bytes, size_t ou
     if (size) memcpy(out_bytes + pos, payload + off, size);
     pos += size;
   }
+  return ORACLE_SUCCESS;
+}
+
+/* ------------------------------------------------------------------------ */
+/* Incremental checkpoint (FORMAT.md "Incremental images"; PAPER.md L45      */
+/* §IV-D future work: write only what was updated since the last checkpoint) */
+/* ------------------------------------------------------------------------ */
+
+static uint32_t table_crc_of(const uint8_t* img) {
+  uint64_t nch = get_u64(img + 32), crc_off = get_u64(img + 48);
+  return oracle_crc32c(img + crc_off, 4u * nch);
+}
+
+int oracle_checkpoint_incremental(const oracle_buffer* bufs, size_t n, int32_t device, uint64_t epoch,
+                                  const uint8_t* base, size_t base_len, uint8_t* out, size_t out_cap,
+                                  uint64_t* out_len) {
+  oracle_report brep;
+  int st;
+  if (!out_len) return ORACLE_INVALID_VALUE;
+  /* the base must be a valid image (full or incremental) */
+  st = oracle_validate(base, base_len, &brep);
+  if (st) return st;
+
+  /* Step 1: the full image of the registry now (the definition of its content). */
+  oracle_layout L;
+  st = oracle_layout_of(bufs, n, &L);
+  if (st) return st;
+  uint8_t* full = (uint8_t*)malloc(L.image_bytes ? L.image_bytes : 1);
+  if (!full) return ORACLE_OUT_OF_HOST_MEMORY;
+  st = oracle_checkpoint(bufs, n, device, epoch, full, L.image_bytes);
+  if (st) {
+    free(full);
+    return st;
+  }
+
+  /* Step 2: same layout as the base? (manifest, chunk count, device) — else full. */
+  int same = get_u64(base + 32) == L.n_chunks && get_u64(base + 48) == L.crc_off &&
+             get_u32(base + 80) == (uint32_t)device &&
+             memcmp(base + O_HEADER, full + O_HEADER, L.crc_off - O_HEADER) == 0;
+  if (!same) {
+    *out_len = L.image_bytes;
+    if (out_cap < L.image_bytes || !out) {
+      free(full);
+      return ORACLE_INVALID_VALUE;
+    }
+    memcpy(out, full, L.image_bytes);
+    free(full);
+    return ORACLE_SUCCESS;
+  }
+
+  /* Step 3: chunk k is present iff its CRC differs from the base's entry. */
+  uint64_t nch = L.n_chunks, crc_off = L.crc_off;
+  uint64_t map_bytes = nch / 8 + (nch % 8 ? 1 : 0);
+  uint64_t n_present = 0, payload = 0;
+  for (uint64_t b = 0; b < L.n_buffers; ++b) {
+    uint64_t nb = chunks_of(get_u64(full + O_HEADER + O_RECORD * b + 8));
+    uint64_t first = get_u64(full + O_HEADER + O_RECORD * b + 24);
+    for (uint64_t j = 0; j < nb; ++j) {
+      uint64_t k = first + j;
+      if (get_u32(full + crc_off + 4u * k) == get_u32(base + crc_off + 4u * k)) continue;
+      uint64_t start, stop;
+      chunk_span(full, L.n_buffers, b, j, L.payload_bytes, &start, &stop);
+      n_present++;
+      payload += stop - start;
+    }
+  }
+
+  /* Step 4: layout of the delta. */
+  uint64_t payload_off = 0;
+  if (!align_ok(crc_off + 4u * nch + map_bytes, O_PAYLOAD_ALIGN, &payload_off)) {
+    free(full);
+    return ORACLE_INVALID_VALUE;
+  }
+  uint64_t image_bytes = payload_off + payload;
+  *out_len = image_bytes;
+  if (out_cap < image_bytes || !out) {
+    free(full);
+    return ORACLE_INVALID_VALUE;
+  }
+  memset(out, 0, image_bytes);
+
+  /* Step 5: header (the full image's, then the incremental fields), manifest,
+   * CRC table of every chunk, bitmap, and the present spans in ascending order. */
+  memcpy(out, full, O_HEADER);
+  put_u64(out + 56, payload_off);
+  put_u64(out + 64, payload);
+  put_u64(out + 72, image_bytes);
+  put_u32(out + 84, 1);
+  put_u64(out + 96, get_u64(base + 88));
+  put_u32(out + 104, table_crc_of(base));
+  put_u64(out + 112, n_present);
+  memcpy(out + O_HEADER, full + O_HEADER, crc_off - O_HEADER);
+  memcpy(out + crc_off, full + crc_off, 4u * nch);
+  uint8_t* map = out + crc_off + 4u * nch;
+  uint64_t pos = payload_off;
+  for (uint64_t b = 0; b < L.n_buffers; ++b) {
+    uint64_t nb = chunks_of(get_u64(full + O_HEADER + O_RECORD * b + 8));
+    uint64_t first = get_u64(full + O_HEADER + O_RECORD * b + 24);
+    for (uint64_t j = 0; j < nb; ++j) {
+      uint64_t k = first + j;
+      if (get_u32(full + crc_off + 4u * k) == get_u32(base + crc_off + 4u * k)) continue;
+      uint64_t start, stop;
+      chunk_span(full, L.n_buffers, b, j, L.payload_bytes, &start, &stop);
+      map[k / 8] |= (uint8_t)(1u << (k % 8));
+      memcpy(out + pos, full + L.payload_off + start, stop - start);
+      pos += stop - start;
+    }
+  }
+  put_u32(out + 124, meta_crc_of(out, payload_off));
+  free(full);
+  return ORACLE_SUCCESS;
+}
+
+int oracle_merge(const uint8_t* full, size_t full_len, const uint8_t* delta, size_t delta_len, uint8_t* out,
+                 size_t out_cap, uint64_t* out_len) {
+  oracle_report fr, dr;
+  if (!out_len) return ORACLE_INVALID_VALUE;
+  if (oracle_validate(full, full_len, &fr) || oracle_validate(delta, delta_len, &dr)) return ORACLE_BAD_IMAGE;
+  if (get_u32(full + 84) != 0 || get_u32(delta + 84) != 1) return ORACLE_BAD_IMAGE;
+  /* the link: base epoch, base CRC-table CRC, identical manifest and device */
+  uint64_t crc_off = get_u64(full + 48), nch = get_u64(full + 32);
+  if (get_u64(delta + 96) != get_u64(full + 88) || get_u32(delta + 104) != table_crc_of(full) ||
+      get_u64(delta + 32) != nch || get_u64(delta + 48) != crc_off || get_u32(delta + 80) != get_u32(full + 80) ||
+      memcmp(delta + O_HEADER, full + O_HEADER, crc_off - O_HEADER) != 0)
+    return ORACLE_BAD_IMAGE;
+  uint64_t image_bytes = get_u64(full + 72), payload_off = get_u64(full + 56), payload_bytes = get_u64(full + 64);
+  *out_len = image_bytes;
+  if (out_cap < image_bytes || !out) return ORACLE_INVALID_VALUE;
+  /* F's bytes, then D's header with flags 0 and the full-image fields, D's CRC table */
+  memcpy(out, full, image_bytes);
+  memcpy(out, delta, O_HEADER);
+  put_u32(out + 84, 0);
+  put_u64(out + 56, payload_off);
+  put_u64(out + 64, payload_bytes);
+  put_u64(out + 72, image_bytes);
+  memset(out + 96, 0, 28);
+  memcpy(out + crc_off, delta + crc_off, 4u * nch);
+  /* every present chunk's span replaced by D's, in ascending order */
+  const uint8_t* map = delta + crc_off + 4u * nch;
+  uint64_t n = get_u64(full + 24), pos = get_u64(delta + 56);
+  for (uint64_t b = 0; b < n; ++b) {
+    uint64_t nb = chunks_of(get_u64(full + O_HEADER + O_RECORD * b + 8));
+    uint64_t first = get_u64(full + O_HEADER + O_RECORD * b + 24);
+    for (uint64_t j = 0; j < nb; ++j) {
+      uint64_t k = first + j;
+      if (!(map[k / 8] & (1u << (k % 8)))) continue;
+      uint64_t start, stop;
+      chunk_span(full, n, b, j, payload_bytes, &start, &stop);
+      memcpy(out + payload_off + start, delta + pos, stop - start);
+      pos += stop - start;
+    }
+  }
+  put_u32(out + 124, meta_crc_of(out, payload_off));
   return ORACLE_SUCCESS;
 }

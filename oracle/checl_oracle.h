@@ -72,10 +72,12 @@ typedef struct {
   uint64_t first_bad_handle, first_bad_chunk;
 } oracle_report;
 
-/* Header + manifest validation only (FORMAT.md "Validation order" step 1). */
+/* Header + manifest validation only (FORMAT.md "Validation order" step 1), for
+ * full (flags 0) and incremental (flags 1) images. */
 int oracle_validate(const uint8_t* img, size_t len, oracle_report* rep);
 
-/* Restart (L16 restart steps 2-3): validate, verify every chunk, and on success
+/* Restart (L16 restart steps 2-3) of a full image (an incremental image alone is
+ * ORACLE_BAD_IMAGE: chains restore through oracle_merge): validate, verify every chunk, and on success
  * copy every buffer's bytes, in manifest order, into out_bytes (concatenated,
  * no padding) and the records into out_handles / out_sizes / out_flags (each
  * n_buffers long). Capacities are checked: ORACLE_INVALID_VALUE when too small.
@@ -83,6 +85,27 @@ int oracle_validate(const uint8_t* img, size_t len, oracle_report* rep);
 int oracle_restore(const uint8_t* img, size_t len, uint8_t* out_bytes,
                    size_t out_bytes_cap, uint64_t* out_handles, uint64_t* out_sizes,
                    uint32_t* out_flags, size_t out_cap, oracle_report* rep);
+
+/* ---- Incremental images (FORMAT.md "Incremental images") ----
+ * PAPER.md L45 §IV-D (future work): "only the OpenCL objects updated since the
+ * last checkpoint need to be written". Unit = 64 KiB chunk; updated = its CRC32C
+ * differs from the base image's entry (reading 21). */
+
+/* Writes into out[0, *out_len) the incremental image of the registry at `epoch`
+ * relative to `base` (a full or incremental image). When base's manifest, chunk
+ * count or device differ from this registry's, the output is the full image
+ * (flags 0) instead. ORACLE_BAD_IMAGE if base does not validate;
+ * ORACLE_INVALID_VALUE if out_cap < the size needed (*out_len is set to it). */
+int oracle_checkpoint_incremental(const oracle_buffer* bufs, size_t n, int32_t device, uint64_t epoch,
+                                  const uint8_t* base, size_t base_len, uint8_t* out, size_t out_cap,
+                                  uint64_t* out_len);
+
+/* merge(F, D): the full image of D's epoch from full image F and delta D whose
+ * link names F. ORACLE_BAD_IMAGE if either does not validate, F is not full, D is
+ * not incremental, or the link (base epoch, base table CRC, manifest) does not
+ * match; ORACLE_INVALID_VALUE if out_cap is too small (*out_len set). */
+int oracle_merge(const uint8_t* full, size_t full_len, const uint8_t* delta, size_t delta_len, uint8_t* out,
+                 size_t out_cap, uint64_t* out_len);
 
 #ifdef __cplusplus
 }

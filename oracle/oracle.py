@@ -157,3 +157,56 @@ def restore(img) -> Tuple[int, dict, List[Entry]]:
         ents.append(Entry(int(hs[i]), out[pos:pos + s].copy(), int(fs[i])))
         pos += s
     return 0, r.as_dict(), ents
+
+
+def _sigs_incremental(L):
+    if getattr(L, "_incr", False):
+        return L
+    L.oracle_checkpoint_incremental.argtypes = [C.POINTER(_Buf), C.c_size_t, C.c_int32, C.c_uint64, C.c_void_p,
+                                                C.c_size_t, C.c_void_p, C.c_size_t, C.POINTER(C.c_uint64)]
+    L.oracle_merge.argtypes = [C.c_void_p, C.c_size_t, C.c_void_p, C.c_size_t, C.c_void_p, C.c_size_t,
+                               C.POINTER(C.c_uint64)]
+    L._incr = True
+    return L
+
+
+def checkpoint_incremental(entries: Sequence[Entry], base, device: int = 0, epoch: int = 0) -> np.ndarray:
+    """Incremental image of the registry relative to `base` (FORMAT.md "Incremental
+    images"); the full image when the layout differs from the base's."""
+    L = _sigs_incremental(lib())
+    arr, keep = _bufs(entries, device)
+    b = _u8(base)
+    need = C.c_uint64(0)
+    st = L.oracle_checkpoint_incremental(arr, len(entries), device, epoch, b.ctypes.data if b.size else None, b.size,
+                                         None, 0, C.byref(need))
+    if st != INVALID_VALUE or need.value == 0:  # cap 0: reports the size it needs
+        raise ValueError(f"oracle_checkpoint_incremental status {st}")
+    out = np.empty(max(1, need.value), dtype=np.uint8)
+    st = L.oracle_checkpoint_incremental(arr, len(entries), device, epoch, b.ctypes.data if b.size else None, b.size,
+                                         out.ctypes.data, out.size, C.byref(need))
+    if st:
+        raise ValueError(f"oracle_checkpoint_incremental status {st}")
+    return out[: need.value]
+
+
+def merge(full, delta) -> Tuple[int, np.ndarray]:
+    """(status, merge(F, D)) — the full image of D's epoch (FORMAT.md "Merge")."""
+    L = _sigs_incremental(lib())
+    f, d = _u8(full), _u8(delta)
+    need = C.c_uint64(0)
+    st = L.oracle_merge(f.ctypes.data, f.size, d.ctypes.data, d.size, None, 0, C.byref(need))
+    if st != INVALID_VALUE:
+        return int(st), np.zeros(0, np.uint8)
+    out = np.empty(max(1, need.value), dtype=np.uint8)
+    st = L.oracle_merge(f.ctypes.data, f.size, d.ctypes.data, d.size, out.ctypes.data, out.size, C.byref(need))
+    return int(st), out[: need.value]
+
+
+def restore_chain(chain) -> Tuple[int, dict, List[Entry]]:
+    """Restores [F, D1, ..., Dn] as restore(merge(...merge(F, D1)..., Dn))."""
+    cur = _u8(chain[0])
+    for d in chain[1:]:
+        st, cur = merge(cur, d)
+        if st:
+            return st, {}, []
+    return restore(cur)
