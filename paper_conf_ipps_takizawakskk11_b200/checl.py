@@ -43,6 +43,7 @@ EXPORTS = (
     "checl_image_view", "checl_image_info", "checl_image_wrap", "checl_image_to_host", "checl_image_free",
     "checl_restore", "checl_migrate", "checl_last_timing", "checl_status_string", "checl_last_cuda_error",
     "checl_version", "checl_debug_fill", "checl_debug_compare", "checl_debug_corrupt",
+    "checl_checkpoint_incremental", "checl_restore_chain", "checl_image_merge",
 )
 
 
@@ -92,6 +93,9 @@ def _load() -> C.CDLL:
         "checl_debug_fill": [C.c_int, V, SZ, U64, U64, C.c_int, V],
         "checl_debug_compare": [C.c_int, V, V, SZ, C.POINTER(U64)],
         "checl_debug_corrupt": [P, U64, C.c_uint8],
+        "checl_checkpoint_incremental": [P, C.c_int, V, U64, P, PP],
+        "checl_restore_chain": [P, C.POINTER(C.c_void_p), U32, C.c_int, V, C.POINTER(_Report)],
+        "checl_image_merge": [P, P, PP],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -184,6 +188,23 @@ class Image:
         arr = np.ctypeslib.as_array(C.cast(b, C.POINTER(C.c_uint8)), shape=(n.value,))
         arr.flags.writeable = False
         return arr
+
+    def merge(self, delta: "Image") -> "Image":
+        """FORMAT.md "Merge": the full image of `delta`'s epoch (self = the full base)."""
+        out = C.c_void_p()
+        _check(lib.checl_image_merge(self.handle, delta.handle, C.byref(out)), "checl_image_merge")
+        return Image(out.value)
+
+    def header(self) -> dict:
+        """Header fields (FORMAT.md) read from the image bytes."""
+        v = self.view()
+        u32 = lambda o: int(v[o:o + 4].view("<u4")[0])  # noqa: E731
+        u64 = lambda o: int(v[o:o + 8].view("<u8")[0])  # noqa: E731
+        h = {"n_buffers": u64(24), "n_chunks": u64(32), "crc_off": u64(48), "payload_off": u64(56),
+             "payload_bytes": u64(64), "image_bytes": u64(72), "device": u32(80), "flags": u32(84), "epoch": u64(88)}
+        if h["flags"] == 1:
+            h.update(base_epoch=u64(96), base_table_crc=u32(104), n_present=u64(112))
+        return h
 
     def to_host(self) -> "Image":
         out = C.c_void_p()
@@ -326,6 +347,23 @@ class Context:
         _check(lib.checl_checkpoint_device(self._p, device, _stream_ptr(stream), epoch, C.byref(out)),
                "checl_checkpoint_device")
         return Image(out.value)
+
+    def checkpoint_incremental(self, device: int, base: Image, stream=None, epoch: int = 0) -> Image:
+        """Incremental checkpoint (L45 future work; FORMAT.md "Incremental images"):
+        only chunks whose CRC32C differs from `base`'s table are drained."""
+        out = C.c_void_p()
+        _check(lib.checl_checkpoint_incremental(self._p, device, _stream_ptr(stream), epoch, base.handle, C.byref(out)),
+               "checl_checkpoint_incremental")
+        return Image(out.value)
+
+    def restore_chain(self, chain, device: int, stream=None) -> Report:
+        """Restores [full, delta1, ..., deltaN] (all or nothing)."""
+        arr = (C.c_void_p * len(chain))(*[im.handle.value for im in chain])
+        r = _Report()
+        st = lib.checl_restore_chain(self._p, arr, len(chain), device, _stream_ptr(stream), C.byref(r))
+        rep = Report._from(r)
+        _check(st, "checl_restore_chain", rep)
+        return rep
 
     def restore(self, image: Image, device: int, stream=None) -> Report:
         """Restart steps 2-3 (L16): verify every chunk, then rebind every handle."""

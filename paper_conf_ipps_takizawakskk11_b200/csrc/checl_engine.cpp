@@ -32,6 +32,10 @@ cudaError_t launch_build_tables(const TableParams& tp, uint32_t* out, cudaStream
 cudaError_t launch_fill(uint8_t* ptr, uint64_t bytes, uint64_t key, int kind, int n_sms, cudaStream_t s);
 cudaError_t launch_compare(const uint8_t* a, const uint8_t* b, uint64_t bytes, unsigned long long* n_diff, int n_sms,
                            cudaStream_t s);
+cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, const uint32_t* crc_base, uint64_t n,
+                              uint32_t* map_words, ChunkDesc* cdesc, unsigned long long* totals, cudaStream_t s);
+cudaError_t launch_delta_stages(const ChunkDesc* cdesc, const unsigned long long* totals, uint64_t W, uint64_t n_stages,
+                                unsigned long long* first, unsigned long long* lo, cudaStream_t s);
 cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload_bytes, uint64_t n_chunks,
                           ChunkDesc* out, int n_sms, cudaStream_t s);
 uint32_t host_crc32c_update(uint32_t crc, const void* data, size_t n);
@@ -230,6 +234,12 @@ struct DevState {
   DevBuf<BufferRecord> recs_scratch;
   DevBuf<unsigned long long> status;
   DevBuf<unsigned long long> unit_acc;
+  // incremental checkpoint (f1): base CRC table, bitmap words, compacted chunk
+  // list, [n_present, bytes], stage table
+  DevBuf<uint32_t> base_crc, map_words;
+  DevBuf<ChunkDesc> cdesc;
+  DevBuf<unsigned long long> dtotals, stage_first, stage_lo;
+  PinnedBuf<unsigned long long> h_dtab;
   // 1 = warp per chunk (throughput), 2 = 4 KiB units swept by the grid (latency of
   // small launches); 0 = by size; env CHECL_KERNEL=1|2 forces one
   int kernel = 0;
@@ -277,6 +287,13 @@ struct DevState {
     status.release();
     unit_acc.release();
     tables.release();
+    base_crc.release();
+    map_words.release();
+    cdesc.release();
+    dtotals.release();
+    stage_first.release();
+    stage_lo.release();
+    h_dtab.release();
     plan.d_desc.release();
     h_status.release();
     h_recs.release();
@@ -577,19 +594,41 @@ bool add_ok(uint64_t a, uint64_t b, uint64_t* out) {
 
 struct Parsed {
   int source_device = 0;
-  Layout L;
+  Layout L;  // L.payload_bytes = the header field (the compacted payload of a delta)
   std::vector<BufRec> bufs;
+  uint32_t flags = 0;          // 0 full, 1 incremental (FORMAT.md "Incremental images")
+  uint64_t epoch = 0, full_payload = 0, map_off = 0, map_bytes = 0, n_present = 0;
+  uint64_t base_epoch = 0;
+  uint32_t base_table_crc = 0;
 };
+
+// Full-payload span [start, stop) of chunk j of buffer b: its bytes plus, for the
+// buffer's last chunk, the padding it owns (FORMAT.md "Span of a chunk").
+void chunk_span(const std::vector<BufRec>& bufs, size_t b, uint64_t j, uint64_t full_payload, uint64_t* start,
+                uint64_t* stop) {
+  *start = bufs[b].off + (uint64_t)kChunkBytes * j;
+  if (j + 1 < chunks_of(bufs[b].size))
+    *stop = *start + kChunkBytes;
+  else
+    *stop = b + 1 < bufs.size() ? bufs[b + 1].off : full_payload;
+}
+
+bool bit_set(const uint8_t* map, uint64_t k) { return (map[k >> 3] >> (k & 7)) & 1u; }
 
 checl_status parse_image(const uint8_t* img, size_t len, bool meta_only, Parsed* out) {
   // meta_only: `len` covers [0, payload_off) only (device image mirror)
   if (!img || len < kHeaderBytes) return CHECL_ERR_BAD_IMAGE;
   if (std::memcmp(img, "CHECLIM1", 8) != 0) return CHECL_ERR_BAD_IMAGE;
+  const uint32_t flags = get_u32(img + 84);
   if (get_u32(img + 8) != 1 || get_u32(img + 12) != kHeaderBytes || get_u32(img + 16) != kChunkBytes ||
-      get_u32(img + 20) != kBufferAlign || get_u64(img + 40) != kHeaderBytes || get_u32(img + 84) != 0)
+      get_u32(img + 20) != kBufferAlign || get_u64(img + 40) != kHeaderBytes || flags > 1)
     return CHECL_ERR_BAD_IMAGE;
-  for (int i = 96; i < 124; ++i)
-    if (img[i]) return CHECL_ERR_BAD_IMAGE;
+  if (flags == 0) {
+    for (int i = 96; i < 124; ++i)
+      if (img[i]) return CHECL_ERR_BAD_IMAGE;
+  } else if (get_u32(img + 108) != 0 || get_u32(img + 120) != 0) {
+    return CHECL_ERR_BAD_IMAGE;
+  }
   const uint64_t n = get_u64(img + 24), nch = get_u64(img + 32);
   Layout L;
   L.n_chunks = nch;
@@ -599,13 +638,14 @@ checl_status parse_image(const uint8_t* img, size_t len, bool meta_only, Parsed*
   L.image_bytes = get_u64(img + 72);
   if (n > (~0ull - kHeaderBytes) / kRecordBytes || L.crc_off != kHeaderBytes + kRecordBytes * n)
     return CHECL_ERR_BAD_IMAGE;
-  if (nch > (~0ull - L.crc_off - kPayloadAlign) / 4) return CHECL_ERR_BAD_IMAGE;
-  if (L.payload_off != align_up(L.crc_off + 4 * nch, kPayloadAlign)) return CHECL_ERR_BAD_IMAGE;
+  if (nch > (~0ull - L.crc_off - kPayloadAlign) / 5) return CHECL_ERR_BAD_IMAGE;
+  const uint64_t map_bytes = flags ? (nch + 7) / 8 : 0;
+  if (L.payload_off != align_up(L.crc_off + 4 * nch + map_bytes, kPayloadAlign)) return CHECL_ERR_BAD_IMAGE;
   uint64_t want;
   if (!add_ok(L.payload_off, L.payload_bytes, &want) || want != L.image_bytes) return CHECL_ERR_BAD_IMAGE;
   if ((uint64_t)len < (meta_only ? L.payload_off : L.image_bytes)) return CHECL_ERR_BAD_IMAGE;
   if (get_u32(img + 124) != meta_crc(img, L.payload_off)) return CHECL_ERR_BAD_IMAGE;
-  for (uint64_t i = L.crc_off + 4 * nch; i < L.payload_off; ++i)
+  for (uint64_t i = L.crc_off + 4 * nch + map_bytes; i < L.payload_off; ++i)
     if (img[i]) return CHECL_ERR_BAD_IMAGE;
   const int device = (int32_t)get_u32(img + 80);
   std::vector<BufRec> bufs(n);
@@ -625,9 +665,35 @@ checl_status parse_image(const uint8_t* img, size_t len, bool meta_only, Parsed*
     bufs[b] = BufRec{h, size, off, get_u64(r + 24), get_u32(r + 32), nullptr};
     prev = h;
   }
-  if (chunk != nch || L.payload_bytes != (n ? end : 0)) return CHECL_ERR_BAD_IMAGE;
+  const uint64_t full_payload = n ? end : 0;
+  if (chunk != nch || (flags == 0 && L.payload_bytes != full_payload)) return CHECL_ERR_BAD_IMAGE;
   // the kernels address chunk offsets as u32 multiples of 256 (1 TiB payload)
-  if (L.payload_bytes > (1ull << 40)) return CHECL_ERR_BAD_IMAGE;
+  if (full_payload > (1ull << 40)) return CHECL_ERR_BAD_IMAGE;
+  if (flags == 1) {  // present bitmap: unused bits zero, popcount, spans
+    const uint8_t* map = img + L.crc_off + 4 * nch;
+    for (uint64_t k = nch; k < map_bytes * 8; ++k)
+      if (bit_set(map, k)) return CHECL_ERR_BAD_IMAGE;
+    uint64_t np = 0, sum = 0;
+    for (size_t b = 0; b < bufs.size(); ++b) {
+      const uint64_t nb = chunks_of(bufs[b].size);
+      for (uint64_t j = 0; j < nb; ++j) {
+        if (!bit_set(map, bufs[b].first_chunk + j)) continue;
+        uint64_t a, z;
+        chunk_span(bufs, b, j, full_payload, &a, &z);
+        ++np;
+        sum += z - a;
+      }
+    }
+    if (np != get_u64(img + 112) || sum != L.payload_bytes) return CHECL_ERR_BAD_IMAGE;
+    out->n_present = np;
+    out->base_epoch = get_u64(img + 96);
+    out->base_table_crc = get_u32(img + 104);
+  }
+  out->flags = flags;
+  out->epoch = get_u64(img + 88);
+  out->full_payload = full_payload;
+  out->map_off = L.crc_off + 4 * nch;
+  out->map_bytes = map_bytes;
   out->source_device = device;
   out->L = L;
   out->bufs = std::move(bufs);
@@ -827,7 +893,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
 void set_report(checl_report* rep, const Parsed& P, uint64_t n_bad, uint64_t first_bad) {
   if (!rep) return;
   rep->n_buffers = P.bufs.size();
-  rep->payload_bytes = P.L.payload_bytes;
+  rep->payload_bytes = P.full_payload;
   rep->n_chunks = P.L.n_chunks;
   rep->n_bad_chunks = n_bad;
   rep->first_bad_chunk = n_bad ? first_bad : ~0ull;
@@ -919,6 +985,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   const bool dev_img = img->location == CHECL_IMAGE_DEVICE;
   checl_status st = parse_image(img->host, dev_img ? img->payload_off : img->image_bytes, dev_img, &P);
   if (st) return st;
+  if (P.flags != 0) return CHECL_ERR_BAD_IMAGE;  // a delta restores only as part of a chain
   if (rep) set_report(rep, P, 0, 0);
 
   // r2: re-create the buffers: one allocation laid out like the payload
@@ -1033,6 +1100,335 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   (void)in_migrate;
   const double tc = now_ms();
   commit(ctx, P, device, arena);
+  tm.commit_ms = now_ms() - tc;
+  tm.total_ms = now_ms() - t0;
+  ctx->last = tm;
+  return CHECL_SUCCESS;
+}
+
+// -- incremental checkpoint (f1; §IV-D; FORMAT.md "Incremental images") --
+
+// True when `base` describes the same registry layout as plan P (identical manifest
+// bytes, chunk count and device): only then is a delta written.
+bool same_layout(const uint8_t* base, const Parsed& B, const Plan& P, int device) {
+  return B.L.n_chunks == P.n_chunks && B.L.crc_off == P.crc_off && B.source_device == device &&
+         std::memcmp(base + kHeaderBytes, P.meta.data() + kHeaderBytes, P.crc_off - kHeaderBytes) == 0;
+}
+
+checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream, uint64_t epoch,
+                                       const checl_image* base, checl_image* img) {
+  // r1-style validation of the base's metadata (header, manifest, CRC table, bitmap)
+  Parsed B;
+  checl_status st = parse_image(base->host, base->location == CHECL_IMAGE_DEVICE ? base->payload_off : base->image_bytes,
+                                true, &B);
+  if (st) return st;
+  const double t0 = now_ms();
+  DeviceGuard g(device);
+  DevState& ds = ctx->dev(device);
+  {
+    // the plan (and so the layout test) needs the registry as of this call
+    Plan& P0 = get_plan(ctx, ds, device);
+    if (!same_layout(base->host, B, P0, device)) return do_checkpoint(ctx, device, stream, epoch, img, false);
+  }
+  ds.events.reset();
+  KernelTimer kt;
+  checl_timing tm{};
+
+  // a1: quiesce (L16 step 1)
+  const double ts = now_ms();
+  ck(cudaDeviceSynchronize());
+  tm.sync_ms = now_ms() - ts;
+  const double tp = now_ms();
+  Plan& P = get_plan(ctx, ds, device);
+  const uint64_t n = P.n_chunks;
+  const uint64_t map_bytes = (n + 7) / 8;
+  const uint64_t W = ctx->slot_bytes - (kChunkBytes + kBufferAlign);  // stage window (a span fits the slack)
+  const uint64_t max_stages = (P.payload_bytes + W - 1) / W + 1;
+  ds.crc_scratch.ensure(std::max<uint64_t>(n, 1));
+  ds.base_crc.ensure(std::max<uint64_t>(n, 1));
+  ds.map_words.ensure(std::max<uint64_t>((n + 31) / 32, 1));
+  ds.cdesc.ensure(std::max<uint64_t>(n, 1));
+  ds.dtotals.ensure(2);
+  ds.stage_first.ensure(max_stages + 1);
+  ds.stage_lo.ensure(max_stages + 1);
+  ds.h_dtab.ensure(2 + 2 * (max_stages + 1));
+  tm.plan_ms = now_ms() - tp;
+
+  // CRC of every chunk as it is now (kOpCrc: read-only pass), then the present set,
+  // the compacted chunk list and the stage table (delta_scan / delta_stages)
+  LaunchParams lp = base_params(ds);
+  lp.desc = P.d_desc.p;
+  lp.crc = ds.crc_scratch.p;
+  lp.c0 = 0;
+  lp.c1 = n;
+  if (n) ck(cudaMemcpyAsync(ds.base_crc.p, base->host + B.L.crc_off, 4 * n, cudaMemcpyHostToDevice, ds.compute));
+  if (n) timed_launch(ds, kt, kOpCrc, lp, ds.compute);
+  cudaEvent_t sa = ds.events.get(), sb = ds.events.get();
+  ck(cudaEventRecord(sa, ds.compute));
+  ck(launch_delta_scan(P.d_desc.p, ds.crc_scratch.p, ds.base_crc.p, n, ds.map_words.p, ds.cdesc.p, ds.dtotals.p,
+                       ds.compute));
+  ck(launch_delta_stages(ds.cdesc.p, ds.dtotals.p, W, max_stages, ds.stage_first.p, ds.stage_lo.p, ds.compute));
+  ck(cudaEventRecord(sb, ds.compute));
+  kt.spans.push_back({sa, sb});
+  unsigned long long* h = ds.h_dtab.p;
+  ck(cudaMemcpyAsync(h, ds.dtotals.p, 16, cudaMemcpyDeviceToHost, ds.compute));
+  ck(cudaMemcpyAsync(h + 2, ds.stage_first.p, 8 * (max_stages + 1), cudaMemcpyDeviceToHost, ds.compute));
+  ck(cudaMemcpyAsync(h + 3 + max_stages, ds.stage_lo.p, 8 * (max_stages + 1), cudaMemcpyDeviceToHost, ds.compute));
+  ck(cudaStreamSynchronize(ds.compute));
+  const uint64_t n_present = h[0], dbytes = h[1];
+  const unsigned long long* first = h + 2;
+  const unsigned long long* lo = h + 3 + max_stages;
+
+  // delta layout (FORMAT.md): bitmap after the CRC table, compacted payload
+  const uint64_t payload_off = align_up(P.crc_off + 4 * n + map_bytes, kPayloadAlign);
+  const uint64_t image_bytes = payload_off + dbytes;
+  if (img->location != CHECL_IMAGE_HOST) {
+    img->free_device();
+    img->free_host();
+    img->location = CHECL_IMAGE_HOST;
+    img->device = -1;
+  }
+  img->ensure_host(image_bytes, true);
+
+  // a3 + a4 over the present chunks only: gather (kOpCopy, the CRCs are known)
+  // into slot s % n_slots while the copy engine drains the previous slot
+  ds.ensure_slots(ctx->slot_bytes, ctx->n_slots);
+  std::vector<cudaEvent_t> packed(ds.n_slots), drained(ds.n_slots);
+  for (uint32_t i = 0; i < ds.n_slots; ++i) {
+    packed[i] = ds.events.get();
+    drained[i] = ds.events.get();
+  }
+  cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
+  ck(cudaEventRecord(c_begin, ds.copy));
+  lp.desc = ds.cdesc.p;
+  size_t used = 0;
+  for (uint64_t s = 0; s < max_stages; ++s) {
+    if (first[s] == first[s + 1]) continue;
+    const uint32_t k = (uint32_t)(used % ds.n_slots);
+    if (used >= ds.n_slots) ck(cudaStreamWaitEvent(ds.compute, drained[k], 0));
+    lp.c0 = first[s];
+    lp.c1 = first[s + 1];
+    lp.image = ds.slot(k);
+    lp.image_base = lo[s];
+    timed_launch(ds, kt, kOpCopy, lp, ds.compute);
+    ck(cudaEventRecord(packed[k], ds.compute));
+    ck(cudaStreamWaitEvent(ds.copy, packed[k], 0));
+    ck(cudaMemcpyAsync(img->host_mut + payload_off + lo[s], ds.slot(k), lo[s + 1] - lo[s], cudaMemcpyDeviceToHost,
+                       ds.copy));
+    ck(cudaEventRecord(drained[k], ds.copy));
+    ++used;
+  }
+  if (n) {
+    ck(cudaMemcpyAsync(img->host_mut + P.crc_off, ds.crc_scratch.p, 4 * n, cudaMemcpyDeviceToHost, ds.copy));
+    ck(cudaMemcpyAsync(img->host_mut + P.crc_off + 4 * n, ds.map_words.p, map_bytes, cudaMemcpyDeviceToHost, ds.copy));
+  }
+  ck(cudaEventRecord(c_end, ds.copy));
+  tm.n_stages = used;
+  ck(cudaStreamSynchronize(ds.copy));
+
+  // a5: header (the full image's, then the incremental fields), manifest, meta CRC
+  const double tf = now_ms();
+  uint8_t* o = img->host_mut;
+  std::memcpy(o, P.meta.data(), P.crc_off);
+  put_u64(o + 56, payload_off);
+  put_u64(o + 64, dbytes);
+  put_u64(o + 72, image_bytes);
+  put_u32(o + 84, 1);
+  put_u64(o + 88, epoch);
+  put_u64(o + 96, B.epoch);
+  put_u32(o + 104, host_crc32c(base->host + B.L.crc_off, 4 * n));
+  put_u32(o + 108, 0);
+  put_u64(o + 112, n_present);
+  put_u32(o + 120, 0);
+  std::memset(o + P.crc_off + 4 * n + map_bytes, 0, payload_off - P.crc_off - 4 * n - map_bytes);
+  put_u32(o + 124, meta_crc(o, payload_off));
+  tm.commit_ms = now_ms() - tf;
+  img->image_bytes = image_bytes;
+  img->payload_off = payload_off;
+  float cms = 0;
+  if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
+  tm.kernel_ms = kt.sum_ms();
+  tm.n_kernels = kt.spans.size();
+  tm.total_ms = now_ms() - t0;
+  ctx->last = tm;
+  return CHECL_SUCCESS;
+}
+
+// Link of a delta D to the previous image E of a chain (FORMAT.md "Base link").
+bool linked(const checl_image* e, const Parsed& E, const checl_image* d, const Parsed& D) {
+  return D.flags == 1 && D.base_epoch == E.epoch && D.L.n_chunks == E.L.n_chunks && D.L.crc_off == E.L.crc_off &&
+         D.source_device == E.source_device &&
+         D.base_table_crc == host_crc32c(e->host + E.L.crc_off, 4 * E.L.n_chunks) &&
+         std::memcmp(d->host + kHeaderBytes, e->host + kHeaderBytes, D.L.crc_off - kHeaderBytes) == 0;
+}
+
+// Restore of a chain [F, D1, ..., Dn] of host images: F's payload is copied into
+// the new allocation (laid out like the full payload), each delta's present spans
+// are scattered over it in chain order (kOpScatter from the staging slots), and
+// one in-place verify (kOpCheck) checks every chunk against the last CRC table.
+// All-or-nothing like checl_restore.
+checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, uint32_t n_img, int device,
+                              void* stream, checl_report* rep) {
+  const double t0 = now_ms();
+  if (rep) std::memset(rep, 0, sizeof(*rep)), rep->first_bad_chunk = ~0ull;
+  const double tp = now_ms();
+  std::vector<Parsed> Ps(n_img);
+  for (uint32_t i = 0; i < n_img; ++i) {
+    if (chain[i]->location != CHECL_IMAGE_HOST) return CHECL_ERR_INVALID_VALUE;
+    checl_status st = parse_image(chain[i]->host, chain[i]->image_bytes, false, &Ps[i]);
+    if (st) return st;
+    if ((i == 0) != (Ps[i].flags == 0)) return CHECL_ERR_BAD_IMAGE;
+    if (i > 0 && !linked(chain[i - 1], Ps[i - 1], chain[i], Ps[i])) return CHECL_ERR_BAD_IMAGE;
+  }
+  const Parsed& F = Ps[0];
+  const Parsed& Z = Ps[n_img - 1];
+  DeviceGuard g(device);
+  DevState& ds = ctx->dev(device);
+  ds.events.reset();
+  KernelTimer kt;
+  checl_timing tm{};
+  const double ts = now_ms();
+  ck(cudaDeviceSynchronize());
+  tm.sync_ms = now_ms() - ts;
+  if (rep) set_report(rep, Z, 0, 0);
+
+  // r2: one allocation laid out like the full payload
+  auto arena = std::make_shared<Arena>();
+  arena->alloc = ctx->alloc;
+  arena->device = device;
+  arena->stream = stream;
+  arena->bytes = F.full_payload;
+  const double ta = now_ms();
+  if (F.full_payload) {
+    if (ctx->alloc.alloc)
+      arena->base = ctx->alloc.alloc(F.full_payload, device, stream, ctx->alloc.user);
+    else if (cudaMalloc(&arena->base, F.full_payload) != cudaSuccess) {
+      cudaGetLastError();
+      arena->base = nullptr;
+    }
+    if (!arena->base) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
+  }
+  tm.alloc_ms = now_ms() - ta;
+  uint8_t* abase = static_cast<uint8_t*>(arena->base);
+  const uint64_t nch = F.L.n_chunks;
+
+  // descriptors of every delta's present chunks: ptr = destination in the arena,
+  // img_off = position in that delta's compacted payload; stages per delta
+  struct DStage {
+    uint32_t img;
+    uint64_t c0, c1, lo, hi;
+  };
+  std::vector<ChunkDesc> hdesc;
+  std::vector<DStage> dst;
+  for (uint32_t i = 1; i < n_img; ++i) {
+    const Parsed& D = Ps[i];
+    const uint8_t* map = chain[i]->host + D.map_off;
+    uint64_t pos = 0;
+    bool open = false;
+    DStage cur{i, 0, 0, 0, 0};
+    for (size_t b = 0; b < D.bufs.size(); ++b) {
+      const uint64_t nb = chunks_of(D.bufs[b].size);
+      for (uint64_t j = 0; j < nb; ++j) {
+        if (!bit_set(map, D.bufs[b].first_chunk + j)) continue;
+        uint64_t a, z;
+        chunk_span(D.bufs, b, j, D.full_payload, &a, &z);
+        const uint32_t len = (uint32_t)std::min<uint64_t>(kChunkBytes, D.bufs[b].size - (uint64_t)kChunkBytes * j);
+        if (open && pos + (z - a) - cur.lo > ctx->slot_bytes) {
+          dst.push_back(cur);
+          open = false;
+        }
+        if (!open) {
+          cur = DStage{i, hdesc.size(), hdesc.size(), pos, pos};
+          open = true;
+        }
+        hdesc.push_back(ChunkDesc{reinterpret_cast<uint64_t>(abase + a), (uint32_t)(pos / kBufferAlign),
+                                  make_len_pad(len, (uint32_t)(z - a - len))});
+        pos += z - a;
+        cur.c1 = hdesc.size();
+        cur.hi = pos;
+      }
+    }
+    if (open) dst.push_back(cur);
+  }
+  ds.desc_scratch.ensure(std::max<uint64_t>(std::max<uint64_t>(nch, hdesc.size()), 1));
+  ds.cdesc.ensure(std::max<size_t>(hdesc.size(), 1));
+  ds.crc_scratch.ensure(std::max<uint64_t>(nch, 1));
+  ds.h_recs.ensure(std::max<size_t>(F.bufs.size(), 1));
+  ds.recs_scratch.ensure(std::max<size_t>(F.bufs.size(), 1));
+  build_records(F.bufs, [&](size_t b) { return abase + F.bufs[b].off; }, ds.h_recs.p);
+  tm.plan_ms = now_ms() - tp;
+
+  cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get(), base_in = ds.events.get();
+  ck(cudaEventRecord(c_begin, ds.copy));
+  // r3: F's payload straight into the arena; the last CRC table; the delta chunk list
+  if (F.full_payload)
+    ck(cudaMemcpyAsync(abase, chain[0]->host + F.L.payload_off, F.full_payload, cudaMemcpyHostToDevice, ds.copy));
+  ck(cudaEventRecord(base_in, ds.copy));
+  if (nch)
+    ck(cudaMemcpyAsync(ds.crc_scratch.p, chain[n_img - 1]->host + Z.L.crc_off, 4 * nch, cudaMemcpyHostToDevice, ds.copy));
+  if (!hdesc.empty())
+    ck(cudaMemcpyAsync(ds.cdesc.p, hdesc.data(), hdesc.size() * sizeof(ChunkDesc), cudaMemcpyHostToDevice, ds.copy));
+  ds.h_status.p[0] = ~0ull;
+  ds.h_status.p[1] = 0;
+  ck(cudaMemcpyAsync(ds.status.p, ds.h_status.p, 16, cudaMemcpyHostToDevice, ds.copy));
+  if (nch) {
+    ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, F.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
+                       ds.compute));
+    ck(launch_expand(ds.recs_scratch.p, (uint32_t)F.bufs.size(), F.full_payload, nch, ds.desc_scratch.p, ds.n_sms,
+                     ds.compute));
+  }
+  ck(cudaStreamWaitEvent(ds.compute, base_in, 0));
+  // deltas in chain order: fill slot k over PCIe, scatter its spans (later deltas
+  // overwrite earlier ones: every scatter runs on the compute stream in order)
+  ds.ensure_slots(ctx->slot_bytes, ctx->n_slots);
+  std::vector<cudaEvent_t> filled(ds.n_slots), done(ds.n_slots);
+  for (uint32_t i = 0; i < ds.n_slots; ++i) {
+    filled[i] = ds.events.get();
+    done[i] = ds.events.get();
+  }
+  LaunchParams lp = base_params(ds);
+  lp.desc = ds.cdesc.p;
+  for (size_t s = 0; s < dst.size(); ++s) {
+    const DStage& S = dst[s];
+    const uint32_t k = (uint32_t)(s % ds.n_slots);
+    if (s >= ds.n_slots) ck(cudaStreamWaitEvent(ds.copy, done[k], 0));
+    ck(cudaMemcpyAsync(ds.slot(k), chain[S.img]->host + Ps[S.img].L.payload_off + S.lo, S.hi - S.lo,
+                       cudaMemcpyHostToDevice, ds.copy));
+    ck(cudaEventRecord(filled[k], ds.copy));
+    ck(cudaStreamWaitEvent(ds.compute, filled[k], 0));
+    lp.c0 = S.c0;
+    lp.c1 = S.c1;
+    lp.image = ds.slot(k);
+    lp.image_base = S.lo;
+    timed_launch(ds, kt, kOpScatter, lp, ds.compute);
+    ck(cudaEventRecord(done[k], ds.compute));
+  }
+  ck(cudaEventRecord(c_end, ds.copy));
+  ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
+  // r4: every chunk of the result against the last CRC table, in place
+  lp.desc = ds.desc_scratch.p;
+  lp.crc = ds.crc_scratch.p;
+  lp.c0 = 0;
+  lp.c1 = nch;
+  lp.image = nullptr;
+  lp.image_base = 0;
+  if (nch) timed_launch(ds, kt, kOpCheck, lp, ds.compute);
+  ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
+  ck(cudaStreamSynchronize(ds.compute));
+  ck(cudaStreamSynchronize(ds.copy));
+  const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
+  float cms = 0;
+  if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
+  tm.kernel_ms = kt.sum_ms();
+  tm.n_kernels = kt.spans.size();
+  tm.n_stages = dst.size() + 1;
+  if (rep) set_report(rep, Z, n_bad, first_bad);
+  if (n_bad) {
+    ctx->last = tm;
+    return CHECL_ERR_CRC_MISMATCH;
+  }
+  const double tc = now_ms();
+  commit(ctx, Z, device, arena);
   tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
   ctx->last = tm;
@@ -1330,6 +1726,82 @@ checl_status checl_migrate(checl_ctx* ctx, int src_device, int dst_device, void*
     t.n_stages += ck_t.n_stages;
     t.total_ms = now_ms() - t0;
     return st;
+  });
+}
+
+checl_status checl_checkpoint_incremental(checl_ctx* ctx, int device, void* cuda_stream, uint64_t epoch,
+                                          const checl_image* base, checl_image** out) {
+  if (!ctx || !out || !base || !base->host) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  checl_image* img = new (std::nothrow) checl_image();
+  if (!img) return CHECL_ERR_OUT_OF_HOST_MEMORY;
+  BusyGuard b(ctx);
+  checl_status st = b.ok ? guarded([&]() { return do_checkpoint_incremental(ctx, device, cuda_stream, epoch, base, img); })
+                         : CHECL_ERR_BUSY;
+  if (st) {
+    checl_image_free(img);
+    return st;
+  }
+  *out = img;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_restore_chain(checl_ctx* ctx, const checl_image* const* chain, uint32_t n, int device,
+                                 void* cuda_stream, checl_report* rep) {
+  if (!ctx || !chain || n == 0) return CHECL_ERR_INVALID_VALUE;
+  for (uint32_t i = 0; i < n; ++i)
+    if (!chain[i]) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  if (n == 1) return checl_restore(ctx, chain[0], device, cuda_stream, rep);
+  BusyGuard b(ctx);
+  if (!b.ok) return CHECL_ERR_BUSY;
+  return guarded([&]() { return do_restore_chain(ctx, chain, n, device, cuda_stream, rep); });
+}
+
+checl_status checl_image_merge(const checl_image* full, const checl_image* delta, checl_image** out) {
+  if (!full || !delta || !out) return CHECL_ERR_INVALID_VALUE;
+  if (full->location != CHECL_IMAGE_HOST || delta->location != CHECL_IMAGE_HOST) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    Parsed Fp, Dp;
+    checl_status st = parse_image(full->host, full->image_bytes, false, &Fp);
+    if (!st) st = parse_image(delta->host, delta->image_bytes, false, &Dp);
+    if (st) return st;
+    if (Fp.flags != 0 || !linked(full, Fp, delta, Dp)) return CHECL_ERR_BAD_IMAGE;
+    checl_image* m = new checl_image();
+    try {
+      m->ensure_host(Fp.L.image_bytes, false);
+    } catch (...) {
+      delete m;
+      throw;
+    }
+    uint8_t* o = m->host_mut;
+    // FORMAT.md "Merge": F's bytes; D's header with flags 0 and the full-image
+    // fields; D's CRC table; every present chunk's span from D, in ascending order
+    std::memcpy(o, full->host, Fp.L.image_bytes);
+    std::memcpy(o, delta->host, kHeaderBytes);
+    put_u32(o + 84, 0);
+    put_u64(o + 56, Fp.L.payload_off);
+    put_u64(o + 64, Fp.L.payload_bytes);
+    put_u64(o + 72, Fp.L.image_bytes);
+    std::memset(o + 96, 0, 28);
+    std::memcpy(o + Fp.L.crc_off, delta->host + Dp.L.crc_off, 4 * Fp.L.n_chunks);
+    const uint8_t* map = delta->host + Dp.map_off;
+    uint64_t pos = Dp.L.payload_off;
+    for (size_t b = 0; b < Fp.bufs.size(); ++b) {
+      const uint64_t nb = chunks_of(Fp.bufs[b].size);
+      for (uint64_t j = 0; j < nb; ++j) {
+        if (!bit_set(map, Fp.bufs[b].first_chunk + j)) continue;
+        uint64_t a, z;
+        chunk_span(Fp.bufs, b, j, Fp.full_payload, &a, &z);
+        std::memcpy(o + Fp.L.payload_off + a, delta->host + pos, z - a);
+        pos += z - a;
+      }
+    }
+    put_u32(o + 124, meta_crc(o, Fp.L.payload_off));
+    m->image_bytes = Fp.L.image_bytes;
+    m->payload_off = Fp.L.payload_off;
+    *out = m;
+    return CHECL_SUCCESS;
   });
 }
 

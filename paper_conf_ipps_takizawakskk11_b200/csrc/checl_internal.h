@@ -109,7 +109,9 @@ constexpr int kFoldLevels = 5;
 //   kOpCrc    f1  CRC only (no copy): the table of the current contents
 //   kOpCheck  f1  CRC only, compared with the table (in-place verify of a restore)
 //   kOpCopy   f1  buffer -> image without CRC (gather of an incremental image)
-enum : int { kOpPack = 0, kOpVerify = 1, kOpCrc = 2, kOpCheck = 3, kOpCopy = 4 };
+//   kOpScatter f1 image -> buffer without CRC, owned padding included (a delta's
+//                 chunks over a restored base; the result is checked by kOpCheck)
+enum : int { kOpPack = 0, kOpVerify = 1, kOpCrc = 2, kOpCheck = 3, kOpCopy = 4, kOpScatter = 5 };
 
 // Lane-private lookup tables, computed once per device into global memory and
 // bulk-copied (cp.async.bulk) into shared memory by every CTA. Word offsets:

@@ -125,12 +125,13 @@ __device__ __forceinline__ uint32_t horner_mul(uint32_t s, const uint8_t* hb, ui
 // What each op does (kOp* in checl_internal.h).
 template <int kOp>
 struct OpT {
-  static constexpr bool kSrcImg = kOp == kOpVerify;   // read the image, write the buffer
-  static constexpr bool kStore = kOp == kOpPack || kOp == kOpVerify || kOp == kOpCopy;
-  static constexpr bool kCrc = kOp != kOpCopy;
+  static constexpr bool kSrcImg = kOp == kOpVerify || kOp == kOpScatter;  // read the image, write the buffer
+  static constexpr bool kStore = kOp == kOpPack || kOp == kOpVerify || kOp == kOpCopy || kOp == kOpScatter;
+  static constexpr bool kCrc = kOp != kOpCopy && kOp != kOpScatter;
   static constexpr bool kCompare = kOp == kOpVerify || kOp == kOpCheck;  // vs table + owned padding zero
   static constexpr bool kZeroPad = kOp == kOpPack || kOp == kOpCopy;     // destination is the image
-  static constexpr bool kExactTail = kOp == kOpVerify;                   // destination is a buffer
+  static constexpr bool kCopyPad = kOp == kOpScatter;                    // padding copied as is
+  static constexpr bool kExactTail = kOp == kOpVerify || kOp == kOpScatter;  // destination is a buffer
 };
 
 __device__ __forceinline__ uint32_t smem_addr(const void* p) {
@@ -238,6 +239,8 @@ __device__ __forceinline__ void finish_chunk(const LaunchParams& p, uint64_t c, 
         *reinterpret_cast<uint4*>(dst + o) = make_uint4(0u, 0u, 0u, 0u);
     } else if (O::kCompare) {
       for (uint32_t o = len + lane; o < len + pad; o += 32u) pad_bad |= src[o];
+    } else if (O::kCopyPad) {
+      for (uint32_t o = len + lane; o < len + pad; o += 32u) dst[o] = src[o];
     }
   }
   if (O::kCompare) pad_bad = __any_sync(0xFFFFFFFFu, pad_bad != 0);
@@ -587,6 +590,92 @@ __global__ void expand_plan_kernel(const BufferRecord* __restrict__ recs, uint32
   }
 }
 
+// ---- incremental checkpoint: present set, compaction, stages (f1) -----------
+// FORMAT.md "Incremental images": chunk k is present iff crc_now[k] != crc_base[k];
+// the compacted payload is the concatenation of the present chunks' spans (chunk
+// bytes + owned padding) in ascending k. One CTA walks the chunk list in tiles of
+// 1024 (C4: 1 M chunks = 1024 tiles, tens of us next to a 17 ms CRC pass): a
+// ballot writes 32 bitmap bits per warp, a block scan of (span, present) gives
+// each present chunk its compacted offset and index, and the chunk's descriptor is
+// re-emitted with the compacted offset (same ptr / len / pad).
+__global__ void __launch_bounds__(1024, 1) delta_scan_kernel(const ChunkDesc* __restrict__ desc,
+                                                             const uint32_t* __restrict__ crc_now,
+                                                             const uint32_t* __restrict__ crc_base, uint64_t n,
+                                                             uint32_t* __restrict__ map_words,
+                                                             ChunkDesc* __restrict__ cdesc,
+                                                             unsigned long long* __restrict__ totals) {
+  __shared__ unsigned long long w_bytes[32];
+  __shared__ uint32_t w_cnt[32];
+  __shared__ unsigned long long carry_bytes, carry_cnt;
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  if (threadIdx.x == 0) carry_bytes = carry_cnt = 0;
+  __syncthreads();
+  for (uint64_t base = 0; base < n; base += 1024) {
+    const uint64_t i = base + threadIdx.x;
+    const bool present = i < n && crc_now[i] != crc_base[i];
+    ChunkDesc d{};
+    if (present) d = desc[i];
+    const unsigned long long span = present ? (unsigned long long)(desc_len(d) + desc_pad(d)) : 0ull;
+    const uint32_t bits = __ballot_sync(0xFFFFFFFFu, present);
+    if (lane == 0 && base + warp * 32 < n) map_words[(base >> 5) + warp] = bits;
+    unsigned long long sb = span;
+    uint32_t sc = present ? 1u : 0u;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned long long tb = __shfl_up_sync(0xFFFFFFFFu, sb, o);
+      const uint32_t tc = __shfl_up_sync(0xFFFFFFFFu, sc, o);
+      if (lane >= o) sb += tb, sc += tc;
+    }
+    if (lane == 31) w_bytes[warp] = sb, w_cnt[warp] = sc;
+    __syncthreads();
+    if (warp == 0) {
+      unsigned long long xb = w_bytes[lane];
+      uint32_t xc = w_cnt[lane];
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long tb = __shfl_up_sync(0xFFFFFFFFu, xb, o);
+        const uint32_t tc = __shfl_up_sync(0xFFFFFFFFu, xc, o);
+        if (lane >= o) xb += tb, xc += tc;
+      }
+      w_bytes[lane] = xb - w_bytes[lane];  // exclusive warp offsets
+      w_cnt[lane] = xc - w_cnt[lane];
+    }
+    __syncthreads();
+    const unsigned long long off = carry_bytes + w_bytes[warp] + sb - span;
+    const unsigned long long idx = carry_cnt + w_cnt[warp] + sc - (present ? 1u : 0u);
+    if (present) {
+      ChunkDesc o;
+      o.ptr = d.ptr;
+      o.img_off_256 = (uint32_t)(off / kBufferAlign);
+      o.len_pad = d.len_pad;
+      cdesc[idx] = o;
+    }
+    __syncthreads();
+    if (threadIdx.x == 1023) carry_bytes = off + span, carry_cnt = idx + (present ? 1u : 0u);
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) totals[0] = carry_cnt, totals[1] = carry_bytes;
+}
+
+// Stage s of the compacted payload = the present chunks whose compacted start lies
+// in [s*W, (s+1)*W); with W = slot - (64 KiB + 256) every stage fits one staging
+// slot. first[s] = index of its first chunk (binary search over the ascending
+// compacted offsets), lo[s] = that chunk's compacted start (total bytes if none).
+__global__ void delta_stages_kernel(const ChunkDesc* __restrict__ cdesc, const unsigned long long* __restrict__ totals,
+                                    uint64_t W, uint64_t n_stages, unsigned long long* __restrict__ first,
+                                    unsigned long long* __restrict__ lo) {
+  const uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x;
+  if (s > n_stages) return;
+  const uint64_t np = totals[0], bytes = totals[1], want = s * W;
+  uint64_t a = 0, b = np;  // first i with start(i) >= want
+  while (a < b) {
+    const uint64_t m = (a + b) >> 1;
+    if ((uint64_t)cdesc[m].img_off_256 * kBufferAlign >= want) b = m; else a = m + 1;
+  }
+  first[s] = a;
+  lo[s] = a < np ? (unsigned long long)cdesc[a].img_off_256 * kBufferAlign : bytes;
+}
+
 // ---- launchers (called from checl_engine.cpp) --------------------------------
 
 cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload_bytes, uint64_t n_chunks,
@@ -614,6 +703,7 @@ cudaError_t snapshot_configure() {
   if (e == cudaSuccess) e = configure_op<kOpCrc>();
   if (e == cudaSuccess) e = configure_op<kOpCheck>();
   if (e == cudaSuccess) e = configure_op<kOpCopy>();
+  if (e == cudaSuccess) e = configure_op<kOpScatter>();
   return e;
 }
 
@@ -644,8 +734,22 @@ cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream
     case kOpCrc: launch_op<kOpCrc>(p, (unsigned)ctas, s, kernel); break;
     case kOpCheck: launch_op<kOpCheck>(p, (unsigned)ctas, s, kernel); break;
     case kOpCopy: launch_op<kOpCopy>(p, (unsigned)ctas, s, kernel); break;
+    case kOpScatter: launch_op<kOpScatter>(p, (unsigned)ctas, s, kernel); break;
     default: return cudaErrorInvalidValue;
   }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, const uint32_t* crc_base, uint64_t n,
+                              uint32_t* map_words, ChunkDesc* cdesc, unsigned long long* totals, cudaStream_t s) {
+  delta_scan_kernel<<<1, 1024, 0, s>>>(desc, crc_now, crc_base, n, map_words, cdesc, totals);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_delta_stages(const ChunkDesc* cdesc, const unsigned long long* totals, uint64_t W, uint64_t n_stages,
+                                unsigned long long* first, unsigned long long* lo, cudaStream_t s) {
+  const uint64_t n = n_stages + 1;
+  delta_stages_kernel<<<(unsigned)((n + 255) / 256), 256, 0, s>>>(cdesc, totals, W, n_stages, first, lo);
   return cudaGetLastError();
 }
 
