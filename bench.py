@@ -42,6 +42,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--c4-scale", type=float, default=1.0)
     ap.add_argument("--c5-large", action="store_true", help="C5 with 16 x 1 GiB instead of the C2 set")
+    ap.add_argument("--mode", default="snapshot", choices=["snapshot", "incremental"],
+                    help="incremental: checl_checkpoint_incremental with --dirty of the chunks rewritten per step")
+    ap.add_argument("--dirty", type=float, default=0.1)
     return ap.parse_args()
 
 
@@ -267,8 +270,111 @@ def run_migration(a):
         dist.destroy_process_group()
 
 
+def run_incremental(a):
+    """incremental checkpoint (PAPER.md L45 future work). Between
+    steps the "application" rewrites one byte in a fraction `--dirty` of the
+    workload's chunks (untimed); each timed step is checl_checkpoint_incremental on
+    the previous image (pinned host image, PCIe drain of the changed chunks only).
+    Reported next to a full checkpoint of the same workload and a chain restore."""
+    import numpy as np
+    import torch
+    from paper_conf_ipps_takizawakskk11_b200 import checl
+
+    dev = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(dev)
+    w = workload(a.config, 0, a.c4_scale)
+    tensors = [torch.empty(b.size, dtype=torch.uint8, device=dev) for b in w.buffers]
+    for t, b in zip(tensors, w.buffers):
+        checl.debug_fill(t, w.seed, b.stream)
+    torch.cuda.synchronize()
+    ctx = checl.Context()
+    for t, b in zip(tensors, w.buffers):
+        ctx.register(t, b.flags)
+    S = w.total_bytes
+    # chunk start positions (buffer, offset) for the mutation
+    starts = [(i, j * 65536) for i, b in enumerate(w.buffers) for j in range((b.size + 65535) // 65536)]
+    rng = np.random.default_rng(5)
+    k = max(1, int(len(starts) * a.dirty))
+
+    def mutate():
+        pick = rng.choice(len(starts), size=k, replace=False)
+        by_buf = {}
+        for c in pick:
+            i, o = starts[c]
+            by_buf.setdefault(i, []).append(o + int(rng.integers(0, min(65536, w.buffers[i].size - o))))
+        for i, offs in by_buf.items():
+            idx = torch.tensor(offs, dtype=torch.int64, device=dev)
+            tensors[i][idx] ^= 0x5A
+        torch.cuda.synchronize()
+
+    cur = torch.cuda.current_stream(dev)
+
+    def timed(fn):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(cur)
+        r = fn()
+        e1.record(cur)
+        e1.synchronize()
+        return e0.elapsed_time(e1), r
+
+    full = ctx.checkpoint(dev, epoch=0)
+    full_ms = []
+    for i in range(a.warmup + a.steps):
+        ms, _ = timed(lambda: ctx.checkpoint(dev, epoch=0, into=full))
+        if i >= a.warmup:
+            full_ms.append(ms)
+    base = full
+    for i in range(a.warmup):
+        mutate()
+        base = ctx.checkpoint_incremental(dev, base, epoch=i + 1)
+    ms_steps, drained, present, tms = [], [], [], []
+    with ClockSampler(dev) as clk:
+        for i in range(a.steps):
+            mutate()
+            ms, d = timed(lambda: ctx.checkpoint_incremental(dev, base, epoch=a.warmup + i + 1))
+            h = d.header()
+            ms_steps.append(ms)
+            drained.append(h["payload_bytes"])
+            present.append(h["n_present"])
+            tms.append(ctx.last_timing())
+            if i:
+                base.free()
+            base = d
+    # chain restore of [full, last delta] is not linked (intermediate deltas freed):
+    # restore [merge(full@now), ...] instead: take a fresh full and one delta
+    f2 = ctx.checkpoint(dev, epoch=100)
+    mutate()
+    d2 = ctx.checkpoint_incremental(dev, f2, epoch=101)
+    rs_ms, rep = timed(lambda: ctx.restore_chain([f2, d2], dev))
+    n_diff = 0
+    for h, t in zip(range(1, len(tensors) + 1), tensors):
+        ptr, nb, _ = ctx.translate(h)
+        n_diff += checl.debug_compare(dev, ptr, t.data_ptr(), nb) if nb else 0
+    t_inc = sum(ms_steps) / len(ms_steps)
+    t_full = sum(full_ms) / len(full_ms)
+    crc_ms = statistics.mean(t["kernel_ms"] for t in tms)
+    pk = peaks()
+    hbm = pk.get("hbm_gbs") or 6650.0
+    print(json.dumps({
+        "metric": "incremental checkpoint GB/s (logical payload / time), pinned host image",
+        "value": S / (t_inc * 1e-3) / 1e9, "unit": "GB/s", "n_gpus": 1, "steps": a.steps, "warmup": a.warmup,
+        "ms_per_step": t_inc, "higher_is_better": True, "dtype": "u8", "data": "synthetic",
+        "config": {"workload": w.name, "payload_bytes_per_gpu": S, "n_chunks": len(starts),
+                   "dirty_fraction": a.dirty, "chunks_rewritten_per_step": k},
+        "full_checkpoint_ms": t_full, "speedup_vs_full": t_full / t_inc,
+        "drained_bytes_per_step": statistics.mean(drained), "present_chunks_per_step": statistics.mean(present),
+        "kernel_ms_per_step": crc_ms,
+        "crc_pass": {"bytes_read": S, "note": "kOpCrc reads S; gather reads + writes only the present spans"},
+        "last_timing": tms[-1], "chain_restore_ms": rs_ms, "chain_restore_GBs": S / (rs_ms * 1e-3) / 1e9,
+        "verified": n_diff == 0 and rep.n_bad_chunks == 0, "clocks": clk.summary(), "hbm_peak": hbm}))
+    ctx.close()
+
+
 def main():
     a = parse()
+    if a.mode == "incremental":
+        run_incremental(a)
+        return
     if a.impl == "reference":
         run_reference(a)
         return

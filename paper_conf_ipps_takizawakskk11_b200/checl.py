@@ -35,6 +35,7 @@ ERR_PEER_ACCESS = -9
 ERR_BUSY = -10
 
 IMAGE_HOST, IMAGE_DEVICE = 0, 1
+IO_DIRECT, IO_SYNC = 1, 2
 FILL_RANDOM, FILL_FLOAT, FILL_ZEROS = 0, 1, 2
 
 EXPORTS = (
@@ -44,6 +45,8 @@ EXPORTS = (
     "checl_restore", "checl_migrate", "checl_last_timing", "checl_status_string", "checl_last_cuda_error",
     "checl_version", "checl_debug_fill", "checl_debug_compare", "checl_debug_corrupt",
     "checl_checkpoint_incremental", "checl_restore_chain", "checl_image_merge",
+    "checl_request_checkpoint", "checl_checkpoint_pending", "checl_install_signal", "checl_sync_point",
+    "checl_image_write", "checl_image_read",
 )
 
 
@@ -96,6 +99,12 @@ def _load() -> C.CDLL:
         "checl_checkpoint_incremental": [P, C.c_int, V, U64, P, PP],
         "checl_restore_chain": [P, C.POINTER(C.c_void_p), U32, C.c_int, V, C.POINTER(_Report)],
         "checl_image_merge": [P, P, PP],
+        "checl_request_checkpoint": [P],
+        "checl_checkpoint_pending": [P, C.POINTER(C.c_int)],
+        "checl_install_signal": [P, C.c_int],
+        "checl_sync_point": [P, C.c_int, V, U64, P, PP],
+        "checl_image_write": [P, C.c_char_p, U32],
+        "checl_image_read": [C.c_char_p, U32, PP],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -205,6 +214,18 @@ class Image:
         if h["flags"] == 1:
             h.update(base_epoch=u64(96), base_table_crc=u32(104), n_present=u64(112))
         return h
+
+    def write(self, path: str, direct: bool = True, sync: bool = False):
+        """Writing phase (L16 step 3 analogue): the image bytes to a file."""
+        _check(lib.checl_image_write(self.handle, os.fsencode(path), (IO_DIRECT if direct else 0) | (IO_SYNC if sync else 0)),
+               "checl_image_write")
+
+    @classmethod
+    def read(cls, path: str, direct: bool = True) -> "Image":
+        """An image file read back into a (pinned) host image; metadata validated."""
+        out = C.c_void_p()
+        _check(lib.checl_image_read(os.fsencode(path), IO_DIRECT if direct else 0, C.byref(out)), "checl_image_read")
+        return cls(out.value)
 
     def to_host(self) -> "Image":
         out = C.c_void_p()
@@ -379,6 +400,28 @@ class Context:
         rep = Report._from(r)
         _check(st, "checl_migrate", rep)
         return rep
+
+    # -- delayed checkpointing mode (L16 §III-C)
+    def request_checkpoint(self):
+        _check(lib.checl_request_checkpoint(self._p), "checl_request_checkpoint")
+
+    def checkpoint_pending(self) -> bool:
+        v = C.c_int()
+        _check(lib.checl_checkpoint_pending(self._p, C.byref(v)), "checl_checkpoint_pending")
+        return bool(v.value)
+
+    def install_signal(self, signo: int):
+        """A handler for `signo` (e.g. signal.SIGUSR1) that requests a checkpoint."""
+        _check(lib.checl_install_signal(self._p, signo), "checl_install_signal")
+
+    def sync_point(self, device: int, stream=None, epoch: int = 0, into: Optional[Image] = None) -> Optional[Image]:
+        """clFinish analogue: synchronises `stream`; checkpoints iff one was requested."""
+        out = C.c_void_p()
+        _check(lib.checl_sync_point(self._p, device, _stream_ptr(stream), epoch, into.handle if into else None,
+                                    C.byref(out)), "checl_sync_point")
+        if not out.value:
+            return None
+        return into if into is not None else Image(out.value)
 
     def last_timing(self) -> dict:
         t = _Timing()

@@ -7,6 +7,10 @@
 // plans it (flat chunk list, stages), drives the staging pipeline on two streams
 // (copy engine D2H/H2D overlapped with the pack / verify kernels), and commits.
 #include <cuda_runtime.h>
+#include <fcntl.h>
+#include <signal.h>
+#include <sys/stat.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <atomic>
@@ -52,6 +56,46 @@ constexpr size_t kSlotSlack = 256;  // pack writes whole 16-B granules past a la
 constexpr size_t kDefaultSlotBytes = 64ull << 20;
 
 thread_local std::string t_last_cuda_error;
+
+// signal number -> context of checl_install_signal (delayed checkpointing mode)
+constexpr int kMaxSignal = 65;
+std::atomic<checl_ctx*> g_signal_ctx[kMaxSignal];
+
+// Pinned host buffers of freed library-owned images, kept for the next image
+// (cudaHostAlloc of a large buffer costs ~1 ms per few MB: an incremental
+// checkpoint loop would otherwise pin a new image every step). Bounded by
+// CHECL_PINNED_POOL_BYTES (default 4 GiB); buffers beyond it are freed.
+struct PinnedPool {
+  std::mutex mu;
+  std::multimap<size_t, void*> free_;  // capacity -> buffer
+  size_t bytes = 0, limit = 0;
+  PinnedPool() {
+    const char* e = std::getenv("CHECL_PINNED_POOL_BYTES");
+    limit = e ? (size_t)std::strtoull(e, nullptr, 10) : (4ull << 30);
+  }
+  // a pooled buffer with n <= capacity <= 2n + 64 MiB, or nullptr
+  void* take(size_t n, size_t* cap) {
+    std::lock_guard<std::mutex> lk(mu);
+    auto it = free_.lower_bound(n);
+    if (it == free_.end() || it->first > 2 * n + (64ull << 20)) return nullptr;
+    void* p = it->second;
+    *cap = it->first;
+    bytes -= it->first;
+    free_.erase(it);
+    return p;
+  }
+  bool give(void* p, size_t cap) {
+    std::lock_guard<std::mutex> lk(mu);
+    if (bytes + cap > limit) return false;
+    free_.emplace(cap, p);
+    bytes += cap;
+    return true;
+  }
+};
+PinnedPool& pinned_pool() {
+  static PinnedPool* pool = new PinnedPool();  // never destroyed: may outlive the CUDA runtime
+  return *pool;
+}
 
 double now_ms() {
   return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
@@ -383,10 +427,11 @@ struct checl_image {
   }
   void free_host() {
     if (owned && host_mut) {
-      if (pinned)
-        cudaFreeHost(host_mut);
-      else
+      if (pinned) {
+        if (!pinned_pool().give(host_mut, host_cap)) cudaFreeHost(host_mut);
+      } else {
         std::free(host_mut);
+      }
     }
     host = host_mut = nullptr;
     host_cap = 0;
@@ -396,14 +441,16 @@ struct checl_image {
     free_host();
     owned = true;
     void* p = nullptr;
+    size_t cap = std::max<size_t>(n, 1);
     if (want_pinned) {
-      ck(cudaHostAlloc(&p, std::max<size_t>(n, 1), cudaHostAllocDefault));
+      p = pinned_pool().take(cap, &cap);
+      if (!p) ck(cudaHostAlloc(&p, cap, cudaHostAllocDefault));
     } else {
       p = std::malloc(std::max<size_t>(n, 1));
       if (!p) throw std::bad_alloc();
     }
     host = host_mut = static_cast<uint8_t*>(p);
-    host_cap = n;
+    host_cap = cap;
     pinned = want_pinned;
   }
 };
@@ -421,6 +468,9 @@ struct checl_ctx {
   uint64_t version[kMaxDevices] = {};
   uint64_t next_id = 1;
   std::atomic<bool> busy{false};
+  // delayed checkpointing mode (L16 §III-C): set by checl_request_checkpoint (or
+  // the installed signal handler), consumed by checl_sync_point
+  std::atomic<uint32_t> requested{0};
   DevState* devs[kMaxDevices] = {};
   size_t slot_bytes = kDefaultSlotBytes;
   uint32_t n_slots = 2;
@@ -1490,6 +1540,10 @@ checl_status checl_destroy(checl_ctx* ctx) {
         m = nullptr;
       }
     }
+    for (auto& c : g_signal_ctx) {
+      checl_ctx* expect = ctx;
+      c.compare_exchange_strong(expect, nullptr);
+    }
     delete ctx;
     return CHECL_SUCCESS;
   });
@@ -1801,6 +1855,172 @@ checl_status checl_image_merge(const checl_image* full, const checl_image* delta
     m->image_bytes = Fp.L.image_bytes;
     m->payload_off = Fp.L.payload_off;
     *out = m;
+    return CHECL_SUCCESS;
+  });
+}
+
+// ---- delayed checkpointing mode (L16 §III-C) ----------------
+
+namespace {
+void on_checkpoint_signal(int signo) {  // async-signal-safe: one lock-free atomic store
+  if (signo <= 0 || signo >= kMaxSignal) return;
+  checl_ctx* c = g_signal_ctx[signo].load(std::memory_order_relaxed);
+  if (c) c->requested.store(1, std::memory_order_relaxed);
+}
+}  // namespace
+
+checl_status checl_request_checkpoint(checl_ctx* ctx) {
+  if (!ctx) return CHECL_ERR_INVALID_VALUE;
+  ctx->requested.store(1, std::memory_order_relaxed);
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_checkpoint_pending(const checl_ctx* ctx, int* pending) {
+  if (!ctx || !pending) return CHECL_ERR_INVALID_VALUE;
+  *pending = ctx->requested.load(std::memory_order_relaxed) ? 1 : 0;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_install_signal(checl_ctx* ctx, int signo) {
+  if (signo <= 0 || signo >= kMaxSignal || signo == SIGKILL || signo == SIGSTOP) return CHECL_ERR_INVALID_VALUE;
+  struct sigaction sa;
+  std::memset(&sa, 0, sizeof sa);
+  sigemptyset(&sa.sa_mask);
+  sa.sa_flags = SA_RESTART;
+  sa.sa_handler = ctx ? on_checkpoint_signal : SIG_DFL;
+  g_signal_ctx[signo].store(ctx);
+  if (sigaction(signo, &sa, nullptr) != 0) {
+    g_signal_ctx[signo].store(nullptr);
+    return CHECL_ERR_INVALID_VALUE;
+  }
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_sync_point(checl_ctx* ctx, int device, void* cuda_stream, uint64_t epoch, checl_image* reuse,
+                              checl_image** out) {
+  if (!ctx || !out) return CHECL_ERR_INVALID_VALUE;
+  if (reuse && !reuse->owned) return CHECL_ERR_INVALID_VALUE;
+  if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
+  *out = nullptr;
+  checl_status st = guarded([&]() -> checl_status {
+    DeviceGuard g(device);
+    ck(cudaStreamSynchronize(static_cast<cudaStream_t>(cuda_stream)));  // the clFinish the application asked for
+    return CHECL_SUCCESS;
+  });
+  if (st) return st;
+  if (!ctx->requested.exchange(0, std::memory_order_relaxed)) return CHECL_SUCCESS;
+  if (reuse) {
+    st = checl_checkpoint_into(ctx, device, cuda_stream, epoch, reuse);
+    if (!st) *out = reuse;
+  } else {
+    st = checl_checkpoint(ctx, device, cuda_stream, epoch, out);
+  }
+  if (st) ctx->requested.store(1, std::memory_order_relaxed);  // still owed
+  return st;
+}
+
+// ---- writing phase: image <-> file (L16 step 3 analogue; Table I) ----
+
+namespace {
+constexpr size_t kIoPiece = 64ull << 20;
+
+bool write_all(int fd, const uint8_t* p, size_t n, uint64_t off) {
+  while (n) {
+    const ssize_t w = pwrite(fd, p, n, (off_t)off);
+    if (w <= 0) return false;
+    p += w;
+    n -= (size_t)w;
+    off += (uint64_t)w;
+  }
+  return true;
+}
+
+// Writes [p, p+n) at file offset `off`: the 4 KiB-multiple part through the O_DIRECT
+// descriptor when both are usable (page-aligned source), the rest buffered.
+bool write_span(int dfd, int bfd, const uint8_t* p, size_t n, uint64_t off) {
+  size_t direct = 0;
+  if (dfd >= 0 && (reinterpret_cast<uintptr_t>(p) & 4095u) == 0 && (off & 4095u) == 0) direct = n & ~(size_t)4095;
+  if (direct && !write_all(dfd, p, direct, off)) return false;
+  return write_all(bfd, p + direct, n - direct, off + direct);
+}
+}  // namespace
+
+checl_status checl_image_write(const checl_image* img, const char* path, uint32_t flags) {
+  if (!img || !path || flags & ~3u) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    const int bfd = ::open(path, O_WRONLY | O_CREAT | O_TRUNC, 0644);
+    if (bfd < 0) return CHECL_ERR_INVALID_VALUE;
+    int dfd = (flags & CHECL_IO_DIRECT) ? ::open(path, O_WRONLY | O_DIRECT) : -1;
+    bool ok = true;
+    if (img->location == CHECL_IMAGE_HOST) {
+      for (uint64_t o = 0; ok && o < img->image_bytes; o += kIoPiece)
+        ok = write_span(dfd, bfd, img->host + o, std::min<uint64_t>(kIoPiece, img->image_bytes - o), o);
+    } else {
+      // device image: the host mirror, then the payload through a pinned bounce buffer
+      ok = write_span(dfd, bfd, img->host, img->payload_off, 0);
+      DeviceGuard g(img->device);
+      PinnedBuf<uint8_t> bounce;
+      const uint64_t pay = img->image_bytes - img->payload_off;
+      bounce.ensure(std::min<uint64_t>(kIoPiece, std::max<uint64_t>(pay, 1)));
+      for (uint64_t o = 0; ok && o < pay; o += kIoPiece) {
+        const uint64_t n = std::min<uint64_t>(kIoPiece, pay - o);
+        ck(cudaMemcpy(bounce.p, img->d_payload + o, n, cudaMemcpyDeviceToHost));
+        ok = write_span(dfd, bfd, bounce.p, n, img->payload_off + o);
+      }
+      bounce.release();
+    }
+    if (ok && (flags & CHECL_IO_SYNC)) ok = ::fsync(bfd) == 0;
+    if (dfd >= 0) ::close(dfd);
+    if (::close(bfd) != 0) ok = false;
+    return ok ? CHECL_SUCCESS : CHECL_ERR_INVALID_VALUE;
+  });
+}
+
+checl_status checl_image_read(const char* path, uint32_t flags, checl_image** out) {
+  if (!path || !out || flags & ~1u) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    struct stat sb;
+    if (::stat(path, &sb) != 0 || sb.st_size < (off_t)kHeaderBytes) return CHECL_ERR_BAD_IMAGE;
+    const uint64_t size = (uint64_t)sb.st_size, cap = align_up(size, 4096);
+    checl_image* img = new checl_image();
+    void* p = nullptr;
+    // pinned when a device is present (restore then fills over PCIe at full rate)
+    if (device_count() > 0 && cudaHostAlloc(&p, cap, cudaHostAllocDefault) == cudaSuccess) {
+      img->pinned = true;
+    } else {
+      cudaGetLastError();
+      p = nullptr;
+      if (posix_memalign(&p, 4096, cap) != 0) {
+        delete img;
+        throw std::bad_alloc();
+      }
+      img->pinned = false;
+    }
+    img->owned = true;
+    img->host = img->host_mut = static_cast<uint8_t*>(p);
+    img->host_cap = cap;
+    int fd = (flags & CHECL_IO_DIRECT) ? ::open(path, O_RDONLY | O_DIRECT) : -1;
+    if (fd < 0) fd = ::open(path, O_RDONLY);
+    bool ok = fd >= 0;
+    for (uint64_t o = 0; ok && o < size;) {
+      const ssize_t r = pread(fd, img->host_mut + o, (size_t)std::min<uint64_t>(kIoPiece, cap - o), (off_t)o);
+      if (r <= 0) {
+        ok = false;
+        break;
+      }
+      o += (uint64_t)r;
+    }
+    if (fd >= 0) ::close(fd);
+    Parsed P;
+    checl_status st = ok ? parse_image(img->host, size, false, &P) : CHECL_ERR_BAD_IMAGE;
+    if (st) {
+      img->free_host();
+      delete img;
+      return st;
+    }
+    img->image_bytes = P.L.image_bytes;
+    img->payload_off = P.L.payload_off;
+    *out = img;
     return CHECL_SUCCESS;
   });
 }

@@ -104,3 +104,73 @@ def test_missing_library_fails_loudly(tmp_path):
     r = subprocess.run([sys.executable, "-c", "import paper_conf_ipps_takizawakskk11_b200"], cwd=tmp_path,
                        capture_output=True, text=True)
     assert r.returncode != 0 and "ImportError" in r.stderr and "no CPU fallback" in r.stderr
+
+
+PY_HOST_PATHS = r"""
+import os, signal, sys, struct
+sys.path.insert(0, %r)
+import numpy as np
+from paper_conf_ipps_takizawakskk11_b200 import checl
+from oracle import oracle as O
+tmp = sys.argv[1]
+
+# delayed checkpointing mode (L16): the signal only marks the request
+c = checl.Context(allocator="cuda")
+assert not c.checkpoint_pending()
+c.install_signal(signal.SIGUSR1)
+os.kill(os.getpid(), signal.SIGUSR1)
+assert c.checkpoint_pending()
+c2 = checl.Context(allocator="cuda")
+assert not c2.checkpoint_pending()
+c2.request_checkpoint()
+assert c2.checkpoint_pending()
+try:
+    c.install_signal(signal.SIGKILL)
+    raise SystemExit("SIGKILL accepted")
+except checl.CheclError as e:
+    assert e.status == checl.ERR_INVALID_VALUE
+c.close()   # unregisters its handler binding
+os.kill(os.getpid(), signal.SIGUSR1)   # handler sees no context: ignored
+c2.close()
+
+# writing phase: oracle images (full and incremental) through write/read, both I/O modes
+rng = np.random.default_rng(1)
+ents = [O.Entry(1, rng.integers(0, 256, 300001, dtype=np.uint8)), O.Entry(4, rng.integers(0, 256, 13, dtype=np.uint8))]
+full = O.checkpoint(ents, device=0, epoch=7)
+ents[0].data[100000] ^= 1
+delta = O.checkpoint_incremental(ents, full, device=0, epoch=8)
+for name, arr in (("full", full), ("delta", delta)):
+    for direct in (True, False):
+        img = checl.Image.wrap(arr)
+        path = os.path.join(tmp, f"{name}{int(direct)}.checl")
+        img.write(path, direct=direct, sync=True)
+        assert os.path.getsize(path) == arr.size
+        back = checl.Image.read(path, direct=direct)
+        assert np.array_equal(back.view(), arr)
+        assert back.header()["flags"] == (1 if name == "delta" else 0)
+        back.free(); img.free()
+# library merge of the re-read images == oracle merge
+F = checl.Image.read(os.path.join(tmp, "full1.checl"))
+D = checl.Image.read(os.path.join(tmp, "delta1.checl"))
+st, want = O.merge(full, delta)
+assert st == 0 and np.array_equal(F.merge(D).view(), want)
+# damaged files are refused at read
+p = os.path.join(tmp, "full1.checl")
+raw = bytearray(open(p, "rb").read())
+for bad in (raw[:-1], raw[:100], raw[:40] + bytes([raw[40] ^ 1]) + raw[41:]):
+    q = os.path.join(tmp, "bad.checl")
+    open(q, "wb").write(bytes(bad))
+    try:
+        checl.Image.read(q)
+        raise SystemExit("damaged image accepted")
+    except checl.CheclError as e:
+        assert e.status == checl.ERR_BAD_IMAGE, e
+print("ok")
+"""
+
+
+def test_delayed_mode_signal_and_image_files_without_gpu(built, tmp_path):
+    env = dict(os.environ, CHECL_FAKE_DEVICES="1")
+    r = subprocess.run([sys.executable, "-c", PY_HOST_PATHS % ROOT, str(tmp_path)], capture_output=True, text=True,
+                       env=env, cwd=ROOT)
+    assert r.returncode == 0 and "ok" in r.stdout, r.stdout + r.stderr
