@@ -23,6 +23,7 @@
 #include <mutex>
 #include <new>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "../../include/checl.h"
@@ -1945,6 +1946,27 @@ bool write_span(int dfd, int bfd, const uint8_t* p, size_t n, uint64_t off) {
 }
 }  // namespace
 
+// Runs fn(lo, hi) over [0, n) split into up to kIoThreads 4 KiB-aligned pieces on
+// parallel threads (one thread's memcpy into the page cache / tmpfs tops out at a few
+// GB/s); true iff every piece succeeded.
+extern "C++" {
+constexpr int kIoThreads = 8;
+template <typename F>
+static bool parallel_io(uint64_t n, F fn) {
+  const uint64_t per = std::max<uint64_t>(align_up((n + kIoThreads - 1) / kIoThreads, 4096), kIoPiece);
+  std::vector<std::thread> th;
+  std::atomic<bool> ok{true};
+  for (uint64_t lo = 0; lo < n; lo += per) {
+    const uint64_t hi = std::min(n, lo + per);
+    th.emplace_back([&, lo, hi] {
+      if (!fn(lo, hi)) ok.store(false);
+    });
+  }
+  for (auto& t : th) t.join();
+  return ok.load();
+}
+}  // extern "C++"
+
 checl_status checl_image_write(const checl_image* img, const char* path, uint32_t flags) {
   if (!img || !path || flags & ~3u) return CHECL_ERR_INVALID_VALUE;
   return guarded([&]() -> checl_status {
@@ -1953,8 +1975,11 @@ checl_status checl_image_write(const checl_image* img, const char* path, uint32_
     int dfd = (flags & CHECL_IO_DIRECT) ? ::open(path, O_WRONLY | O_DIRECT) : -1;
     bool ok = true;
     if (img->location == CHECL_IMAGE_HOST) {
-      for (uint64_t o = 0; ok && o < img->image_bytes; o += kIoPiece)
-        ok = write_span(dfd, bfd, img->host + o, std::min<uint64_t>(kIoPiece, img->image_bytes - o), o);
+      ok = parallel_io(img->image_bytes, [&](uint64_t lo, uint64_t hi) {
+        for (uint64_t o = lo; o < hi; o += kIoPiece)
+          if (!write_span(dfd, bfd, img->host + o, std::min<uint64_t>(kIoPiece, hi - o), o)) return false;
+        return true;
+      });
     } else {
       // device image: the host mirror, then the payload through a pinned bounce buffer
       ok = write_span(dfd, bfd, img->host, img->payload_off, 0);
@@ -1984,8 +2009,10 @@ checl_status checl_image_read(const char* path, uint32_t flags, checl_image** ou
     const uint64_t size = (uint64_t)sb.st_size, cap = align_up(size, 4096);
     checl_image* img = new checl_image();
     void* p = nullptr;
+    size_t pcap = cap;
     // pinned when a device is present (restore then fills over PCIe at full rate)
-    if (device_count() > 0 && cudaHostAlloc(&p, cap, cudaHostAllocDefault) == cudaSuccess) {
+    if (device_count() > 0 && ((p = pinned_pool().take(cap, &pcap)) != nullptr ||
+                               cudaHostAlloc(&p, cap, cudaHostAllocDefault) == cudaSuccess)) {
       img->pinned = true;
     } else {
       cudaGetLastError();
@@ -1998,18 +2025,19 @@ checl_status checl_image_read(const char* path, uint32_t flags, checl_image** ou
     }
     img->owned = true;
     img->host = img->host_mut = static_cast<uint8_t*>(p);
-    img->host_cap = cap;
+    img->host_cap = img->pinned ? pcap : cap;
     int fd = (flags & CHECL_IO_DIRECT) ? ::open(path, O_RDONLY | O_DIRECT) : -1;
     if (fd < 0) fd = ::open(path, O_RDONLY);
-    bool ok = fd >= 0;
-    for (uint64_t o = 0; ok && o < size;) {
-      const ssize_t r = pread(fd, img->host_mut + o, (size_t)std::min<uint64_t>(kIoPiece, cap - o), (off_t)o);
-      if (r <= 0) {
-        ok = false;
-        break;
+    bool ok = fd >= 0 && parallel_io(size, [&](uint64_t lo, uint64_t hi) {
+      // pieces start 4 KiB-aligned; the last one may read up to `cap` (aligned length)
+      const uint64_t end = hi == size ? cap : hi;
+      for (uint64_t o = lo; o < hi;) {
+        const ssize_t r = pread(fd, img->host_mut + o, (size_t)std::min<uint64_t>(kIoPiece, end - o), (off_t)o);
+        if (r <= 0) return false;
+        o += (uint64_t)r;
       }
-      o += (uint64_t)r;
-    }
+      return true;
+    });
     if (fd >= 0) ::close(fd);
     Parsed P;
     checl_status st = ok ? parse_image(img->host, size, false, &P) : CHECL_ERR_BAD_IMAGE;
