@@ -9,6 +9,7 @@
 #include <cuda_runtime.h>
 #include <fcntl.h>
 #include <signal.h>
+#include <sys/mman.h>
 #include <sys/stat.h>
 #include <unistd.h>
 
@@ -65,32 +66,57 @@ std::atomic<checl_ctx*> g_signal_ctx[kMaxSignal];
 // Pinned host buffers of freed library-owned images, kept for the next image
 // (cudaHostAlloc of a large buffer costs ~1 ms per few MB: an incremental
 // checkpoint loop would otherwise pin a new image every step). Bounded by
-// CHECL_PINNED_POOL_BYTES (default 4 GiB); buffers beyond it are freed.
+// CHECL_PINNED_POOL_BYTES (default 4 GiB); the least recently returned buffers are
+// released first. Pinned sizes are rounded up to size classes (<= 12.5% slack) so
+// that images of similar size reuse each other's buffers.
+size_t pinned_class(size_t n) {
+  if (n <= (2u << 20)) return (n + 4095) & ~(size_t)4095;
+  size_t p2 = 1;
+  while (p2 * 2 <= n) p2 *= 2;
+  const size_t step = std::max<size_t>(p2 / 8, 2u << 20);
+  return (n + step - 1) / step * step;
+}
+
 struct PinnedPool {
   std::mutex mu;
-  std::multimap<size_t, void*> free_;  // capacity -> buffer
+  std::vector<std::pair<size_t, void*>> free_;  // oldest first
   size_t bytes = 0, limit = 0;
   PinnedPool() {
     const char* e = std::getenv("CHECL_PINNED_POOL_BYTES");
     limit = e ? (size_t)std::strtoull(e, nullptr, 10) : (4ull << 30);
   }
-  // a pooled buffer with n <= capacity <= 2n + 64 MiB, or nullptr
+  // the smallest pooled buffer with n <= capacity <= 2n + 64 MiB, or nullptr
   void* take(size_t n, size_t* cap) {
     std::lock_guard<std::mutex> lk(mu);
-    auto it = free_.lower_bound(n);
-    if (it == free_.end() || it->first > 2 * n + (64ull << 20)) return nullptr;
-    void* p = it->second;
-    *cap = it->first;
-    bytes -= it->first;
-    free_.erase(it);
+    size_t best = free_.size();
+    for (size_t i = 0; i < free_.size(); ++i)
+      if (free_[i].first >= n && free_[i].first <= 2 * n + (64ull << 20) &&
+          (best == free_.size() || free_[i].first < free_[best].first))
+        best = i;
+    if (best == free_.size()) return nullptr;
+    void* p = free_[best].second;
+    *cap = free_[best].first;
+    bytes -= *cap;
+    free_.erase(free_.begin() + (long)best);
     return p;
   }
-  bool give(void* p, size_t cap) {
-    std::lock_guard<std::mutex> lk(mu);
-    if (bytes + cap > limit) return false;
-    free_.emplace(cap, p);
-    bytes += cap;
-    return true;
+  void give(void* p, size_t cap) {
+    std::vector<void*> drop;
+    {
+      std::lock_guard<std::mutex> lk(mu);
+      if (cap > limit) {
+        drop.push_back(p);
+      } else {
+        free_.emplace_back(cap, p);
+        bytes += cap;
+        while (bytes > limit) {  // evict the oldest
+          drop.push_back(free_.front().second);
+          bytes -= free_.front().first;
+          free_.erase(free_.begin());
+        }
+      }
+    }
+    for (void* d : drop) cudaFreeHost(d);
   }
 };
 PinnedPool& pinned_pool() {
@@ -429,7 +455,7 @@ struct checl_image {
   void free_host() {
     if (owned && host_mut) {
       if (pinned) {
-        if (!pinned_pool().give(host_mut, host_cap)) cudaFreeHost(host_mut);
+        pinned_pool().give(host_mut, host_cap);
       } else {
         std::free(host_mut);
       }
@@ -444,6 +470,7 @@ struct checl_image {
     void* p = nullptr;
     size_t cap = std::max<size_t>(n, 1);
     if (want_pinned) {
+      cap = pinned_class(cap);
       p = pinned_pool().take(cap, &cap);
       if (!p) ck(cudaHostAlloc(&p, cap, cudaHostAllocDefault));
     } else {
@@ -1974,13 +2001,31 @@ checl_status checl_image_write(const checl_image* img, const char* path, uint32_
     if (bfd < 0) return CHECL_ERR_INVALID_VALUE;
     int dfd = (flags & CHECL_IO_DIRECT) ? ::open(path, O_WRONLY | O_DIRECT) : -1;
     bool ok = true;
-    if (img->location == CHECL_IMAGE_HOST) {
-      ok = parallel_io(img->image_bytes, [&](uint64_t lo, uint64_t hi) {
-        for (uint64_t o = lo; o < hi; o += kIoPiece)
-          if (!write_span(dfd, bfd, img->host + o, std::min<uint64_t>(kIoPiece, hi - o), o)) return false;
-        return true;
-      });
-    } else {
+    if (img->location == CHECL_IMAGE_HOST && img->image_bytes) {
+      // blocks allocated up front: the parallel pieces then overwrite in place
+      if (posix_fallocate(bfd, 0, (off_t)img->image_bytes) != 0) ok = ::ftruncate(bfd, (off_t)img->image_bytes) == 0;
+      void* map = MAP_FAILED;
+      if (ok && (dfd < 0 || (reinterpret_cast<uintptr_t>(img->host) & 4095u)))
+        map = ::mmap(nullptr, img->image_bytes, PROT_WRITE, MAP_SHARED, bfd, 0);
+      if (!ok) {
+      } else if (map != MAP_FAILED) {
+        // page-cache / tmpfs target: parallel copies into the shared mapping (write(2)
+        // on one file serialises on the inode lock; page faults of a mapping do not)
+        uint8_t* m = static_cast<uint8_t*>(map);
+        parallel_io(img->image_bytes, [&](uint64_t lo, uint64_t hi) {
+          std::memcpy(m + lo, img->host + lo, hi - lo);
+          return true;
+        });
+        if (flags & CHECL_IO_SYNC) ok = ::msync(map, img->image_bytes, MS_SYNC) == 0;
+        ::munmap(map, img->image_bytes);
+      } else {
+        ok = parallel_io(img->image_bytes, [&](uint64_t lo, uint64_t hi) {
+          for (uint64_t o = lo; o < hi; o += kIoPiece)
+            if (!write_span(dfd, bfd, img->host + o, std::min<uint64_t>(kIoPiece, hi - o), o)) return false;
+          return true;
+        });
+      }
+    } else if (img->location == CHECL_IMAGE_DEVICE) {
       // device image: the host mirror, then the payload through a pinned bounce buffer
       ok = write_span(dfd, bfd, img->host, img->payload_off, 0);
       DeviceGuard g(img->device);
@@ -2006,7 +2051,7 @@ checl_status checl_image_read(const char* path, uint32_t flags, checl_image** ou
   return guarded([&]() -> checl_status {
     struct stat sb;
     if (::stat(path, &sb) != 0 || sb.st_size < (off_t)kHeaderBytes) return CHECL_ERR_BAD_IMAGE;
-    const uint64_t size = (uint64_t)sb.st_size, cap = align_up(size, 4096);
+    const uint64_t size = (uint64_t)sb.st_size, cap = pinned_class(align_up(size, 4096));
     checl_image* img = new checl_image();
     void* p = nullptr;
     size_t pcap = cap;
