@@ -2002,11 +2002,13 @@ checl_status checl_image_write(const checl_image* img, const char* path, uint32_
     int dfd = (flags & CHECL_IO_DIRECT) ? ::open(path, O_WRONLY | O_DIRECT) : -1;
     bool ok = true;
     if (img->location == CHECL_IMAGE_HOST && img->image_bytes) {
-      // blocks allocated up front: the parallel pieces then overwrite in place
-      if (posix_fallocate(bfd, 0, (off_t)img->image_bytes) != 0) ok = ::ftruncate(bfd, (off_t)img->image_bytes) == 0;
+      const bool direct = dfd >= 0 && (reinterpret_cast<uintptr_t>(img->host) & 4095u) == 0;
+      // O_DIRECT: blocks allocated up front so the parallel pieces overwrite in place;
+      // mapping: only the size (pages are then allocated by the parallel copies)
+      if (!direct || posix_fallocate(bfd, 0, (off_t)img->image_bytes) != 0)
+        ok = ::ftruncate(bfd, (off_t)img->image_bytes) == 0;
       void* map = MAP_FAILED;
-      if (ok && (dfd < 0 || (reinterpret_cast<uintptr_t>(img->host) & 4095u)))
-        map = ::mmap(nullptr, img->image_bytes, PROT_WRITE, MAP_SHARED, bfd, 0);
+      if (ok && !direct) map = ::mmap(nullptr, img->image_bytes, PROT_WRITE, MAP_SHARED, bfd, 0);
       if (!ok) {
       } else if (map != MAP_FAILED) {
         // page-cache / tmpfs target: parallel copies into the shared mapping (write(2)
