@@ -33,7 +33,7 @@
 namespace checl {
 size_t snapshot_smem_bytes();
 cudaError_t snapshot_configure();
-cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel);
+cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel, uint64_t rounds);
 cudaError_t launch_build_tables(const TableParams& tp, uint32_t* out, cudaStream_t s);
 cudaError_t launch_fill(uint8_t* ptr, uint64_t bytes, uint64_t key, int kind, int n_sms, cudaStream_t s);
 cudaError_t launch_compare(const uint8_t* a, const uint8_t* b, uint64_t bytes, unsigned long long* n_diff, int n_sms,
@@ -43,7 +43,7 @@ cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, co
 cudaError_t launch_delta_stages(const ChunkDesc* cdesc, const unsigned long long* totals, uint64_t W, uint64_t n_stages,
                                 unsigned long long* first, unsigned long long* lo, cudaStream_t s);
 cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload_bytes, uint64_t n_chunks,
-                          ChunkDesc* out, int n_sms, cudaStream_t s);
+                          ChunkDesc* out, uint32_t* round_base, uint64_t total_rounds, int n_sms, cudaStream_t s);
 uint32_t host_crc32c_update(uint32_t crc, const void* data, size_t n);
 uint32_t host_crc32c(const void* data, size_t n);
 }  // namespace checl
@@ -291,6 +291,7 @@ struct Plan {
   std::vector<Stage> stages;
   std::vector<uint8_t> meta;  // header (meta_crc = 0, epoch = 0) + manifest
   DevBuf<ChunkDesc> d_desc;
+  DevBuf<uint32_t> d_round;  // round_base of the balanced kernel (n_chunks + 1)
   DevBuf<BufferRecord> d_recs;
 };
 
@@ -302,6 +303,7 @@ struct DevState {
   uint32_t n_slots = 0;
   DevBuf<uint32_t> inv_z, crc_scratch, tables;
   DevBuf<ChunkDesc> desc_scratch;
+  DevBuf<uint32_t> round_scratch;
   DevBuf<BufferRecord> recs_scratch;
   DevBuf<unsigned long long> status;
   DevBuf<unsigned long long> unit_acc;
@@ -333,7 +335,7 @@ struct DevState {
     tables.ensure(kTableWords);
     ck(launch_build_tables(table_params(), tables.p, compute));
     ck(cudaStreamSynchronize(compute));
-    if (const char* k = std::getenv("CHECL_KERNEL")) kernel = std::atoi(k) == 1 ? 1 : std::atoi(k) == 2 ? 2 : 0;
+    if (const char* k = std::getenv("CHECL_KERNEL")) kernel = std::atoi(k) >= 1 && std::atoi(k) <= 3 ? std::atoi(k) : 0;
   }
   void ensure_slots(size_t bytes, uint32_t n) {
     if (slot_bytes == bytes && n_slots == n && slots.p) return;
@@ -354,6 +356,8 @@ struct DevState {
     crc_scratch.release();
     desc_scratch.release();
     recs_scratch.release();
+    round_scratch.release();
+    plan.d_round.release();
     plan.d_recs.release();
     status.release();
     unit_acc.release();
@@ -573,10 +577,19 @@ Layout layout_records(std::vector<BufRec>& bufs) {
 
 // Per-buffer records for the GPU chunk-list expansion (expand_plan_kernel);
 // ptr(b) is the device address of record b (pack: source; restore: destination).
+// Returns the total number of 4 KiB rounds (a chunk of len bytes has ceil(len/4096)).
 template <typename PtrOf>
-void build_records(const std::vector<BufRec>& bufs, PtrOf ptr_of, BufferRecord* out) {
-  for (size_t b = 0; b < bufs.size(); ++b)
-    out[b] = BufferRecord{reinterpret_cast<uint64_t>(ptr_of(b)), bufs[b].size, bufs[b].off, bufs[b].first_chunk};
+uint64_t build_records(const std::vector<BufRec>& bufs, PtrOf ptr_of, BufferRecord* out) {
+  uint64_t rounds = 0;
+  for (size_t b = 0; b < bufs.size(); ++b) {
+    out[b] = BufferRecord{reinterpret_cast<uint64_t>(ptr_of(b)), bufs[b].size, bufs[b].off, bufs[b].first_chunk,
+                          rounds, 0};
+    const uint64_t nch = chunks_of(bufs[b].size);
+    if (nch)
+      rounds += (nch - 1) * (kChunkBytes / kRoundBytes) +
+                (bufs[b].size - (nch - 1) * kChunkBytes + kRoundBytes - 1) / kRoundBytes;
+  }
+  return rounds;
 }
 
 // Stages = maximal runs of consecutive chunks whose image span (chunk bytes plus
@@ -797,18 +810,20 @@ Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
   P.payload_off = L.payload_off;
   P.image_bytes = L.image_bytes;
   P.recs.resize(P.bufs.size());
-  build_records(P.bufs, [&](size_t b) { return P.bufs[b].ptr; }, P.recs.data());
+  const uint64_t rounds = build_records(P.bufs, [&](size_t b) { return P.bufs[b].ptr; }, P.recs.data());
+  if (rounds >= (1ull << 32)) throw std::bad_alloc();  // round_base is u32 (16 TiB of payload)
   P.stages = build_stages(P.bufs, L.payload_bytes, ctx->slot_bytes);
   P.meta.assign(L.crc_off, 0);
   write_header(P.meta.data(), L, P.bufs.size(), device, 0);
   write_manifest(P.meta.data() + kHeaderBytes, P.bufs, device);
   P.d_desc.ensure(std::max<uint64_t>(L.n_chunks, 1));
+  P.d_round.ensure(L.n_chunks + 1);
   P.d_recs.ensure(std::max<size_t>(P.recs.size(), 1));
   if (L.n_chunks) {  // chunk list expanded on the GPU from one record per buffer
     ck(cudaMemcpyAsync(P.d_recs.p, P.recs.data(), P.recs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
-    ck(launch_expand(P.d_recs.p, (uint32_t)P.recs.size(), L.payload_bytes, L.n_chunks, P.d_desc.p, ds.n_sms,
-                     ds.compute));
+    ck(launch_expand(P.d_recs.p, (uint32_t)P.recs.size(), L.payload_bytes, L.n_chunks, P.d_desc.p, P.d_round.p,
+                     rounds, ds.n_sms, ds.compute));
     // no sync: a pageable-source cudaMemcpyAsync returns once P.recs has been staged
   }
   P.version = ctx->version[device];
@@ -826,11 +841,25 @@ LaunchParams base_params(DevState& ds) {
 
 void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0, cudaStream_t s) {
   LaunchParams p = p0;
+  // experiments only (tools/exp_run.py): CHECL_EXP_PACK_OP=2|4 replaces the pack
+  // launches by the CRC-only / copy-only op over the same plan (no valid image)
+  static const int exp_pack_op = [] {
+    const char* e = std::getenv("CHECL_EXP_PACK_OP");
+    return e ? std::atoi(e) : -1;
+  }();
+  if (op == kOpPack && (exp_pack_op == kOpCrc || exp_pack_op == kOpCopy)) op = exp_pack_op;
   const uint64_t chunks = p.c1 - p.c0;
-  // a warp needs ~55 us per 64 KiB chunk in kernel 1: when chunks are fewer than
-  // half the warps, the 4 KiB-unit sweep finishes sooner (tools/size_scan.py)
-  const int kernel = ds.kernel ? ds.kernel : (chunks * 2 <= (uint64_t)ds.n_sms * kWarpsPerCta ? 2 : 1);
-  if (kernel == 2) {
+  // kernel 3 (balanced stretches of rounds) whenever the chunk list has a
+  // round_base; otherwise a warp needs ~55 us per 64 KiB chunk in kernel 1, and when
+  // chunks are fewer than half the warps the 4 KiB-unit sweep finishes sooner
+  // (measured, W = 10: the verify op runs ~4-7% slower in kernel 3 than in kernel
+  // 1 at C2/C3 sizes, so large verify launches stay on kernel 1)
+  int kernel = ds.kernel;
+  if (kernel == 3 && !p.round_base) kernel = 0;
+  const bool small = chunks * 2 <= (uint64_t)ds.n_sms * kWarpsPerCta;
+  if (!kernel) kernel = p.round_base && (op != kOpVerify || small) ? 3 : (small ? 2 : 1);
+  if (kernel != 3) p.round_base = nullptr;
+  if (kernel >= 2) {
     if (ds.unit_acc.cap < chunks) {  // zeroed once; every sweep launch leaves it zero
       ds.unit_acc.ensure(chunks);
       ck(cudaMemsetAsync(ds.unit_acc.p, 0, ds.unit_acc.cap * 8, s));
@@ -839,7 +868,7 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
   }
   cudaEvent_t a = ds.events.get(), b = ds.events.get();
   ck(cudaEventRecord(a, s));
-  ck(launch_snapshot(op, p, ds.n_sms, s, kernel));
+  ck(launch_snapshot(op, p, ds.n_sms, s, kernel, chunks * (kChunkBytes / kRoundBytes)));
   ck(cudaEventRecord(b, s));
   kt.spans.push_back({a, b});
 }
@@ -873,6 +902,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
   Plan& P = get_plan(ctx, ds, device);
   LaunchParams lp = base_params(ds);
   lp.desc = P.d_desc.p;
+  lp.round_base = P.d_round.p;
   tm.plan_ms = now_ms() - tp;
 
   cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
@@ -1086,11 +1116,13 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   const uint64_t nch = P.L.n_chunks;
   ds.h_recs.ensure(std::max<size_t>(P.bufs.size(), 1));
   uint8_t* abase = static_cast<uint8_t*>(arena->base);
-  build_records(P.bufs, [&](size_t b) { return abase + P.bufs[b].off; }, ds.h_recs.p);
+  const uint64_t rounds = build_records(P.bufs, [&](size_t b) { return abase + P.bufs[b].off; }, ds.h_recs.p);
   ds.desc_scratch.ensure(std::max<uint64_t>(nch, 1));
+  ds.round_scratch.ensure(nch + 1);
   ds.recs_scratch.ensure(std::max<size_t>(P.bufs.size(), 1));
   LaunchParams lp = base_params(ds);
   lp.desc = ds.desc_scratch.p;
+  lp.round_base = ds.round_scratch.p;
   tm.plan_ms = now_ms() - tp;
 
   cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
@@ -1098,8 +1130,8 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   if (nch) {  // chunk list expanded on the GPU (compute stream, ahead of the verify launches)
     ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, P.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
-    ck(launch_expand(ds.recs_scratch.p, (uint32_t)P.bufs.size(), P.L.payload_bytes, nch, ds.desc_scratch.p, ds.n_sms,
-                     ds.compute));
+    ck(launch_expand(ds.recs_scratch.p, (uint32_t)P.bufs.size(), P.L.payload_bytes, nch, ds.desc_scratch.p,
+                     ds.round_scratch.p, rounds, ds.n_sms, ds.compute));
   }
   ds.h_status.p[0] = ~0ull;
   ds.h_status.p[1] = 0;
@@ -1236,6 +1268,7 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   // the compacted chunk list and the stage table (delta_scan / delta_stages)
   LaunchParams lp = base_params(ds);
   lp.desc = P.d_desc.p;
+  lp.round_base = P.d_round.p;
   lp.crc = ds.crc_scratch.p;
   lp.c0 = 0;
   lp.c1 = n;
@@ -1279,6 +1312,7 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
   ck(cudaEventRecord(c_begin, ds.copy));
   lp.desc = ds.cdesc.p;
+  lp.round_base = nullptr;  // compacted list: grid-stride kernels
   size_t used = 0;
   for (uint64_t s = 0; s < max_stages; ++s) {
     if (first[s] == first[s + 1]) continue;
@@ -1433,7 +1467,8 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   ds.crc_scratch.ensure(std::max<uint64_t>(nch, 1));
   ds.h_recs.ensure(std::max<size_t>(F.bufs.size(), 1));
   ds.recs_scratch.ensure(std::max<size_t>(F.bufs.size(), 1));
-  build_records(F.bufs, [&](size_t b) { return abase + F.bufs[b].off; }, ds.h_recs.p);
+  const uint64_t rounds = build_records(F.bufs, [&](size_t b) { return abase + F.bufs[b].off; }, ds.h_recs.p);
+  ds.round_scratch.ensure(nch + 1);
   tm.plan_ms = now_ms() - tp;
 
   cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get(), base_in = ds.events.get();
@@ -1452,8 +1487,8 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   if (nch) {
     ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, F.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
-    ck(launch_expand(ds.recs_scratch.p, (uint32_t)F.bufs.size(), F.full_payload, nch, ds.desc_scratch.p, ds.n_sms,
-                     ds.compute));
+    ck(launch_expand(ds.recs_scratch.p, (uint32_t)F.bufs.size(), F.full_payload, nch, ds.desc_scratch.p,
+                     ds.round_scratch.p, rounds, ds.n_sms, ds.compute));
   }
   ck(cudaStreamWaitEvent(ds.compute, base_in, 0));
   // deltas in chain order: fill slot k over PCIe, scatter its spans (later deltas
@@ -1466,6 +1501,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   }
   LaunchParams lp = base_params(ds);
   lp.desc = ds.cdesc.p;
+  lp.round_base = nullptr;  // host-built list: grid-stride kernels
   for (size_t s = 0; s < dst.size(); ++s) {
     const DStage& S = dst[s];
     const uint32_t k = (uint32_t)(s % ds.n_slots);
@@ -1485,6 +1521,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
   // r4: every chunk of the result against the last CRC table, in place
   lp.desc = ds.desc_scratch.p;
+  lp.round_base = ds.round_scratch.p;
   lp.crc = ds.crc_scratch.p;
   lp.c0 = 0;
   lp.c1 = nch;

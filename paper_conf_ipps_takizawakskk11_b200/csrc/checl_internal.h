@@ -38,13 +38,15 @@ struct ChunkDesc {
 };
 static_assert(sizeof(ChunkDesc) == 16, "ChunkDesc is 16 bytes");
 
-// One buffer of a plan (32 bytes); the GPU expands records into ChunkDescs.
+// One buffer of a plan (48 bytes); the GPU expands records into ChunkDescs.
 // ptr = the buffer's device address (pack: source; restore: destination),
-// off = payload offset (256-aligned), first_chunk = global index of its chunk 0.
+// off = payload offset (256-aligned), first_chunk = global index of its chunk 0,
+// first_round = global index of its first 4 KiB round (rounds of the chunk list
+// enumerated in order: a chunk of len bytes has ceil(len / 4096) rounds).
 struct BufferRecord {
-  uint64_t ptr, size, off, first_chunk;
+  uint64_t ptr, size, off, first_chunk, first_round, reserved;
 };
-static_assert(sizeof(BufferRecord) == 32, "BufferRecord is 32 bytes");
+static_assert(sizeof(BufferRecord) == 48, "BufferRecord is 48 bytes");
 
 CHECL_HD uint32_t desc_len(const ChunkDesc& d) { return d.len_pad & 0x1FFFFu; }
 CHECL_HD uint32_t desc_pad(const ChunkDesc& d) { return d.len_pad >> 24; }
@@ -96,11 +98,16 @@ constexpr int kRoundBytes = 4096;
 constexpr int kSegBytes = 128;                   // per lane per round
 constexpr int kRowPitch = kSegBytes + 16;        // padded smem row: conflict-free LDS.128
 #ifndef CHECL_WARPS
-#define CHECL_WARPS 16
+#define CHECL_WARPS 10  // measured best of 4..16 (tools/exp_sweep2.sh): fewer warps contend less for the LSU/MIO
 #endif
 constexpr int kWarpsPerCta = CHECL_WARPS;
 constexpr int kThreadsPerCta = kWarpsPerCta * 32;
 constexpr int kFoldLevels = 5;
+#ifndef CHECL_PREFETCH
+#define CHECL_PREFETCH 1
+#endif
+constexpr int kPrefetch = CHECL_PREFETCH;  // rounds of loads in flight per warp (registers)
+static_assert(kPrefetch == 1 || kPrefetch == 2, "prefetch depth 1 or 2");
 
 // What one launch does with each chunk of its list (the same data path serves
 // every step that streams chunks):
@@ -146,6 +153,8 @@ struct LaunchParams {
   uint32_t* crc;            // pack/crc: output table (global chunk index); verify/check: reference table
   const uint32_t* inv_z;    // kRoundBytes entries, x^(-8z) mod P
   const uint32_t* tables;   // kTableWords words (build_tables)
+  const uint32_t* round_base;  // per chunk: global index of its round 0 (+ one past the end);
+                               // nullptr: the launch runs the grid-stride kernels
   unsigned long long* status;  // verify/check: [0] = first bad chunk (atomicMin), [1] = bad count
   // sweep kernel (one 4 KiB unit per warp-iteration)
   unsigned long long* unit_acc;  // per chunk: low 32 = XOR of unit terms, high = finished-unit mask (zeroed)

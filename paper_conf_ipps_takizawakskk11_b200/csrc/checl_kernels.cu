@@ -134,6 +134,12 @@ struct OpT {
   static constexpr bool kExactTail = kOp == kOpVerify || kOp == kOpScatter;  // destination is a buffer
 };
 
+__device__ __forceinline__ uint32_t warp_xor(uint32_t v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v ^= __shfl_xor_sync(0xFFFFFFFFu, v, o);
+  return v;
+}
+
 __device__ __forceinline__ uint32_t smem_addr(const void* p) {
   return static_cast<uint32_t>(__cvta_generic_to_shared(p));
 }
@@ -300,13 +306,12 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     const int nrounds = (int)((len + kRoundBytes - 1) / kRoundBytes);
     uint32_t ch = lane == 0 ? 0xFFFFFFFFu : 0u;
 
-    uint4 v[8];
-    load_round(v, src, len, mode, 0, lane_off);
-    for (int r = 0; r < nrounds; ++r) {
+    // one round: store + stage it, issue the loads of round r + kPrefetch into the
+    // registers just stored, then CRC the staged round while those loads fly
+    auto round = [&](uint4 (&v)[8], int r) {
       store_round<kOp>(v, dst, len, r, lane_off, tile_w);
       __syncwarp();
-      // next round's loads stay in flight while this round's CRC runs
-      if (r + 1 < nrounds) load_round(v, src, len, mode, r + 1, lane_off);
+      if (r + kPrefetch < nrounds) load_round(v, src, len, mode, r + kPrefetch, lane_off);
       if (O::kCrc) {
         // lane l: segment 32r + l; Horner step over the rest of the round first
         if (r > 0) ch = horner_mul(ch, hb, l4);
@@ -315,7 +320,20 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
         for (int g = 0; g < 8; ++g) ch = crc_step16(ch, row[g], tb, l4);
       }
       __syncwarp();
+    };
+#if CHECL_PREFETCH == 2
+    uint4 va[8], vb[8];
+    load_round(va, src, len, mode, 0, lane_off);
+    if (nrounds > 1) load_round(vb, src, len, mode, 1, lane_off);
+    for (int r = 0; r < nrounds; r += 2) {
+      round(va, r);
+      if (r + 1 < nrounds) round(vb, r + 1);
     }
+#else
+    uint4 v[8];
+    load_round(v, src, len, mode, 0, lane_off);
+    for (int r = 0; r < nrounds; ++r) round(v, r);
+#endif
 
     // Fold the lanes: at level k, lane l (l % 2^(k+1) == 0) shifts its group past
     // the 128*2^k bytes of the group to its right and adds it. The result is the
@@ -330,6 +348,115 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
       }
     }
     finish_chunk<kOp>(p, c, src, dst, len, pad, nrounds, f, lane);
+  }
+}
+
+// ---- balanced kernel: an equal contiguous stretch of rounds per warp ---------
+//
+// The rounds of the launch's chunks, enumerated in order (round_base), are split
+// into one contiguous stretch per warp of the grid, equal to within one round. That
+// removes the wave quantisation of the grid-stride chunk loop (7070 C2 chunks over
+// 1480 warps leave its last wave 78% full; measured C2 pack 168 -> 163 us; a variant
+// taking whole waves first and splitting only the last one measured 168 us). A
+// stretch covers whole chunks and at most a partial chunk at each end. A part [r0, r1) of a chunk of n
+// rounds is CRC'd exactly like a whole chunk (lane chains with Horner steps, lane
+// fold) from a zero register (the CRC init only when r0 = 0), giving F = the
+// register of those rounds; the chunk register is XOR_parts F * x^(8*4096*(n - r1)).
+// Whole chunks finish directly; split ones XOR their term into the chunk's 64-bit
+// accumulator together with their rounds' bits of a completion mask (the sweep
+// kernel's scheme): the part that completes the mask holds the chunk register.
+// Small launches degenerate to about one round per warp.
+constexpr size_t kBalUnitOff = kTileOff;                         // x^(8*4096*k)*x^i table
+constexpr size_t kBalTileOff = kBalUnitOff + (size_t)kUnitWords * 4;
+constexpr size_t kBalMbarOff = kBalTileOff + (size_t)kWarpsPerCta * kStageBytes;
+constexpr size_t kBalSmemBytes = kBalMbarOff + 16;
+static_assert(kBalSmemBytes <= 232448, "fits the 227 KiB opt-in shared memory");
+
+template <int kOp>
+__global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const LaunchParams p) {
+  using O = OpT<kOp>;
+  extern __shared__ __align__(128) uint8_t smem[];
+  if (O::kCrc) {
+    const TableCopy cp[2] = {{0u, (uint32_t)kTabOff, (uint32_t)kSnapTabWords * 4u},
+                             {(uint32_t)kBalUnitOff, (uint32_t)kUnitOff, (uint32_t)kUnitWords * 4u}};
+    load_tables(smem, p.tables, cp, reinterpret_cast<uint64_t*>(smem + kBalMbarOff));
+  }
+  const uint8_t* tb = smem + kTabOff * 4;
+  const uint8_t* hb = smem + kHornerOff * 4;
+  const uint32_t* ftab = reinterpret_cast<const uint32_t*>(smem + kFoldOff * 4);
+  const uint32_t* utab = reinterpret_cast<const uint32_t*>(smem + kBalUnitOff);
+
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint8_t* stage = smem + kBalTileOff + warp * kStageBytes;
+  const uint32_t l4 = (uint32_t)lane * 4u;
+  const unsigned full = 0xFFFFFFFFu;
+  const int g_lane = lane & 7, s_lane = lane >> 3;
+  const uint32_t lane_off = (uint32_t)s_lane * kSegBytes + (uint32_t)g_lane * 16;
+  uint8_t* tile_w = stage + s_lane * kRowPitch + g_lane * 16;
+
+  const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta, wid = (uint64_t)blockIdx.x * kWarpsPerCta + warp;
+  const uint64_t R0 = p.round_base[p.c0], R = p.round_base[p.c1] - R0;
+  uint64_t g = R0 + R * wid / nw;
+  const uint64_t g_end = R0 + R * (wid + 1) / nw;
+  // the chunk holding round g: the last c in [c0, c1) with round_base[c] <= g
+  uint64_t lo = p.c0, hi = p.c1 - 1;
+  while (lo < hi) {
+    const uint64_t mid = (lo + hi + 1) >> 1;
+    if (p.round_base[mid] <= g) lo = mid; else hi = mid - 1;
+  }
+  for (uint64_t cur = lo; g < g_end; ++cur) {
+    const uint64_t rb = p.round_base[cur];
+    const ChunkDesc d = p.desc[cur];
+    const uint32_t len = desc_len(d), pad = desc_pad(d);
+    const uint8_t* src;
+    uint8_t* dst;
+    int mode;
+    chunk_ptrs<kOp>(p, d, src, dst, mode);
+    const int nrounds = (int)((len + kRoundBytes - 1) / kRoundBytes);
+    const int r0 = (int)(g - rb);
+    const int r1 = (int)(g_end - rb < (uint64_t)nrounds ? g_end - rb : (uint64_t)nrounds);
+    g = rb + (uint64_t)r1;
+    uint32_t ch = (lane == 0 && r0 == 0) ? 0xFFFFFFFFu : 0u;
+
+    uint4 v[8];
+    load_round(v, src, len, mode, r0, lane_off);
+    for (int r = r0; r < r1; ++r) {
+      store_round<kOp>(v, dst, len, r, lane_off, tile_w);
+      __syncwarp();
+      if (r + 1 < r1) load_round(v, src, len, mode, r + 1, lane_off);
+      if (O::kCrc) {
+        if (r > r0) ch = horner_mul(ch, hb, l4);
+        const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
+#pragma unroll
+        for (int q = 0; q < 8; ++q) ch = crc_step16(ch, row[q], tb, l4);
+      }
+      __syncwarp();
+    }
+    uint32_t f = ch;
+    if (O::kCrc) {
+#pragma unroll
+      for (int k = 0; k < kFoldLevels; ++k) {
+        const uint32_t o = __shfl_down_sync(full, f, 1 << k);
+        if ((lane & ((2 << k) - 1)) == 0) f = fold_mul(f, ftab + k * 128) ^ o;
+      }
+    }
+    if (!O::kCrc || (r0 == 0 && r1 == nrounds)) {
+      if (O::kCrc || r1 == nrounds) finish_chunk<kOp>(p, cur, src, dst, len, pad, nrounds, f, lane);
+      continue;
+    }
+    // split chunk: this part's term, shifted past the rounds after it
+    f = __shfl_sync(full, f, 0);
+    const int k = nrounds - r1;
+    const uint32_t term = warp_xor(((f >> (31 - lane)) & 1u) ? utab[k * 32 + lane] : 0u);
+    const unsigned long long mine =
+        (unsigned long long)term | ((((1ull << (r1 - r0)) - 1ull) << r0) << 32);
+    unsigned long long old = 0;
+    if (lane == 0) old = atomicXor(&p.unit_acc[cur - p.c0], mine);
+    const unsigned long long now = __shfl_sync(full, old, 0) ^ mine;
+    if ((now >> 32) == (1ull << nrounds) - 1) {
+      if (lane == 0) p.unit_acc[cur - p.c0] = 0ull;  // zero again for the next launch
+      finish_chunk<kOp>(p, cur, src, dst, len, pad, nrounds, (uint32_t)now, lane);
+    }
   }
 }
 
@@ -356,11 +483,6 @@ __device__ __forceinline__ uint32_t lanepos_mul(uint32_t s, const uint8_t* pb, u
   return r;
 }
 
-__device__ __forceinline__ uint32_t warp_xor(uint32_t v) {
-#pragma unroll
-  for (int o = 16; o > 0; o >>= 1) v ^= __shfl_xor_sync(0xFFFFFFFFu, v, o);
-  return v;
-}
 
 template <int kOp>
 __global__ void __launch_bounds__(kThreadsPerCta, 1) sweep_kernel(const LaunchParams p) {
@@ -568,7 +690,9 @@ __global__ void compare_kernel(const uint8_t* a, const uint8_t* b, uint64_t byte
 // The pad of a buffer's last chunk runs to the next record's offset (or to
 // payload_bytes): FORMAT.md "Chunk ownership of padding".
 __global__ void expand_plan_kernel(const BufferRecord* __restrict__ recs, uint32_t n, uint64_t payload_bytes,
-                                   uint64_t n_chunks, ChunkDesc* __restrict__ out) {
+                                   uint64_t n_chunks, ChunkDesc* __restrict__ out, uint32_t* __restrict__ round_base,
+                                   uint64_t total_rounds) {
+  if (blockIdx.x == 0 && threadIdx.x == 0 && round_base) round_base[n_chunks] = (uint32_t)total_rounds;
   for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < n_chunks;
        c += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t lo = 0, hi = n - 1;
@@ -587,6 +711,7 @@ __global__ void expand_plan_kernel(const BufferRecord* __restrict__ recs, uint32
     d.img_off_256 = (uint32_t)((r.off + base) / kBufferAlign);
     d.len_pad = make_len_pad(len, pad);
     out[c] = d;
+    if (round_base) round_base[c] = (uint32_t)(r.first_round + k * (kChunkBytes / kRoundBytes));
   }
 }
 
@@ -679,11 +804,11 @@ __global__ void delta_stages_kernel(const ChunkDesc* __restrict__ cdesc, const u
 // ---- launchers (called from checl_engine.cpp) --------------------------------
 
 cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload_bytes, uint64_t n_chunks,
-                          ChunkDesc* out, int n_sms, cudaStream_t s) {
+                          ChunkDesc* out, uint32_t* round_base, uint64_t total_rounds, int n_sms, cudaStream_t s) {
   if (n_chunks == 0) return cudaSuccess;
   uint64_t blocks = (n_chunks + 255) / 256;
   if (blocks > (uint64_t)n_sms * 8) blocks = (uint64_t)n_sms * 8;
-  expand_plan_kernel<<<(unsigned)blocks, 256, 0, s>>>(recs, n, payload_bytes, n_chunks, out);
+  expand_plan_kernel<<<(unsigned)blocks, 256, 0, s>>>(recs, n, payload_bytes, n_chunks, out, round_base, total_rounds);
   return cudaGetLastError();
 }
 
@@ -694,6 +819,8 @@ static cudaError_t configure_op() {
   cudaError_t e = cudaFuncSetAttribute(snapshot_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(sweep_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
+  if (e == cudaSuccess)
+    e = cudaFuncSetAttribute(balanced_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBalSmemBytes);
   return e;
 }
 
@@ -714,7 +841,9 @@ cudaError_t launch_build_tables(const TableParams& tp, uint32_t* out, cudaStream
 
 template <int kOp>
 static void launch_op(const LaunchParams& p, unsigned ctas, cudaStream_t s, int kernel) {
-  if (kernel == 2)
+  if (kernel == 3)
+    balanced_kernel<kOp><<<ctas, kThreadsPerCta, kBalSmemBytes, s>>>(p);
+  else if (kernel == 2)
     sweep_kernel<kOp><<<ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
   else
     snapshot_kernel<kOp><<<ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
@@ -723,10 +852,12 @@ static void launch_op(const LaunchParams& p, unsigned ctas, cudaStream_t s, int 
 // kernel 1 = warp per chunk (snapshot_kernel), 2 = 4 KiB units swept by the grid
 // (sweep_kernel; p.unit_acc must be zero for the chunk range when the op CRCs —
 // the kernel leaves it zero again)
-cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel) {
+// (3 = balanced_kernel: needs p.round_base; `rounds` = the launch's round count)
+cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel, uint64_t rounds) {
   const uint64_t chunks = p.c1 - p.c0;
   if (chunks == 0) return cudaSuccess;
-  uint64_t ctas = kernel == 2 ? (chunks * 16 + kWarpsPerCta - 1) / kWarpsPerCta : (chunks + kWarpsPerCta - 1) / kWarpsPerCta;
+  const uint64_t units = kernel == 3 ? rounds : kernel == 2 ? chunks * 16 : chunks;
+  uint64_t ctas = (units + kWarpsPerCta - 1) / kWarpsPerCta;
   if (ctas > (uint64_t)n_sms) ctas = (uint64_t)n_sms;
   switch (op) {
     case kOpPack: launch_op<kOpPack>(p, (unsigned)ctas, s, kernel); break;

@@ -1,0 +1,68 @@
+"""-m gpu: every kernel shape of the data path produces the same bytes.
+
+libchecl dispatches a launch to one of three kernels: 1 grid-stride
+warp per chunk, 2 grid-stride 4 KiB units, 3 balanced stretches of rounds (partial
+chunks combined through the atomic CRC accumulator). CHECL_KERNEL=k forces one;
+each run here (a subprocess: the choice is read once per device) checkpoints a
+registry with ragged, misaligned, multi-chunk and zero-size buffers, in one launch
+and through small staging slots, compares the image with the oracle byte for byte,
+restores it (host and HBM images) and checks the restored bytes."""
+import os
+import subprocess
+import sys
+
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+if not torch.cuda.is_available():
+    pytest.skip("needs a CUDA device", allow_module_level=True)
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+SCRIPT = r"""
+import sys
+sys.path.insert(0, %r)
+import numpy as np, torch
+from oracle import oracle as O
+from tests.gpu_util import make_set, oracle_entries, bound_bytes
+from paper_conf_ipps_takizawakskk11_b200 import checl
+sizes = [1 << 20, 0, 65536 * 3 + 17, 4097, 1, 300007, 65535, 65537, 2 << 20]
+for slot in (None, 196608):
+    ctx = checl.Context()
+    if slot:
+        ctx.set_staging(slot, 2)
+    ds = make_set(ctx, sizes, seed=21, offsets=[0, 0, 1, 4, 0, 8, 3, 0, 0])
+    want = O.checkpoint(oracle_entries(ds), device=0, epoch=3)
+    img = ctx.checkpoint(0, epoch=3)
+    assert np.array_equal(img.view(), want), "host image"
+    dimg = ctx.checkpoint_device(0, epoch=3)
+    assert np.array_equal(dimg.view(), want[:dimg.view().size]), "device image metadata"
+    for im in (img, dimg):
+        for t in ds.tensors:
+            t.zero_()
+        rep = ctx.restore(im, 0)
+        assert rep.n_bad_chunks == 0
+        for h, b in zip(ds.handles, ds.host):
+            assert np.array_equal(bound_bytes(ctx, h), b)
+    bad = img.view().copy()
+    poff = int(img.header()["payload_off"])
+    bad[poff + 65536 * 16 + 5] ^= 1
+    st, rep_o, _ = O.restore(bad)
+    try:
+        ctx.restore(checl.Image.wrap(bad), 0)
+        raise SystemExit("corruption not detected")
+    except checl.CheclError as e:
+        assert e.report.first_bad_chunk == rep_o["first_bad_chunk"]
+    ctx.close()
+print("kernel ok")
+"""
+
+
+@pytest.mark.parametrize("kernel", ["1", "2", "3"])
+def test_forced_kernel_shapes_bit_exact(kernel):
+    env = dict(os.environ, CHECL_KERNEL=kernel)
+    r = subprocess.run([sys.executable, "-c", SCRIPT % ROOT], capture_output=True, text=True, env=env, cwd=ROOT,
+                       timeout=600)
+    assert r.returncode == 0 and "kernel ok" in r.stdout, r.stdout + r.stderr
