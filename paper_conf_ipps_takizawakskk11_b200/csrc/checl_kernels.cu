@@ -150,7 +150,17 @@ __device__ __forceinline__ uint32_t smem_addr(const void* p) {
 struct TableCopy {
   uint32_t dst_off, src_word, bytes;
 };
-template <int N>
+__device__ __forceinline__ void wait_tables(uint64_t* mbar) {
+  asm volatile(
+      "{\n .reg .pred p;\n WAIT_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], 0;\n"
+      " @!p bra WAIT_%=;\n}" ::"r"(smem_addr(mbar))
+      : "memory");
+}
+
+// kWait = false: the caller overlaps its first global loads with the table copy
+// and calls wait_tables before the first lookup.
+template <int N, bool kWait = true>
 __device__ __forceinline__ void load_tables(uint8_t* smem, const uint32_t* gtab, const TableCopy (&cp)[N],
                                             uint64_t* mbar) {
   const uint32_t mb = smem_addr(mbar);
@@ -174,11 +184,7 @@ __device__ __forceinline__ void load_tables(uint8_t* smem, const uint32_t* gtab,
     }
   }
   __syncthreads();  // the barrier is initialised before anyone waits on it
-  asm volatile(
-      "{\n .reg .pred p;\n WAIT_%=:\n"
-      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], 0;\n"
-      " @!p bra WAIT_%=;\n}" ::"r"(mb)
-      : "memory");
+  if (kWait) wait_tables(mbar);
 }
 
 // Loads granule set of round `r` (8 x 16 B per lane) of a chunk of `len` bytes.
@@ -379,8 +385,9 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
   if (O::kCrc) {
     const TableCopy cp[2] = {{0u, (uint32_t)kTabOff, (uint32_t)kSnapTabWords * 4u},
                              {(uint32_t)kBalUnitOff, (uint32_t)kUnitOff, (uint32_t)kUnitWords * 4u}};
-    load_tables(smem, p.tables, cp, reinterpret_cast<uint64_t*>(smem + kBalMbarOff));
+    load_tables<2, false>(smem, p.tables, cp, reinterpret_cast<uint64_t*>(smem + kBalMbarOff));
   }
+  bool tables_ready = !O::kCrc;
   const uint8_t* tb = smem + kTabOff * 4;
   const uint8_t* hb = smem + kHornerOff * 4;
   const uint32_t* ftab = reinterpret_cast<const uint32_t*>(smem + kFoldOff * 4);
@@ -398,11 +405,14 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
   const uint64_t R0 = p.round_base[p.c0], R = p.round_base[p.c1] - R0;
   uint64_t g = R0 + R * wid / nw;
   const uint64_t g_end = R0 + R * (wid + 1) / nw;
-  // the chunk holding round g: the last c in [c0, c1) with round_base[c] <= g
-  uint64_t lo = p.c0, hi = p.c1 - 1;
-  while (lo < hi) {
-    const uint64_t mid = (lo + hi + 1) >> 1;
-    if (p.round_base[mid] <= g) lo = mid; else hi = mid - 1;
+  // the chunk holding round g: the last c in [c0, c1) with round_base[c] <= g, by a
+  // 32-way search (one probe per lane: 3 dependent loads for C2, 4 for 1 M chunks)
+  uint64_t lo = p.c0, hi = p.c1;  // invariant: round_base[lo] <= g, answer in [lo, hi)
+  while (hi - lo > 1) {
+    const uint64_t step = (hi - lo + 31) / 32, idx = lo + lane * step;
+    const unsigned m = __ballot_sync(full, idx < hi && p.round_base[idx] <= g);
+    lo += (uint64_t)(31 - __clz(m)) * step;
+    hi = hi < lo + step ? hi : lo + step;
   }
   for (uint64_t cur = lo; g < g_end; ++cur) {
     const uint64_t rb = p.round_base[cur];
@@ -418,12 +428,12 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
     g = rb + (uint64_t)r1;
     uint32_t ch = (lane == 0 && r0 == 0) ? 0xFFFFFFFFu : 0u;
 
-    uint4 v[8];
-    load_round(v, src, len, mode, r0, lane_off);
-    for (int r = r0; r < r1; ++r) {
+    // one round: store + stage it, issue the loads of round r + kPrefetch into the
+    // registers just stored, then CRC the staged round while those loads fly
+    auto round = [&](uint4 (&v)[8], int r) {
       store_round<kOp>(v, dst, len, r, lane_off, tile_w);
       __syncwarp();
-      if (r + 1 < r1) load_round(v, src, len, mode, r + 1, lane_off);
+      if (r + kPrefetch < r1) load_round(v, src, len, mode, r + kPrefetch, lane_off);
       if (O::kCrc) {
         if (r > r0) ch = horner_mul(ch, hb, l4);
         const uint4* row = reinterpret_cast<const uint4*>(stage + lane * kRowPitch);
@@ -431,7 +441,28 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
         for (int q = 0; q < 8; ++q) ch = crc_step16(ch, row[q], tb, l4);
       }
       __syncwarp();
+    };
+#if CHECL_PREFETCH == 2
+    uint4 va[8], vb[8];
+    load_round(va, src, len, mode, r0, lane_off);
+    if (r0 + 1 < r1) load_round(vb, src, len, mode, r0 + 1, lane_off);
+    if (!tables_ready) {
+      wait_tables(reinterpret_cast<uint64_t*>(smem + kBalMbarOff));
+      tables_ready = true;
     }
+    for (int r = r0; r < r1; r += 2) {
+      round(va, r);
+      if (r + 1 < r1) round(vb, r + 1);
+    }
+#else
+    uint4 v[8];
+    load_round(v, src, len, mode, r0, lane_off);
+    if (!tables_ready) {  // the first loads are in flight; the tables have landed by now
+      wait_tables(reinterpret_cast<uint64_t*>(smem + kBalMbarOff));
+      tables_ready = true;
+    }
+    for (int r = r0; r < r1; ++r) round(v, r);
+#endif
     uint32_t f = ch;
     if (O::kCrc) {
 #pragma unroll
@@ -458,6 +489,8 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
       finish_chunk<kOp>(p, cur, src, dst, len, pad, nrounds, (uint32_t)now, lane);
     }
   }
+  // a warp without rounds still waits: the CTA must not exit under the table copy
+  if (!tables_ready) wait_tables(reinterpret_cast<uint64_t*>(smem + kBalMbarOff));
 }
 
 // ---- sweep kernel: one 4 KiB unit per warp-iteration ------------------------

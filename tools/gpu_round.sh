@@ -14,5 +14,5 @@ timeout 300 python bench.py --config C1 --no-cpu-baseline > $O/bench_c1.json 2> 
 timeout 900 python bench.py --config C3 --no-cpu-baseline --steps 5 > $O/bench_c3.json 2> $O/bench_c3.err
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,temperature.gpu,power.draw --format=csv > $O/nvsmi.txt
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 300 --csv --log-file $O/launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline > $O/launches.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:snapshot_kernel -s 2 -c 2 -o $O/prof -f python tools/profile_step.py --reps 2 > $O/ncu_full.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"snapshot_kernel|balanced_kernel" -s 2 -c 2 -o $O/prof -f python tools/profile_step.py --reps 2 > $O/ncu_full.log 2>&1
 tail -1 $O/ncu_full.log
