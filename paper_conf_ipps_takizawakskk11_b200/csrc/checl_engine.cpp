@@ -1062,14 +1062,55 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, const std::shared_ptr<A
       if (a.use_count() == 1 && a->base) ctx->by_addr[a->device].erase(reinterpret_cast<uintptr_t>(a->base));
   }
   // arenas whose last handle moved away are freed here, outside the lock, once
-  // their device is idle
+  // their device is idle (the restore quiesced `device` when it started and has
+  // synchronised its own streams since; another device is synchronised here)
   for (auto& a : dropped) {
-    if (a.use_count() == 1) {
+    if (a.use_count() == 1 && a->device != device) {
       DeviceGuard g(a->device);
       ck(cudaDeviceSynchronize());
     }
     a.reset();
   }
+}
+
+// After a successful restore onto `device`, the chunk list it expanded for the new
+// allocation (ds.desc_scratch / round_scratch) is exactly the plan the next
+// checkpoint of `device` needs when the device's live buffers are the image's: it
+// becomes that plan (buffers swapped, no re-expansion), so a checkpoint right
+// after a restore or migration skips the plan rebuild.
+void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, uint8_t* abase, uint64_t rounds) {
+  std::lock_guard<std::mutex> lk(ctx->mu);
+  uint64_t n_live = 0;
+  for (auto& kv : ctx->entries)
+    if (kv.second.device == device) ++n_live;
+  if (n_live != P.bufs.size() || !P.L.n_chunks) return;
+  Plan& Q = ds.plan;
+  Q.bufs = P.bufs;
+  for (auto& b : Q.bufs) b.ptr = b.size ? abase + b.off : nullptr;
+  Q.n_chunks = P.L.n_chunks;
+  Q.payload_bytes = P.full_payload;
+  Q.crc_off = P.L.crc_off;
+  Q.payload_off = align_up(P.L.crc_off + 4 * P.L.n_chunks, kPayloadAlign);
+  Q.image_bytes = Q.payload_off + Q.payload_bytes;
+  Q.recs.resize(Q.bufs.size());
+  build_records(Q.bufs, [&](size_t b) { return Q.bufs[b].ptr; }, Q.recs.data());
+  Q.stages = build_stages(Q.bufs, Q.payload_bytes, ctx->slot_bytes);
+  Layout L;
+  L.n_chunks = Q.n_chunks;
+  L.payload_bytes = Q.payload_bytes;
+  L.crc_off = Q.crc_off;
+  L.payload_off = Q.payload_off;
+  L.image_bytes = Q.image_bytes;
+  Q.meta.assign(Q.crc_off, 0);
+  write_header(Q.meta.data(), L, Q.bufs.size(), device, 0);
+  write_manifest(Q.meta.data() + kHeaderBytes, Q.bufs, device);
+  std::swap(Q.d_desc.p, ds.desc_scratch.p);
+  std::swap(Q.d_desc.cap, ds.desc_scratch.cap);
+  std::swap(Q.d_round.p, ds.round_scratch.p);
+  std::swap(Q.d_round.cap, ds.round_scratch.cap);
+  (void)rounds;
+  Q.version = ctx->version[device];
+  Q.slot_bytes = ctx->slot_bytes;
 }
 
 checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void* stream, checl_report* rep,
@@ -1210,6 +1251,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   (void)in_migrate;
   const double tc = now_ms();
   commit(ctx, P, device, arena);
+  adopt_plan(ctx, ds, device, P, abase, rounds);
   tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
   ctx->last = tm;
