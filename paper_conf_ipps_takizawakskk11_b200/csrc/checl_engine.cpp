@@ -316,6 +316,7 @@ struct DevState {
   // 1 = warp per chunk (throughput), 2 = 4 KiB units swept by the grid (latency of
   // small launches); 0 = by size; env CHECL_KERNEL=1|2 forces one
   int kernel = 0;
+  uint64_t aux_launches = 0;  // plan expansion / delta scan kernels (checl_timing.n_kernels)
   PinnedBuf<unsigned long long> h_status;
   PinnedBuf<BufferRecord> h_recs;
   EventPool events;
@@ -822,6 +823,7 @@ Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
   if (L.n_chunks) {  // chunk list expanded on the GPU from one record per buffer
     ck(cudaMemcpyAsync(P.d_recs.p, P.recs.data(), P.recs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
+    ++ds.aux_launches;
     ck(launch_expand(P.d_recs.p, (uint32_t)P.recs.size(), L.payload_bytes, L.n_chunks, P.d_desc.p, P.d_round.p,
                      rounds, ds.n_sms, ds.compute));
     // no sync: a pageable-source cudaMemcpyAsync returns once P.recs has been staged
@@ -888,6 +890,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
   const double t0 = now_ms();
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
+  const uint64_t aux0 = ds.aux_launches;
   ds.events.reset();
   KernelTimer kt;
   checl_timing tm{};
@@ -990,7 +993,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
   float cms = 0;
   if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
   tm.kernel_ms = kt.sum_ms();
-  tm.n_kernels = kt.spans.size();
+  tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tm.total_ms = now_ms() - t0;
   ctx->last = tm;
   return CHECL_SUCCESS;
@@ -1118,6 +1121,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   const double t0 = now_ms();
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
+  const uint64_t aux0 = ds.aux_launches;
   ds.events.reset();
   KernelTimer kt;
   checl_timing tm{};
@@ -1171,6 +1175,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   if (nch) {  // chunk list expanded on the GPU (compute stream, ahead of the verify launches)
     ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, P.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
+    ++ds.aux_launches;
     ck(launch_expand(ds.recs_scratch.p, (uint32_t)P.bufs.size(), P.L.payload_bytes, nch, ds.desc_scratch.p,
                      ds.round_scratch.p, rounds, ds.n_sms, ds.compute));
   }
@@ -1239,7 +1244,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   float cms = 0;
   if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
   tm.kernel_ms = kt.sum_ms();
-  tm.n_kernels = kt.spans.size();
+  tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tmp_payload.release();
   tmp_crc.release();
   if (rep) set_report(rep, P, n_bad, first_bad);
@@ -1277,6 +1282,7 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   const double t0 = now_ms();
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
+  const uint64_t aux0 = ds.aux_launches;
   {
     // the plan (and so the layout test) needs the registry as of this call
     Plan& P0 = get_plan(ctx, ds, device);
@@ -1318,6 +1324,7 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   if (n) timed_launch(ds, kt, kOpCrc, lp, ds.compute);
   cudaEvent_t sa = ds.events.get(), sb = ds.events.get();
   ck(cudaEventRecord(sa, ds.compute));
+  ds.aux_launches += 2;
   ck(launch_delta_scan(P.d_desc.p, ds.crc_scratch.p, ds.base_crc.p, n, ds.map_words.p, ds.cdesc.p, ds.dtotals.p,
                        ds.compute));
   ck(launch_delta_stages(ds.cdesc.p, ds.dtotals.p, W, max_stages, ds.stage_first.p, ds.stage_lo.p, ds.compute));
@@ -1402,7 +1409,7 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   float cms = 0;
   if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
   tm.kernel_ms = kt.sum_ms();
-  tm.n_kernels = kt.spans.size();
+  tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tm.total_ms = now_ms() - t0;
   ctx->last = tm;
   return CHECL_SUCCESS;
@@ -1438,6 +1445,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   const Parsed& Z = Ps[n_img - 1];
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
+  const uint64_t aux0 = ds.aux_launches;
   ds.events.reset();
   KernelTimer kt;
   checl_timing tm{};
@@ -1529,6 +1537,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   if (nch) {
     ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, F.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
+    ++ds.aux_launches;
     ck(launch_expand(ds.recs_scratch.p, (uint32_t)F.bufs.size(), F.full_payload, nch, ds.desc_scratch.p,
                      ds.round_scratch.p, rounds, ds.n_sms, ds.compute));
   }
@@ -1577,7 +1586,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   float cms = 0;
   if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
   tm.kernel_ms = kt.sum_ms();
-  tm.n_kernels = kt.spans.size();
+  tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tm.n_stages = dst.size() + 1;
   if (rep) set_report(rep, Z, n_bad, first_bad);
   if (n_bad) {
