@@ -854,12 +854,10 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
   // kernel 3 (balanced stretches of rounds) whenever the chunk list has a
   // round_base; otherwise a warp needs ~55 us per 64 KiB chunk in kernel 1, and when
   // chunks are fewer than half the warps the 4 KiB-unit sweep finishes sooner
-  // (measured, W = 10: the verify op runs ~4-7% slower in kernel 3 than in kernel
-  // 1 at C2/C3 sizes, so large verify launches stay on kernel 1)
   int kernel = ds.kernel;
   if (kernel == 3 && !p.round_base) kernel = 0;
   const bool small = chunks * 2 <= (uint64_t)ds.n_sms * kWarpsPerCta;
-  if (!kernel) kernel = p.round_base && (op != kOpVerify || small) ? 3 : (small ? 2 : 1);
+  if (!kernel) kernel = p.round_base ? 3 : (small ? 2 : 1);
   if (kernel != 3) p.round_base = nullptr;
   if (kernel >= 2) {
     if (ds.unit_acc.cap < chunks) {  // zeroed once; every sweep launch leaves it zero
