@@ -43,7 +43,8 @@ cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, co
 cudaError_t launch_delta_stages(const ChunkDesc* cdesc, const unsigned long long* totals, uint64_t W, uint64_t n_stages,
                                 unsigned long long* first, unsigned long long* lo, cudaStream_t s);
 cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload_bytes, uint64_t n_chunks,
-                          ChunkDesc* out, uint32_t* round_base, uint64_t total_rounds, int n_sms, cudaStream_t s);
+                          ChunkDesc* out, uint32_t* round_base, uint64_t total_rounds, unsigned long long* status,
+                          int n_sms, cudaStream_t s);
 uint32_t host_crc32c_update(uint32_t crc, const void* data, size_t n);
 uint32_t host_crc32c(const void* data, size_t n);
 }  // namespace checl
@@ -509,6 +510,10 @@ struct checl_ctx {
   uint32_t n_slots = 2;
   checl_timing last{};
   checl_image* mig_img[kMaxDevices] = {};  // migration images, reused (HBM of the source)
+  // the last allocation a commit released on each device, kept for the next restore
+  // of (nearly) the same size: skips an allocator round trip per restore (a
+  // checkpoint/restore loop re-creates a same-sized arena every time)
+  std::shared_ptr<Arena> spare[kMaxDevices];
 
   DevState& dev(int d) {
     if (!devs[d]) {
@@ -825,7 +830,7 @@ Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
                        ds.compute));
     ++ds.aux_launches;
     ck(launch_expand(P.d_recs.p, (uint32_t)P.recs.size(), L.payload_bytes, L.n_chunks, P.d_desc.p, P.d_round.p,
-                     rounds, ds.n_sms, ds.compute));
+                     rounds, nullptr, ds.n_sms, ds.compute));
     // no sync: a pageable-source cudaMemcpyAsync returns once P.recs has been staged
   }
   P.version = ctx->version[device];
@@ -935,9 +940,17 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
     lp.image = img->d_payload;
     lp.image_base = 0;
     lp.crc = img->d_crc;
+    // the host mirror's CRC table is written by the kernel itself through the
+    // mapped pinned mirror (no D2H copy after the kernel); plain copy if unmapped
+    void* mirror = nullptr;
+    if (cudaHostGetDevicePointer(&mirror, img->host_mut + P.crc_off, 0) != cudaSuccess) {
+      cudaGetLastError();
+      mirror = nullptr;
+    }
+    lp.crc_mirror = static_cast<uint32_t*>(mirror);
     if (P.n_chunks) timed_launch(ds, kt, kOpPack, lp, ds.compute);
     ck(cudaEventRecord(c_begin, ds.compute));
-    if (P.n_chunks)
+    if (P.n_chunks && !mirror)
       ck(cudaMemcpyAsync(img->host_mut + P.crc_off, img->d_crc, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.compute));
     ck(cudaEventRecord(c_end, ds.compute));
     tm.n_stages = 1;
@@ -1029,6 +1042,35 @@ bool ensure_peer(int dev, int peer) {
   return true;
 }
 
+// r2: one allocation of `bytes` on `device` (through the context's allocator), or
+// the spare the last commit on this device released when it is large enough and
+// at most 1/8 larger. nullptr when the allocator fails.
+std::shared_ptr<Arena> new_arena(checl_ctx* ctx, int device, void* stream, uint64_t bytes) {
+  {
+    std::lock_guard<std::mutex> lk(ctx->mu);
+    std::shared_ptr<Arena>& sp = ctx->spare[device];
+    if (sp && bytes && sp->bytes >= bytes && sp->bytes - bytes <= bytes / 8) {
+      std::shared_ptr<Arena> a = std::move(sp);
+      return a;
+    }
+  }
+  auto arena = std::make_shared<Arena>();
+  arena->alloc = ctx->alloc;
+  arena->device = device;
+  arena->stream = stream;
+  arena->bytes = bytes;
+  if (bytes) {
+    if (ctx->alloc.alloc)
+      arena->base = ctx->alloc.alloc(bytes, device, stream, ctx->alloc.user);
+    else if (cudaMalloc(&arena->base, bytes) != cudaSuccess) {
+      cudaGetLastError();
+      arena->base = nullptr;
+    }
+    if (!arena->base) return nullptr;
+  }
+  return arena;
+}
+
 // Swaps every handle of the image to its new buffer (L15); frees library-owned
 // buffers previously bound to those handles (after their devices are idle).
 void commit(checl_ctx* ctx, const Parsed& P, int device, const std::shared_ptr<Arena>& arena) {
@@ -1069,6 +1111,15 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, const std::shared_ptr<A
     if (a.use_count() == 1 && a->device != device) {
       DeviceGuard g(a->device);
       ck(cudaDeviceSynchronize());
+    }
+    if (a.use_count() == 1 && a->base) {  // becomes the device's spare (the previous spare is freed)
+      std::shared_ptr<Arena> old;
+      {
+        std::lock_guard<std::mutex> lk(ctx->mu);
+        old = std::move(ctx->spare[a->device]);
+        ctx->spare[a->device] = std::move(a);
+      }
+      old.reset();
     }
     a.reset();
   }
@@ -1140,21 +1191,9 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   if (rep) set_report(rep, P, 0, 0);
 
   // r2: re-create the buffers: one allocation laid out like the payload
-  auto arena = std::make_shared<Arena>();
-  arena->alloc = ctx->alloc;
-  arena->device = device;
-  arena->stream = stream;
   const double ta = now_ms();
-  arena->bytes = P.L.payload_bytes;
-  if (P.L.payload_bytes) {
-    if (ctx->alloc.alloc)
-      arena->base = ctx->alloc.alloc(P.L.payload_bytes, device, stream, ctx->alloc.user);
-    else if (cudaMalloc(&arena->base, P.L.payload_bytes) != cudaSuccess) {
-      cudaGetLastError();
-      arena->base = nullptr;
-    }
-    if (!arena->base) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
-  }
+  auto arena = new_arena(ctx, device, stream, P.L.payload_bytes);
+  if (!arena) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
   tm.alloc_ms = now_ms() - ta;
   const uint64_t nch = P.L.n_chunks;
   ds.h_recs.ensure(std::max<size_t>(P.bufs.size(), 1));
@@ -1169,17 +1208,14 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   tm.plan_ms = now_ms() - tp;
 
   cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
-  ck(cudaEventRecord(c_begin, ds.copy));
-  if (nch) {  // chunk list expanded on the GPU (compute stream, ahead of the verify launches)
+  if (nch) {  // chunk list expanded on the GPU (compute stream, ahead of the verify launches);
+              // the same launch initialises the verify status
     ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, P.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
     ++ds.aux_launches;
     ck(launch_expand(ds.recs_scratch.p, (uint32_t)P.bufs.size(), P.L.payload_bytes, nch, ds.desc_scratch.p,
-                     ds.round_scratch.p, rounds, ds.n_sms, ds.compute));
+                     ds.round_scratch.p, rounds, ds.status.p, ds.n_sms, ds.compute));
   }
-  ds.h_status.p[0] = ~0ull;
-  ds.h_status.p[1] = 0;
-  ck(cudaMemcpyAsync(ds.status.p, ds.h_status.p, 16, cudaMemcpyHostToDevice, ds.copy));
   DevBuf<uint8_t> tmp_payload;  // only when the source device is not peer-reachable
   DevBuf<uint32_t> tmp_crc;
   if (dev_img) {
@@ -1187,6 +1223,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     const uint8_t* src = img->d_payload;
     const uint32_t* crc = img->d_crc;
     if (!ensure_peer(device, img->device)) {
+      ck(cudaEventRecord(c_begin, ds.copy));
       tmp_payload.ensure(P.L.payload_bytes + kSlotSlack);
       tmp_crc.ensure(std::max<uint64_t>(nch, 1));
       if (P.L.payload_bytes)
@@ -1194,9 +1231,12 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
       if (nch) ck(cudaMemcpyPeerAsync(tmp_crc.p, device, img->d_crc, img->device, 4 * nch, ds.copy));
       src = tmp_payload.p;
       crc = tmp_crc.p;
+      ck(cudaEventRecord(c_end, ds.copy));
+      ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
+    } else {  // nothing to copy: the kernel reads the image where it is
+      ck(cudaEventRecord(c_begin, ds.compute));
+      ck(cudaEventRecord(c_end, ds.compute));
     }
-    ck(cudaEventRecord(c_end, ds.copy));
-    ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
     lp.c0 = 0;
     lp.c1 = nch;
     lp.image = const_cast<uint8_t*>(src);
@@ -1206,6 +1246,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     tm.n_stages = 1;
   } else {
     // r3 + r4: fill slot s % n_slots over PCIe while the previous slot is verified
+    ck(cudaEventRecord(c_begin, ds.copy));
     ds.ensure_slots(ctx->slot_bytes, ctx->n_slots);
     ds.crc_scratch.ensure(std::max<uint64_t>(nch, 1));
     if (nch) ck(cudaMemcpyAsync(ds.crc_scratch.p, img->host + P.L.crc_off, 4 * nch, cudaMemcpyHostToDevice, ds.copy));
@@ -1235,7 +1276,12 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     if (stages.empty()) ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
     tm.n_stages = stages.size();
   }
-  ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
+  if (nch) {
+    ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
+  } else {
+    ds.h_status.p[0] = ~0ull;
+    ds.h_status.p[1] = 0;
+  }
   ck(cudaStreamSynchronize(ds.compute));
   ck(cudaStreamSynchronize(ds.copy));
   const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
@@ -1453,21 +1499,9 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   if (rep) set_report(rep, Z, 0, 0);
 
   // r2: one allocation laid out like the full payload
-  auto arena = std::make_shared<Arena>();
-  arena->alloc = ctx->alloc;
-  arena->device = device;
-  arena->stream = stream;
-  arena->bytes = F.full_payload;
   const double ta = now_ms();
-  if (F.full_payload) {
-    if (ctx->alloc.alloc)
-      arena->base = ctx->alloc.alloc(F.full_payload, device, stream, ctx->alloc.user);
-    else if (cudaMalloc(&arena->base, F.full_payload) != cudaSuccess) {
-      cudaGetLastError();
-      arena->base = nullptr;
-    }
-    if (!arena->base) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
-  }
+  auto arena = new_arena(ctx, device, stream, F.full_payload);
+  if (!arena) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
   tm.alloc_ms = now_ms() - ta;
   uint8_t* abase = static_cast<uint8_t*>(arena->base);
   const uint64_t nch = F.L.n_chunks;
@@ -1529,15 +1563,12 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
     ck(cudaMemcpyAsync(ds.crc_scratch.p, chain[n_img - 1]->host + Z.L.crc_off, 4 * nch, cudaMemcpyHostToDevice, ds.copy));
   if (!hdesc.empty())
     ck(cudaMemcpyAsync(ds.cdesc.p, hdesc.data(), hdesc.size() * sizeof(ChunkDesc), cudaMemcpyHostToDevice, ds.copy));
-  ds.h_status.p[0] = ~0ull;
-  ds.h_status.p[1] = 0;
-  ck(cudaMemcpyAsync(ds.status.p, ds.h_status.p, 16, cudaMemcpyHostToDevice, ds.copy));
-  if (nch) {
+  if (nch) {  // the expansion also initialises the verify status
     ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, F.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
     ++ds.aux_launches;
     ck(launch_expand(ds.recs_scratch.p, (uint32_t)F.bufs.size(), F.full_payload, nch, ds.desc_scratch.p,
-                     ds.round_scratch.p, rounds, ds.n_sms, ds.compute));
+                     ds.round_scratch.p, rounds, ds.status.p, ds.n_sms, ds.compute));
   }
   ck(cudaStreamWaitEvent(ds.compute, base_in, 0));
   // deltas in chain order: fill slot k over PCIe, scatter its spans (later deltas
@@ -1576,8 +1607,13 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   lp.c1 = nch;
   lp.image = nullptr;
   lp.image_base = 0;
-  if (nch) timed_launch(ds, kt, kOpCheck, lp, ds.compute);
-  ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
+  if (nch) {
+    timed_launch(ds, kt, kOpCheck, lp, ds.compute);
+    ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
+  } else {
+    ds.h_status.p[0] = ~0ull;
+    ds.h_status.p[1] = 0;
+  }
   ck(cudaStreamSynchronize(ds.compute));
   ck(cudaStreamSynchronize(ds.copy));
   const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
@@ -1638,6 +1674,7 @@ checl_status checl_destroy(checl_ctx* ctx) {
       }
       ctx->entries.clear();
       arenas.clear();
+      for (auto& sp : ctx->spare) sp.reset();
     }
     for (auto*& d : ctx->devs) {
       if (d) {

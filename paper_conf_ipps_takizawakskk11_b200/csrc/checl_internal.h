@@ -151,6 +151,7 @@ struct LaunchParams {
   uint8_t* image;           // pack/copy: destination slot; verify: source (may be a peer address)
   uint64_t image_base;      // payload offset that maps to image[0]
   uint32_t* crc;            // pack/crc: output table (global chunk index); verify/check: reference table
+  uint32_t* crc_mirror;     // pack/crc: optional second copy of the table in mapped pinned host memory
   const uint32_t* inv_z;    // kRoundBytes entries, x^(-8z) mod P
   const uint32_t* tables;   // kTableWords words (build_tables)
   const uint32_t* round_base;  // per chunk: global index of its round 0 (+ one past the end);

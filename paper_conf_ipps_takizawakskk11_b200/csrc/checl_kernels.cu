@@ -266,6 +266,7 @@ __device__ __forceinline__ void finish_chunk(const LaunchParams& p, uint64_t c, 
     const uint32_t out = ~(zp ? gf_mul(f, p.inv_z[zp]) : f);
     if (!O::kCompare) {
       p.crc[c] = out;
+      if (p.crc_mirror) p.crc_mirror[c] = out;  // posted write into the image's pinned host mirror
     } else if (out != p.crc[c] || pad_bad) {
       atomicMin(&p.status[0], (unsigned long long)c);
       atomicAdd(&p.status[1], 1ull);
@@ -729,8 +730,11 @@ __global__ void compare_kernel(const uint8_t* a, const uint8_t* b, uint64_t byte
 // payload_bytes): FORMAT.md "Chunk ownership of padding".
 __global__ void expand_plan_kernel(const BufferRecord* __restrict__ recs, uint32_t n, uint64_t payload_bytes,
                                    uint64_t n_chunks, ChunkDesc* __restrict__ out, uint32_t* __restrict__ round_base,
-                                   uint64_t total_rounds) {
-  if (blockIdx.x == 0 && threadIdx.x == 0 && round_base) round_base[n_chunks] = (uint32_t)total_rounds;
+                                   uint64_t total_rounds, unsigned long long* __restrict__ status) {
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    if (round_base) round_base[n_chunks] = (uint32_t)total_rounds;
+    if (status) status[0] = ~0ull, status[1] = 0ull;  // the verify status of the launches that follow
+  }
   for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < n_chunks;
        c += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t lo = 0, hi = n - 1;
@@ -842,11 +846,13 @@ __global__ void delta_stages_kernel(const ChunkDesc* __restrict__ cdesc, const u
 // ---- launchers (called from checl_engine.cpp) --------------------------------
 
 cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload_bytes, uint64_t n_chunks,
-                          ChunkDesc* out, uint32_t* round_base, uint64_t total_rounds, int n_sms, cudaStream_t s) {
+                          ChunkDesc* out, uint32_t* round_base, uint64_t total_rounds, unsigned long long* status,
+                          int n_sms, cudaStream_t s) {
   if (n_chunks == 0) return cudaSuccess;
   uint64_t blocks = (n_chunks + 255) / 256;
   if (blocks > (uint64_t)n_sms * 8) blocks = (uint64_t)n_sms * 8;
-  expand_plan_kernel<<<(unsigned)blocks, 256, 0, s>>>(recs, n, payload_bytes, n_chunks, out, round_base, total_rounds);
+  expand_plan_kernel<<<(unsigned)blocks, 256, 0, s>>>(recs, n, payload_bytes, n_chunks, out, round_base, total_rounds,
+                                                      status);
   return cudaGetLastError();
 }
 
