@@ -278,8 +278,13 @@ def _torch_allocator():
 class Context:
     """The CheCL object database + handle table of one process (L15, L19)."""
 
-    def __init__(self, allocator: str = "torch", slot_bytes: Optional[int] = None, n_slots: int = 2):
-        self._alloc = _torch_allocator() if allocator == "torch" else None
+    def __init__(self, allocator="torch", slot_bytes: Optional[int] = None, n_slots: int = 2):
+        """allocator: "torch" (the caching allocator), "cuda" (cudaMalloc / cudaFree),
+        or an `Allocator` struct of C callbacks (kept alive by the context)."""
+        if isinstance(allocator, Allocator):
+            self._alloc = allocator
+        else:
+            self._alloc = _torch_allocator() if allocator == "torch" else None
         out = C.c_void_p()
         _check(lib.checl_create(C.byref(self._alloc) if self._alloc is not None else None, C.byref(out)), "checl_create")
         self._p = out
