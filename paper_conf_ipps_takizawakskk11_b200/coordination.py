@@ -3,9 +3,9 @@
 PAPER.md L40 §IV-C: "The checkpoint files of individual computing nodes, called
 local snapshots, are aggregated into a global snapshot [14]" (Open MPI's CPR). Here
 each rank snapshots its own GPU's buffers independently (no data crosses ranks);
-the only exchange is a 40-byte status all-reduce over the process group (NCCL over
-NVLink on GPUs, gloo in CPU tests): SUM of [failures, buffers, bytes] and MAX of
-[epoch, -epoch]. The global snapshot commits iff no rank failed and every rank
+the only exchange is one 88-byte status all-reduce over the process group (NCCL over
+NVLink on GPUs, gloo in CPU tests): SUM of [failures, buffers, bytes] and of the
+epoch's 16-bit parts and their squares (agreement test in `agree`). The global snapshot commits iff no rank failed and every rank
 checkpointed the same epoch (reading 16: a two-phase commit); otherwise
 every rank frees its local image.
 """
@@ -27,17 +27,26 @@ class GlobalSnapshot:
 
 
 def agree(failed: bool, n_buffers: int, nbytes: int, epoch: int, group=None, device=None) -> Tuple[int, int, int, bool, int]:
-    """The coordination all-reduce. Returns (failures, buffers, bytes, epochs_agree, epoch)."""
+    """The coordination all-reduce — ONE all-reduce (SUM) of 11 int64 per rank.
+    Returns (failures, buffers, bytes, epochs_agree, epoch).
+
+    Epoch agreement without a MAX: the 64-bit epoch is split into four 16-bit parts
+    x_k and every rank contributes x_k and x_k^2; by the equality case of
+    Cauchy-Schwarz, all ranks hold the same x_k iff N * sum(x_k^2) == (sum x_k)^2
+    (exact: x_k < 2^16, so nothing overflows int64 for any world size < 2^31)."""
     import torch
     import torch.distributed as dist
 
     dev = torch.device("cuda", device) if (device is not None and dist.get_backend(group) == "nccl") else torch.device("cpu")
-    s = torch.tensor([1 if failed else 0, n_buffers, nbytes], dtype=torch.int64, device=dev)
-    e = torch.tensor([epoch, -epoch], dtype=torch.int64, device=dev)
+    e = epoch & 0xFFFFFFFFFFFFFFFF
+    parts = [(e >> (16 * k)) & 0xFFFF for k in range(4)]
+    s = torch.tensor([1 if failed else 0, n_buffers, nbytes] + parts + [x * x for x in parts], dtype=torch.int64, device=dev)
     dist.all_reduce(s, op=dist.ReduceOp.SUM, group=group)
-    dist.all_reduce(e, op=dist.ReduceOp.MAX, group=group)
-    s, e = s.cpu().tolist(), e.cpu().tolist()
-    return int(s[0]), int(s[1]), int(s[2]), e[0] == -e[1], int(e[0])
+    v = s.cpu().tolist()
+    n = dist.get_world_size(group)
+    same = all(n * v[7 + k] == v[3 + k] * v[3 + k] for k in range(4))
+    agreed = sum((v[3 + k] // n) << (16 * k) for k in range(4)) if same else epoch
+    return int(v[0]), int(v[1]), int(v[2]), same, int(agreed)
 
 
 def coordinated(take_local: Callable[[], Tuple[object, int, int]], epoch: int, group=None,

@@ -38,6 +38,10 @@ def _worker(rank, world, port, scenario, q):
         return img, 3 + rank, 1000 * (rank + 1)
 
     epoch = 7 if not (scenario == "epoch" and rank == 0) else 8
+    if scenario == "epoch_hi":  # differ only in the top 16 bits
+        epoch = 7 + ((1 << 48) if rank == 1 else 0)
+    if scenario == "epoch_big":  # equal, all 64 bits in use
+        epoch = (1 << 63) - 3
     g = coordinated(local, epoch)
     q.put((rank, g.committed, g.failures, g.n_buffers, g.total_bytes, g.epochs_agree, img.freed, g.image is None))
     dist.destroy_process_group()
@@ -77,3 +81,10 @@ def test_one_failing_rank_aborts_everyone(world):
 def test_epoch_disagreement_aborts():
     for rank, ok, f, nb, tb, same, freed, none in _run(2, "epoch"):
         assert not ok and f == 0 and not same and none
+
+
+def test_epoch_agreement_exact_in_every_16_bit_part():
+    for rank, ok, f, nb, tb, same, freed, none in _run(3, "epoch_hi"):
+        assert not ok and not same and none
+    for rank, ok, f, nb, tb, same, freed, none in _run(3, "epoch_big"):
+        assert ok and same and not none
