@@ -46,7 +46,7 @@ EXPORTS = (
     "checl_version", "checl_debug_fill", "checl_debug_compare", "checl_debug_corrupt",
     "checl_checkpoint_incremental", "checl_restore_chain", "checl_image_merge",
     "checl_request_checkpoint", "checl_checkpoint_pending", "checl_install_signal", "checl_sync_point",
-    "checl_image_write", "checl_image_read",
+    "checl_image_write", "checl_image_read", "checl_trim",
 )
 
 
@@ -105,6 +105,7 @@ def _load() -> C.CDLL:
         "checl_sync_point": [P, C.c_int, V, U64, P, PP],
         "checl_image_write": [P, C.c_char_p, U32],
         "checl_image_read": [C.c_char_p, U32, PP],
+        "checl_trim": [P],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -427,6 +428,10 @@ class Context:
         if not out.value:
             return None
         return into if into is not None else Image(out.value)
+
+    def trim(self):
+        """Release the spare allocations and pooled pinned buffers kept for reuse."""
+        _check(lib.checl_trim(self._p), "checl_trim")
 
     def last_timing(self) -> dict:
         t = _Timing()

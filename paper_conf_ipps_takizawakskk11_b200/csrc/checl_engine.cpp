@@ -101,6 +101,15 @@ struct PinnedPool {
     free_.erase(free_.begin() + (long)best);
     return p;
   }
+  void trim() {
+    std::vector<std::pair<size_t, void*>> all;
+    {
+      std::lock_guard<std::mutex> lk(mu);
+      all.swap(free_);
+      bytes = 0;
+    }
+    for (auto& e : all) cudaFreeHost(e.second);
+  }
   void give(void* p, size_t cap) {
     std::vector<void*> drop;
     {
@@ -1042,6 +1051,16 @@ bool ensure_peer(int dev, int peer) {
   return true;
 }
 
+// Largest allocation kept as a spare (CHECL_SPARE_BYTES, default 4 GiB): larger
+// re-creations amortise their allocator call anyway, and a spare holds HBM idle.
+uint64_t spare_limit() {
+  static const uint64_t v = [] {
+    const char* e = std::getenv("CHECL_SPARE_BYTES");
+    return e ? (uint64_t)std::strtoull(e, nullptr, 10) : (4ull << 30);
+  }();
+  return v;
+}
+
 // r2: one allocation of `bytes` on `device` (through the context's allocator), or
 // the spare the last commit on this device released when it is large enough and
 // at most 1/8 larger. nullptr when the allocator fails.
@@ -1112,7 +1131,7 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, const std::shared_ptr<A
       DeviceGuard g(a->device);
       ck(cudaDeviceSynchronize());
     }
-    if (a.use_count() == 1 && a->base) {  // becomes the device's spare (the previous spare is freed)
+    if (a.use_count() == 1 && a->base && a->bytes <= spare_limit()) {  // the device's spare (the previous is freed)
       std::shared_ptr<Arena> old;
       {
         std::lock_guard<std::mutex> lk(ctx->mu);
@@ -2219,6 +2238,20 @@ checl_status checl_image_read(const char* path, uint32_t flags, checl_image** ou
     img->image_bytes = P.L.image_bytes;
     img->payload_off = P.L.payload_off;
     *out = img;
+    return CHECL_SUCCESS;
+  });
+}
+
+checl_status checl_trim(checl_ctx* ctx) {
+  if (!ctx) return CHECL_ERR_INVALID_VALUE;
+  return guarded([&]() -> checl_status {
+    std::shared_ptr<Arena> drop[kMaxDevices];
+    {
+      std::lock_guard<std::mutex> lk(ctx->mu);
+      for (int d = 0; d < kMaxDevices; ++d) drop[d] = std::move(ctx->spare[d]);
+    }
+    for (auto& a : drop) a.reset();
+    pinned_pool().trim();
     return CHECL_SUCCESS;
   });
 }

@@ -95,6 +95,8 @@ def test_cudamalloc_allocator_round_trip():
     assert np.array_equal(img.view(), O.checkpoint(oracle_entries(ds), device=DEV, epoch=2))
     ctx.restore(img, DEV)
     ctx.restore(img, DEV)  # the first restore's allocation is released / reused
+    ctx.trim()             # spares and pooled pinned buffers released
+    ctx.restore(img, DEV)
     for h, b in zip(ds.handles, ds.host):
         assert np.array_equal(bound_bytes(ctx, h), b)
     release_all(ctx, ds)
