@@ -4,13 +4,16 @@
 //     ... into one contiguous checkpoint image carrying a per-64 KiB CRC32C")
 //  K2 verify_scatter   (restart step 3, L16 §III-C; north_star "every chunk is
 //     CRC-verified, and its bytes are scattered into freshly re-created buffers")
-//  K6 debug fill / compare (test tooling: synth/ generator on the device)
+//  f1 incremental: CRC-only pass, present-set scan + compaction, gather / scatter
+//  plan expansion (a2 / r2), lookup-table builder, K6 debug fill / compare
 //
-// Both K1 and K2 are one template (snapshot_kernel<kOp>): a persistent grid,
-// one warp per chunk (<= 64 KiB) of a flat chunk list. A chunk is moved in rounds
-// of 4 KiB of contiguous bytes: eight coalesced 16-byte global loads per lane
-// (each warp instruction = 512 contiguous bytes), a coalesced 16-byte store of the
-// same registers to the destination, and a transposition through a padded
+// K1, K2 and the incremental passes are one data path templated on the op
+// (kOp* in checl_internal.h) in three work splits: balanced_kernel (default: equal
+// contiguous stretches of 4 KiB rounds per warp), snapshot_kernel (one warp per
+// chunk, grid-stride) and sweep_kernel (4 KiB units, grid-stride). A chunk is moved
+// in rounds of 4 KiB of contiguous bytes: eight coalesced 16-byte global loads per
+// lane (each warp instruction = 512 contiguous bytes), a coalesced 16-byte store of
+// the same registers to the destination, and a transposition through a padded
 // 32 x 144 B shared tile so that lane l then reads "its" 128-byte segment (segment
 // 32r + l of the chunk) with conflict-free 16-byte shared loads. Each lane runs a
 // slicing-by-4 CRC over its segments, carrying its register from round to round
