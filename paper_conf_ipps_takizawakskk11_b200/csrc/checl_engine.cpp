@@ -138,6 +138,27 @@ double now_ms() {
   return std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now().time_since_epoch()).count();
 }
 
+// CHECL_TRACE=1: host timestamps of an op's phases on stderr (diagnostics only).
+struct Trace {
+  bool on;
+  double t0, last;
+  std::string line;
+  explicit Trace(const char* op) : on(std::getenv("CHECL_TRACE") != nullptr), t0(now_ms()), last(t0) {
+    if (on) line = op;
+  }
+  void operator()(const char* what) {
+    if (!on) return;
+    const double t = now_ms();
+    char buf[64];
+    std::snprintf(buf, sizeof buf, " %s=%.1f", what, (t - last) * 1e3);
+    line += buf;
+    last = t;
+  }
+  ~Trace() {
+    if (on) std::fprintf(stderr, "[checl] %s total=%.1f us\n", line.c_str(), (now_ms() - t0) * 1e3);
+  }
+};
+
 uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 uint64_t chunks_of(uint64_t size) { return (size + kChunkBytes - 1) / kChunkBytes; }
 
@@ -900,21 +921,25 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
                            bool to_device) {
   (void)stream;
   const double t0 = now_ms();
+  Trace tr("checkpoint");
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
   const uint64_t aux0 = ds.aux_launches;
   ds.events.reset();
   KernelTimer kt;
   checl_timing tm{};
+  tr("setup");
 
   // a1: synchronise the host and every queue of the device (L16 step 1)
   const double ts = now_ms();
   ck(cudaDeviceSynchronize());
   tm.sync_ms = now_ms() - ts;
+  tr("sync");
 
   // a2: database walk -> manifest + chunk list (L19), cached per registry version
   const double tp = now_ms();
   Plan& P = get_plan(ctx, ds, device);
+  tr("plan");
   LaunchParams lp = base_params(ds);
   lp.desc = P.d_desc.p;
   lp.round_base = P.d_round.p;
@@ -957,13 +982,16 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       mirror = nullptr;
     }
     lp.crc_mirror = static_cast<uint32_t*>(mirror);
+    tr("mirror");
     if (P.n_chunks) timed_launch(ds, kt, kOpPack, lp, ds.compute);
+    tr("launch");
     ck(cudaEventRecord(c_begin, ds.compute));
     if (P.n_chunks && !mirror)
       ck(cudaMemcpyAsync(img->host_mut + P.crc_off, img->d_crc, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.compute));
     ck(cudaEventRecord(c_end, ds.compute));
     tm.n_stages = 1;
     ck(cudaStreamSynchronize(ds.compute));
+    tr("wait");
   } else {
     // a3 + a4: pack stage s into slot s % n_slots on the compute stream while the
     // copy engine drains the previous slot to the pinned image
@@ -1008,6 +1036,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
   const double tf = now_ms();
   finalize_meta(img->host_mut, P, epoch);
   tm.commit_ms = now_ms() - tf;
+  tr("finalize");
   img->image_bytes = P.image_bytes;
   img->payload_off = P.payload_off;
   float cms = 0;
