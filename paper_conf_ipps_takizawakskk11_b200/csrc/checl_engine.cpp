@@ -1216,6 +1216,7 @@ void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, uint8
 checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void* stream, checl_report* rep,
                         bool in_migrate) {
   const double t0 = now_ms();
+  Trace tr("restore");
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
   const uint64_t aux0 = ds.aux_launches;
@@ -1228,6 +1229,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   const double ts = now_ms();
   ck(cudaDeviceSynchronize());
   tm.sync_ms = now_ms() - ts;
+  tr("sync");
 
   // r1: validate header + manifest (+ meta CRC over the CRC table)
   const double tp = now_ms();
@@ -1237,12 +1239,14 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   if (st) return st;
   if (P.flags != 0) return CHECL_ERR_BAD_IMAGE;  // a delta restores only as part of a chain
   if (rep) set_report(rep, P, 0, 0);
+  tr("parse");
 
   // r2: re-create the buffers: one allocation laid out like the payload
   const double ta = now_ms();
   auto arena = new_arena(ctx, device, stream, P.L.payload_bytes);
   if (!arena) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
   tm.alloc_ms = now_ms() - ta;
+  tr("alloc");
   const uint64_t nch = P.L.n_chunks;
   ds.h_recs.ensure(std::max<size_t>(P.bufs.size(), 1));
   uint8_t* abase = static_cast<uint8_t*>(arena->base);
@@ -1264,6 +1268,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     ck(launch_expand(ds.recs_scratch.p, (uint32_t)P.bufs.size(), P.L.payload_bytes, nch, ds.desc_scratch.p,
                      ds.round_scratch.p, rounds, ds.status.p, ds.n_sms, ds.compute));
   }
+  tr("expand");
   DevBuf<uint8_t> tmp_payload;  // only when the source device is not peer-reachable
   DevBuf<uint32_t> tmp_crc;
   if (dev_img) {
@@ -1292,6 +1297,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     lp.crc = const_cast<uint32_t*>(crc);
     if (nch) timed_launch(ds, kt, kOpVerify, lp, ds.compute);
     tm.n_stages = 1;
+    tr("launch");
   } else {
     // r3 + r4: fill slot s % n_slots over PCIe while the previous slot is verified
     ck(cudaEventRecord(c_begin, ds.copy));
@@ -1332,6 +1338,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   }
   ck(cudaStreamSynchronize(ds.compute));
   ck(cudaStreamSynchronize(ds.copy));
+  tr("wait");
   const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
   float cms = 0;
   if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
@@ -1347,8 +1354,11 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   // r5: rebind every handle (all-or-nothing)
   (void)in_migrate;
   const double tc = now_ms();
+  tr("events");
   commit(ctx, P, device, arena);
+  tr("commit");
   adopt_plan(ctx, ds, device, P, abase, rounds);
+  tr("adopt");
   tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
   ctx->last = tm;
