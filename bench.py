@@ -453,10 +453,10 @@ def main():
                 flush.fill_(i & 0xFF)
                 e0.record(cur)
             ctx.checkpoint(dev, epoch=i + 1, into=img)
-            tc = ctx.last_timing()
+            tc = ctx.last_timing(raw=True)
             coordinate(True, i + 1)
             ctx.restore(img, dev)
-            tr = ctx.last_timing()
+            tr = ctx.last_timing(raw=True)
             if collect is not None:
                 collect.append((tc, tr))
             if flush is not None:
@@ -477,6 +477,7 @@ def main():
     with ClockSampler(dev) as clk:
         ms = run(dimg, a.steps, phases)
     barrier()
+    phases = [(checl.timing_dict(c), checl.timing_dict(r)) for c, r in phases]
     ms_max = max_over_ranks(ms)
     value = sum_over_ranks(S * a.steps) / (ms_max * 1e-3) / 1e9
     # correctness of the last restore: every handle's new buffer == the application's bytes
@@ -516,6 +517,7 @@ def main():
         ph2 = []
         barrier()
         ms2 = run(himg, a.steps, ph2)
+        ph2 = [(checl.timing_dict(c), checl.timing_dict(r)) for c, r in ph2]
         barrier()
         ms2_max = max_over_ranks(ms2)
         E = sum_over_ranks(S * a.steps) / (ms2_max * 1e-3) / 1e9

@@ -433,10 +433,16 @@ class Context:
         """Release the spare allocations and pooled pinned buffers kept for reuse."""
         _check(lib.checl_trim(self._p), "checl_trim")
 
-    def last_timing(self) -> dict:
+    def last_timing(self, raw: bool = False):
+        """Phase times of the last checkpoint / restore (checl_timing); raw=True returns
+        the ctypes struct (cheap inside a timed loop; convert with timing_dict)."""
         t = _Timing()
         _check(lib.checl_last_timing(self._p, C.byref(t)), "checl_last_timing")
-        return {n: (float(getattr(t, n)) if ty is C.c_double else int(getattr(t, n))) for n, ty in _Timing._fields_}
+        return t if raw else timing_dict(t)
+
+
+def timing_dict(t) -> dict:
+    return {n: (float(getattr(t, n)) if ty is C.c_double else int(getattr(t, n))) for n, ty in _Timing._fields_}
 
 
 # -- test / bench tooling -----------------------------------------------------------

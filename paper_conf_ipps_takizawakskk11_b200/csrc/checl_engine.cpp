@@ -286,12 +286,12 @@ template <typename T>
 struct PinnedBuf {  // grow-only pinned host scratch
   T* p = nullptr;
   size_t cap = 0;
-  void ensure(size_t n) {
+  void ensure(size_t n, unsigned flags = cudaHostAllocDefault) {
     if (n <= cap) return;
     if (p) cudaFreeHost(p);
     p = nullptr;
     cap = 0;
-    ck(cudaHostAlloc(reinterpret_cast<void**>(&p), std::max<size_t>(n, 1) * sizeof(T), cudaHostAllocDefault));
+    ck(cudaHostAlloc(reinterpret_cast<void**>(&p), std::max<size_t>(n, 1) * sizeof(T), flags));
     cap = n;
   }
   void release() {
@@ -336,7 +336,15 @@ struct DevState {
   DevBuf<ChunkDesc> desc_scratch;
   DevBuf<uint32_t> round_scratch;
   DevBuf<BufferRecord> recs_scratch;
+  // what desc_scratch / round_scratch hold: the expansion of these records (valid
+  // iff scratch_payload != ~0); a restore whose records match skips its expansion
+  std::vector<BufferRecord> scratch_recs;
+  uint64_t scratch_payload = ~0ull;
+  // verify status {first bad, n bad, CTAs done}; between restores it rests at
+  // {~0, 0, 0} (reset by the publishing launch) unless status_clean is false
   DevBuf<unsigned long long> status;
+  bool status_clean = false;
+  unsigned long long* status_host_dev = nullptr;  // device address of h_status (mapped), or nullptr
   DevBuf<unsigned long long> unit_acc;
   // incremental checkpoint (f1): base CRC table, bitmap words, compacted chunk
   // list, [n_present, bytes], stage table
@@ -362,8 +370,18 @@ struct DevState {
     ck(snapshot_configure());
     inv_z.ensure(kRoundBytes);
     ck(cudaMemcpy(inv_z.p, inv_z_table().data(), kRoundBytes * 4, cudaMemcpyHostToDevice));
-    status.ensure(2);
-    h_status.ensure(2);
+    status.ensure(3);
+    h_status.ensure(2, cudaHostAllocMapped);
+    {
+      void* dp = nullptr;
+      if (cudaHostGetDevicePointer(&dp, h_status.p, 0) == cudaSuccess)
+        status_host_dev = static_cast<unsigned long long*>(dp);
+      else
+        cudaGetLastError();
+      const unsigned long long init[3] = {~0ull, 0ull, 0ull};
+      ck(cudaMemcpy(status.p, init, sizeof(init), cudaMemcpyHostToDevice));
+      status_clean = true;
+    }
     tables.ensure(kTableWords);
     ck(launch_build_tables(table_params(), tables.p, compute));
     ck(cudaStreamSynchronize(compute));
@@ -985,10 +1003,13 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
     tr("mirror");
     if (P.n_chunks) timed_launch(ds, kt, kOpPack, lp, ds.compute);
     tr("launch");
-    ck(cudaEventRecord(c_begin, ds.compute));
-    if (P.n_chunks && !mirror)
+    if (P.n_chunks && !mirror) {
+      ck(cudaEventRecord(c_begin, ds.compute));
       ck(cudaMemcpyAsync(img->host_mut + P.crc_off, img->d_crc, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.compute));
-    ck(cudaEventRecord(c_end, ds.compute));
+      ck(cudaEventRecord(c_end, ds.compute));
+    } else {
+      c_begin = c_end = nullptr;  // nothing copied
+    }
     tm.n_stages = 1;
     ck(cudaStreamSynchronize(ds.compute));
     tr("wait");
@@ -1040,7 +1061,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
   img->image_bytes = P.image_bytes;
   img->payload_off = P.payload_off;
   float cms = 0;
-  if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
+  if (c_begin && cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
   tm.kernel_ms = kt.sum_ms();
   tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tm.total_ms = now_ms() - t0;
@@ -1185,6 +1206,10 @@ void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, uint8
     if (kv.second.device == device) ++n_live;
   if (n_live != P.bufs.size() || !P.L.n_chunks) return;
   Plan& Q = ds.plan;
+  // the plan's current chunk list moves to the scratch buffers: so does its description
+  const bool q_valid = Q.version != ~0ull && Q.n_chunks && Q.recs.size() == Q.bufs.size();
+  ds.scratch_recs.swap(Q.recs);
+  ds.scratch_payload = q_valid ? Q.payload_bytes : ~0ull;
   Q.bufs = P.bufs;
   for (auto& b : Q.bufs) b.ptr = b.size ? abase + b.off : nullptr;
   Q.n_chunks = P.L.n_chunks;
@@ -1250,7 +1275,9 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   const uint64_t nch = P.L.n_chunks;
   ds.h_recs.ensure(std::max<size_t>(P.bufs.size(), 1));
   uint8_t* abase = static_cast<uint8_t*>(arena->base);
-  const uint64_t rounds = build_records(P.bufs, [&](size_t b) { return abase + P.bufs[b].off; }, ds.h_recs.p);
+  // (zero-size buffers get a null pointer, as in adopt_plan's records)
+  const uint64_t rounds = build_records(
+      P.bufs, [&](size_t b) { return P.bufs[b].size ? abase + P.bufs[b].off : nullptr; }, ds.h_recs.p);
   ds.desc_scratch.ensure(std::max<uint64_t>(nch, 1));
   ds.round_scratch.ensure(nch + 1);
   ds.recs_scratch.ensure(std::max<size_t>(P.bufs.size(), 1));
@@ -1260,14 +1287,29 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   tm.plan_ms = now_ms() - tp;
 
   cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
-  if (nch) {  // chunk list expanded on the GPU (compute stream, ahead of the verify launches);
-              // the same launch initialises the verify status
+  // the verify status is at rest unless an earlier restore stopped midway; the
+  // publishing launch below leaves it at rest again (status_clean set after the sync)
+  const bool was_clean = ds.status_clean, status_clean = was_clean && ds.status_host_dev;
+  ds.status_clean = false;
+  // the chunk list of the new allocation: already in the scratch buffers when the
+  // allocation and layout are those of an earlier restore (arenas alternate between
+  // the two allocations of consecutive restores: see adopt_plan), else expanded on
+  // the GPU (compute stream, ahead of the verify launches); the expansion also
+  // initialises the verify status
+  const bool have_list = status_clean && ds.scratch_payload == P.L.payload_bytes &&
+                         ds.scratch_recs.size() == P.bufs.size() &&
+                         std::memcmp(ds.scratch_recs.data(), ds.h_recs.p, P.bufs.size() * sizeof(BufferRecord)) == 0;
+  if (nch && !have_list) {
+    ds.scratch_payload = ~0ull;
     ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, P.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
     ++ds.aux_launches;
     ck(launch_expand(ds.recs_scratch.p, (uint32_t)P.bufs.size(), P.L.payload_bytes, nch, ds.desc_scratch.p,
                      ds.round_scratch.p, rounds, ds.status.p, ds.n_sms, ds.compute));
+    ds.scratch_recs.assign(ds.h_recs.p, ds.h_recs.p + P.bufs.size());
+    ds.scratch_payload = P.L.payload_bytes;
   }
+  lp.status_host = ds.status_host_dev;  // the last verify launch publishes (below)
   tr("expand");
   DevBuf<uint8_t> tmp_payload;  // only when the source device is not peer-reachable
   DevBuf<uint32_t> tmp_crc;
@@ -1287,8 +1329,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
       ck(cudaEventRecord(c_end, ds.copy));
       ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
     } else {  // nothing to copy: the kernel reads the image where it is
-      ck(cudaEventRecord(c_begin, ds.compute));
-      ck(cudaEventRecord(c_end, ds.compute));
+      c_begin = c_end = nullptr;
     }
     lp.c0 = 0;
     lp.c1 = nch;
@@ -1323,25 +1364,28 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
       lp.c1 = S.c1;
       lp.image = ds.slot(k);
       lp.image_base = S.img_lo;
-      timed_launch(ds, kt, kOpVerify, lp, ds.compute);
+      LaunchParams ls = lp;
+      if (s + 1 != stages.size()) ls.status_host = nullptr;  // only the last launch publishes
+      timed_launch(ds, kt, kOpVerify, ls, ds.compute);
       ck(cudaEventRecord(verified[k], ds.compute));
     }
     ck(cudaEventRecord(c_end, ds.copy));
     if (stages.empty()) ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
     tm.n_stages = stages.size();
   }
-  if (nch) {
+  if (nch && !lp.status_host) {
     ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
-  } else {
+  } else if (!nch) {
     ds.h_status.p[0] = ~0ull;
     ds.h_status.p[1] = 0;
   }
   ck(cudaStreamSynchronize(ds.compute));
   ck(cudaStreamSynchronize(ds.copy));
   tr("wait");
+  ds.status_clean = nch ? lp.status_host != nullptr : was_clean;
   const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
   float cms = 0;
-  if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
+  if (c_begin && cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
   tm.kernel_ms = kt.sum_ms();
   tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tmp_payload.release();
@@ -1602,6 +1646,8 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
     }
     if (open) dst.push_back(cur);
   }
+  ds.scratch_payload = ~0ull;  // the scratch list is overwritten (no longer described)
+  ds.status_clean = false;
   ds.desc_scratch.ensure(std::max<uint64_t>(std::max<uint64_t>(nch, hdesc.size()), 1));
   ds.cdesc.ensure(std::max<size_t>(hdesc.size(), 1));
   ds.crc_scratch.ensure(std::max<uint64_t>(nch, 1));
@@ -1666,14 +1712,16 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   lp.image = nullptr;
   lp.image_base = 0;
   if (nch) {
+    lp.status_host = ds.status_host_dev;
     timed_launch(ds, kt, kOpCheck, lp, ds.compute);
-    ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
+    if (!lp.status_host) ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
   } else {
     ds.h_status.p[0] = ~0ull;
     ds.h_status.p[1] = 0;
   }
   ck(cudaStreamSynchronize(ds.compute));
   ck(cudaStreamSynchronize(ds.copy));
+  ds.status_clean = nch && lp.status_host;
   const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
   float cms = 0;
   if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;

@@ -156,7 +156,12 @@ struct LaunchParams {
   const uint32_t* tables;   // kTableWords words (build_tables)
   const uint32_t* round_base;  // per chunk: global index of its round 0 (+ one past the end);
                                // nullptr: the launch runs the grid-stride kernels
-  unsigned long long* status;  // verify/check: [0] = first bad chunk (atomicMin), [1] = bad count
+  unsigned long long* status;  // verify/check: [0] = first bad chunk (atomicMin), [1] = bad count,
+                               // [2] = CTAs finished (publishing launches)
+  // verify/check: the launch that closes a restore copies status[0..1] here (mapped
+  // pinned host memory) from its last CTA and resets status to {~0, 0, 0}; nullptr:
+  // status is left as accumulated
+  unsigned long long* status_host;
   // sweep kernel (one 4 KiB unit per warp-iteration)
   unsigned long long* unit_acc;  // per chunk: low 32 = XOR of unit terms, high = finished-unit mask (zeroed)
 };

@@ -277,6 +277,29 @@ __device__ __forceinline__ void finish_chunk(const LaunchParams& p, uint64_t c, 
   }
 }
 
+// End of a publishing verify/check launch (p.status_host set): the last CTA to
+// finish copies the status words to the pinned host mirror and resets them to
+// {~0, 0, 0}, so the host reads the result without a D2H copy and the next restore
+// needs no initialisation launch. (Each CTA's atomics are ordered before its
+// arrival by __threadfence; the last arrival then sees every CTA's updates.)
+template <int kOp>
+__device__ __forceinline__ void publish_status(const LaunchParams& p) {
+  if (!OpT<kOp>::kCompare || !p.status_host) return;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(&p.status[2], 1ull) == gridDim.x - 1) {
+      __threadfence();
+      const unsigned long long first = atomicExch(&p.status[0], ~0ull);
+      const unsigned long long n_bad = atomicExch(&p.status[1], 0ull);
+      atomicExch(&p.status[2], 0ull);
+      volatile unsigned long long* h = p.status_host;
+      h[0] = first;
+      h[1] = n_bad;
+    }
+  }
+}
+
 template <int kOp>
 __device__ __forceinline__ void chunk_ptrs(const LaunchParams& p, const ChunkDesc& d, const uint8_t*& src,
                                            uint8_t*& dst, int& mode) {
@@ -364,6 +387,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     }
     finish_chunk<kOp>(p, c, src, dst, len, pad, nrounds, f, lane);
   }
+  publish_status<kOp>(p);
 }
 
 // ---- balanced kernel: an equal contiguous stretch of rounds per warp ---------
@@ -500,6 +524,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
   }
   // a warp without rounds still waits: the CTA must not exit under the table copy
   if (!tables_ready) wait_tables(reinterpret_cast<uint64_t*>(smem + kBalMbarOff));
+  publish_status<kOp>(p);
 }
 
 // ---- sweep kernel: one 4 KiB unit per warp-iteration ------------------------
@@ -616,6 +641,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) sweep_kernel(const LaunchPa
     __syncwarp();
     cur = nxt;
   }
+  publish_status<kOp>(p);
 }
 
 // ---- lookup tables: built once per device (DevState::init) -------------------
@@ -736,7 +762,7 @@ __global__ void expand_plan_kernel(const BufferRecord* __restrict__ recs, uint32
                                    uint64_t total_rounds, unsigned long long* __restrict__ status) {
   if (blockIdx.x == 0 && threadIdx.x == 0) {
     if (round_base) round_base[n_chunks] = (uint32_t)total_rounds;
-    if (status) status[0] = ~0ull, status[1] = 0ull;  // the verify status of the launches that follow
+    if (status) status[0] = ~0ull, status[1] = 0ull, status[2] = 0ull;  // the verify status of the launches that follow
   }
   for (uint64_t c = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; c < n_chunks;
        c += (uint64_t)gridDim.x * blockDim.x) {

@@ -330,3 +330,40 @@ def test_c3_handle_stress_full_size_sampled(ctx):
         ptr, nb, _ = ctx.translate(h)
         nd += checl.debug_compare(DEV, ptr, v.data_ptr(), nb)
     assert nd == 0
+
+
+def test_repeated_device_restores_reuse_chunk_list_and_status(ctx):
+    """The bench loop (checkpoint_into a device image -> restore, repeated): restores
+    alternate between two allocations and skip the chunk-list expansion once the
+    scratch list matches; the verify status is published by the last CTA and left at
+    rest, also after a failing restore (DESIGN.md §5 "Restore launches")."""
+    sizes = [1 << 20, 70001, 0, 3 * 65536 + 5, 4097]
+    ds = make_set(ctx, sizes, seed=21, offsets=[0, 4, 0, 1, 0])
+    dimg = ctx.checkpoint_device(DEV, epoch=1)
+    kernels = []
+    for i in range(6):
+        ctx.checkpoint(DEV, epoch=i + 2, into=dimg)
+        ctx.restore(dimg, DEV)
+        kernels.append(ctx.last_timing()["n_kernels"])
+        for h, b in zip(ds.handles, ds.host):
+            assert np.array_equal(bound_bytes(ctx, h), b), (i, h)
+    assert kernels[-1] == 1 and kernels[-2] == 1, kernels  # verify only, no expansion
+    host = dimg.to_host().view().copy()
+    poff = struct.unpack_from("<Q", host.tobytes(), 56)[0]
+    bad = poff + 65536 * 16 + 256 + 3  # second buffer (offset 1 MiB), chunk 0 -> global chunk 16
+    for rep in range(2):
+        dimg.corrupt(bad, 0x01)
+        with pytest.raises(checl.CheclError) as ei:
+            ctx.restore(dimg, DEV)
+        r = ei.value.report
+        assert (r.n_bad_chunks, r.first_bad_chunk, r.first_bad_handle) == (1, 16, ds.handles[1]), rep
+        dimg.corrupt(bad, 0x01)  # undo: the next restore must not see stale status
+        ctx.restore(dimg, DEV)
+        for h, b in zip(ds.handles, ds.host):
+            assert np.array_equal(bound_bytes(ctx, h), b), (rep, h)
+    # a host image and a device image alternating share the status words
+    himg = ctx.checkpoint(DEV, epoch=9)
+    for i in range(3):
+        ctx.restore(himg if i % 2 else dimg, DEV)
+        for h, b in zip(ds.handles, ds.host):
+            assert np.array_equal(bound_bytes(ctx, h), b), (i, h)

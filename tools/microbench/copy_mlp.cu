@@ -2,6 +2,7 @@
 // lane, one CTA per SM (large dynamic smem forces it). Not part of the library.
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 template <int U>
@@ -41,10 +42,10 @@ void run(int warps, int sms, const uint4* a, uint4* b, size_t n16, size_t smem) 
          2.0 * n16 * 16 * 5 / (ms * 1e-3) / 1e9);
 }
 
-int main() {
+int main(int argc, char** argv) {
   int sms;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
-  const size_t bytes = 1ull << 30, n16 = bytes / 16;
+  const size_t bytes = argc > 1 ? (size_t)atoll(argv[1]) : (1ull << 30), n16 = bytes / 16;
   uint4 *a, *b;
   cudaMalloc(&a, bytes);
   cudaMalloc(&b, bytes);

@@ -4,6 +4,7 @@
 // usage: tma_copy  (sweeps W warps/CTA, T tile bytes, NT tiles)
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <cuda_runtime.h>
 
 __device__ __forceinline__ uint32_t sa(const void* p) { return (uint32_t)__cvta_generic_to_shared(p); }
@@ -76,10 +77,10 @@ void run(const uint8_t* s, uint8_t* d, size_t n, int W, int T, int sms) {
          cudaGetErrorString(cudaGetLastError()));
 }
 
-int main() {
+int main(int argc, char** argv) {
   int sms;
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0);
-  const size_t n = 1ull << 31;
+  const size_t n = argc > 1 ? (size_t)atoll(argv[1]) : (1ull << 31);
   uint8_t *s, *d;
   cudaMalloc(&s, n);
   cudaMalloc(&d, n);
