@@ -165,6 +165,27 @@ for bad in (raw[:-1], raw[:100], raw[:40] + bytes([raw[40] ^ 1]) + raw[41:]):
         raise SystemExit("damaged image accepted")
     except checl.CheclError as e:
         assert e.status == checl.ERR_BAD_IMAGE, e
+# host meta CRC (3 interleaved crc32 streams over 3 KiB blocks + a tail) on metadata
+# of 0.2-60 KB: every oracle image is accepted, a flipped metadata bit is refused
+for nb in (1, 20, 63, 64, 65, 200, 1000):
+    ents = [O.Entry(i + 1, rng.integers(0, 256, int(rng.integers(0, 3 * 65536)), dtype=np.uint8)) for i in range(nb)]
+    arr = O.checkpoint(ents, device=0, epoch=nb)
+    q = os.path.join(tmp, "meta.checl")
+    w = checl.Image.wrap(arr)
+    w.write(q)
+    back = checl.Image.read(q)
+    assert np.array_equal(back.view(), arr)
+    back.free(); w.free()
+    poff = struct.unpack_from("<Q", arr.tobytes(), 56)[0]
+    for pos in (130, poff // 2, poff - 1 if nb == 1 else int(poff) - 8):
+        bad = arr.copy()
+        bad[pos] ^= 0x20
+        open(q, "wb").write(bad.tobytes())
+        try:
+            checl.Image.read(q)
+            raise SystemExit(f"metadata flip at {pos} accepted (nb={nb})")
+        except checl.CheclError as e:
+            assert e.status == checl.ERR_BAD_IMAGE, e
 print("ok")
 """
 
