@@ -14,9 +14,11 @@ from ncu_summary import summary  # noqa: E402
 
 src, dst = sys.argv[1], sys.argv[2]
 os.makedirs(dst, exist_ok=True)
-for f in ("bench.json", "bench_c1.json", "bench_c3.json", "pytest_gpu.log", "smoke.log", "nvsmi.txt"):
-    if os.path.exists(os.path.join(src, f)):
-        shutil.copy(os.path.join(src, f), os.path.join(dst, f))
+import glob  # noqa: E402
+for f in sorted(glob.glob(os.path.join(src, "bench*.json"))) + [
+        os.path.join(src, f) for f in ("pytest_gpu.log", "smoke.log", "nvsmi.txt", "trace.log", "sanitizer.txt")]:
+    if os.path.exists(f):
+        shutil.copy(f, os.path.join(dst, os.path.basename(f)))
 lines = []
 lc = os.path.join(src, "launches.csv")
 if os.path.exists(lc):
