@@ -241,6 +241,12 @@ TableParams table_params() {
   tp.horner = gf_x8n(kRoundBytes - kSegBytes);
   for (int l = 0; l < 32; ++l) tp.lanepow[l] = gf_x8n((uint64_t)kSegBytes * (31 - l));
   for (int k = 0; k < 16; ++k) tp.unitpow[k] = gf_x8n((uint64_t)kRoundBytes * k);
+  tp.col_shift = gf_x8n(kSegBytes);
+  for (int k = 0; k < kFoldLevels; ++k) {
+    uint32_t r = kOne;
+    for (int i = 0; i < 32 << k; ++i) r = gf_divx(r);  // x^(-32 * 2^k)
+    tp.col_fold[k] = r;
+  }
   return tp;
 }
 
@@ -346,6 +352,8 @@ struct DevState {
   bool status_clean = false;
   unsigned long long* status_host_dev = nullptr;  // device address of h_status (mapped), or nullptr
   DevBuf<unsigned long long> unit_acc;
+  DevBuf<unsigned long long> warp_trace;  // CHECL_WARP_TRACE diagnostics
+  DevBuf<unsigned long long> work;        // dynamic-block counter + finished CTAs (zero at rest)
   // incremental checkpoint (f1): base CRC table, bitmap words, compacted chunk
   // list, [n_present, bytes], stage table
   DevBuf<uint32_t> base_crc, map_words;
@@ -353,7 +361,9 @@ struct DevState {
   DevBuf<unsigned long long> dtotals, stage_first, stage_lo;
   PinnedBuf<unsigned long long> h_dtab;
   // 1 = warp per chunk (throughput), 2 = 4 KiB units swept by the grid (latency of
-  // small launches); 0 = by size; env CHECL_KERNEL=1|2 forces one
+  // small launches), 3 = balanced stretches of rounds, 4 = balanced stretches with
+  // bulk (TMA) copies and the column CRC; 0 = by plan; env
+  // CHECL_KERNEL=1..4 forces one
   int kernel = 0;
   uint64_t aux_launches = 0;  // plan expansion / delta scan kernels (checl_timing.n_kernels)
   PinnedBuf<unsigned long long> h_status;
@@ -370,6 +380,8 @@ struct DevState {
     ck(snapshot_configure());
     inv_z.ensure(kRoundBytes);
     ck(cudaMemcpy(inv_z.p, inv_z_table().data(), kRoundBytes * 4, cudaMemcpyHostToDevice));
+    work.ensure(2);
+    ck(cudaMemset(work.p, 0, 2 * sizeof(unsigned long long)));
     status.ensure(3);
     h_status.ensure(2, cudaHostAllocMapped);
     {
@@ -385,7 +397,7 @@ struct DevState {
     tables.ensure(kTableWords);
     ck(launch_build_tables(table_params(), tables.p, compute));
     ck(cudaStreamSynchronize(compute));
-    if (const char* k = std::getenv("CHECL_KERNEL")) kernel = std::atoi(k) >= 1 && std::atoi(k) <= 3 ? std::atoi(k) : 0;
+    if (const char* k = std::getenv("CHECL_KERNEL")) kernel = std::atoi(k) >= 1 && std::atoi(k) <= 4 ? std::atoi(k) : 0;
   }
   void ensure_slots(size_t bytes, uint32_t n) {
     if (slot_bytes == bytes && n_slots == n && slots.p) return;
@@ -411,6 +423,8 @@ struct DevState {
     plan.d_recs.release();
     status.release();
     unit_acc.release();
+    warp_trace.release();
+    work.release();
     tables.release();
     base_crc.release();
     map_words.release();
@@ -904,14 +918,40 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
   }();
   if (op == kOpPack && (exp_pack_op == kOpCrc || exp_pack_op == kOpCopy)) op = exp_pack_op;
   const uint64_t chunks = p.c1 - p.c0;
-  // kernel 3 (balanced stretches of rounds) whenever the chunk list has a
-  // round_base; otherwise a warp needs ~55 us per 64 KiB chunk in kernel 1, and when
-  // chunks are fewer than half the warps the 4 KiB-unit sweep finishes sooner
+  // kernel 4 (bulk copies, column CRC; scheduled stretches of rounds) whenever the
+  // chunk list has a round_base (kernel 3 for the ops kernel 4 does not implement);
+  // otherwise a warp needs ~55 us per 64 KiB chunk in kernel 1, and when chunks are
+  // fewer than half the warps the 4 KiB-unit sweep finishes sooner
   int kernel = ds.kernel;
-  if (kernel == 3 && !p.round_base) kernel = 0;
+  if (kernel == 4 && op != kOpPack && op != kOpVerify && op != kOpCrc && op != kOpCheck) kernel = 3;
+  if (kernel >= 3 && !p.round_base) kernel = 0;
   const bool small = chunks * 2 <= (uint64_t)ds.n_sms * kWarpsPerCta;
-  if (!kernel) kernel = p.round_base ? 3 : (small ? 2 : 1);
-  if (kernel != 3) p.round_base = nullptr;
+  if (!kernel)
+    kernel = p.round_base ? ((op == kOpPack || op == kOpVerify || op == kOpCrc || op == kOpCheck) ? 4 : 3)
+                          : (small ? 2 : 1);
+  if (kernel < 3) p.round_base = nullptr;
+  // balanced / TMA launches large enough to have a tail: static stretches for the
+  // first part of the rounds, dynamic blocks for the rest (DESIGN.md §5 "Work split");
+  // CHECL_STATIC_PERMILLE / CHECL_DYN_BLOCK override the defaults (experiments)
+  static const uint32_t static_pm = [] {
+    const char* e = std::getenv("CHECL_STATIC_PERMILLE");
+    return e ? (uint32_t)std::min(1000, std::max(0, std::atoi(e))) : 750u;
+  }();
+  static const uint32_t dyn_block = [] {
+    const char* e = std::getenv("CHECL_DYN_BLOCK");
+    return e ? (uint32_t)std::max(1, std::atoi(e)) : 8u;
+  }();
+  // (kernel 3 keeps static stretches only: measured slower with the dynamic tail)
+  static const uint64_t dyn_min = [] {
+    const char* e = std::getenv("CHECL_DYN_MIN_ROUNDS");
+    return e ? (uint64_t)std::strtoull(e, nullptr, 10) : ~0ull;
+  }();
+  const uint64_t min_rounds = dyn_min != ~0ull ? dyn_min : (uint64_t)ds.n_sms * kWarpsPerCta * 8;
+  if (kernel == 4 && static_pm < 1000 && chunks * (kChunkBytes / kRoundBytes) >= min_rounds) {
+    p.work = ds.work.p;
+    p.static_permille = static_pm;
+    p.dyn_block = dyn_block;
+  }
   if (kernel >= 2) {
     if (ds.unit_acc.cap < chunks) {  // zeroed once; every sweep launch leaves it zero
       ds.unit_acc.ensure(chunks);
@@ -919,11 +959,59 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
     }
     p.unit_acc = ds.unit_acc.p;
   }
+  // diagnostics: CHECL_WARP_TRACE=1 prints the warps' start / tables-ready / end
+  // times of every balanced or TMA launch (relative to the earliest start, us)
+  static const bool warp_tr = std::getenv("CHECL_WARP_TRACE") != nullptr;
+  const uint64_t n_tr = (uint64_t)ds.n_sms * kWarpsPerCta * 4;
+  if (warp_tr && kernel >= 3) {
+    ds.warp_trace.ensure(n_tr);
+    ck(cudaMemsetAsync(ds.warp_trace.p, 0, n_tr * 8, s));
+    p.warp_trace = ds.warp_trace.p;
+  }
   cudaEvent_t a = ds.events.get(), b = ds.events.get();
   ck(cudaEventRecord(a, s));
   ck(launch_snapshot(op, p, ds.n_sms, s, kernel, chunks * (kChunkBytes / kRoundBytes)));
   ck(cudaEventRecord(b, s));
   kt.spans.push_back({a, b});
+  if (p.warp_trace) {
+    std::vector<unsigned long long> h(n_tr);
+    ck(cudaMemcpyAsync(h.data(), p.warp_trace, n_tr * 8, cudaMemcpyDeviceToHost, s));
+    ck(cudaStreamSynchronize(s));
+    std::vector<double> st, tb, en;
+    unsigned long long t0 = ~0ull;
+    for (uint64_t w = 0; w < n_tr / 4; ++w)
+      if (h[4 * w]) t0 = std::min(t0, h[4 * w]);
+    for (uint64_t w = 0; w < n_tr / 4; ++w) {
+      if (!h[4 * w]) continue;
+      st.push_back((h[4 * w] - t0) * 1e-3);
+      if (h[4 * w + 1]) tb.push_back((h[4 * w + 1] - t0) * 1e-3);
+      en.push_back((h[4 * w + 2] - t0) * 1e-3);
+    }
+    auto q = [](std::vector<double>& v, double f) {
+      if (v.empty()) return 0.0;
+      std::sort(v.begin(), v.end());
+      return v[(size_t)(f * (v.size() - 1))];
+    };
+    float ms = 0;
+    cudaEventElapsedTime(&ms, a, b);
+    std::fprintf(stderr,
+                 "[checl] op %d kernel %d warps %zu event %.1f us | start p50 %.1f max %.1f | tables p50 %.1f max %.1f | "
+                 "end min %.1f p10 %.1f p50 %.1f p90 %.1f max %.1f us\n",
+                 op, kernel, st.size(), ms * 1e3, q(st, 0.5), q(st, 1.0), q(tb, 0.5), q(tb, 1.0), q(en, 0.0), q(en, 0.1),
+                 q(en, 0.5), q(en, 0.9), q(en, 1.0));
+    if (std::atoi(std::getenv("CHECL_WARP_TRACE")) == 2) {  // raw end times, one line per CTA
+      for (int c = 0; c < ds.n_sms; ++c) {
+        std::string line = "[checl] cta " + std::to_string(c) + " sm " + std::to_string(h[4 * (uint64_t)c * kWarpsPerCta + 3]);
+        for (int w = 0; w < kWarpsPerCta; ++w) {
+          const uint64_t i = (uint64_t)c * kWarpsPerCta + w;
+          char buf[32];
+          std::snprintf(buf, sizeof buf, " %.1f", h[4 * i] ? (h[4 * i + 2] - t0) * 1e-3 : -1.0);
+          line += buf;
+        }
+        std::fprintf(stderr, "%s\n", line.c_str());
+      }
+    }
+  }
 }
 
 // Writes header + manifest + meta_crc into the image's host bytes [0, payload_off);
@@ -1330,6 +1418,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
       ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
     } else {  // nothing to copy: the kernel reads the image where it is
       c_begin = c_end = nullptr;
+      lp.image_remote = img->device != device;
     }
     lp.c0 = 0;
     lp.c1 = nch;

@@ -127,12 +127,19 @@ constexpr int kHornerWords = 8 * 16 * 32;       // x^(8*3968) nibble tables, 16 
 constexpr int kFoldWords = kFoldLevels * 8 * 16; // fold nibble tables, 2.5 KiB
 constexpr int kPosWords = 8 * 16 * 32;          // sweep: lane-position nibble tables, 16 KiB
 constexpr int kUnitWords = 16 * 32;             // sweep: x^(8*4096*k) * x^i, 2 KiB
+// TMA kernel (column CRC): lane l chains word l of every 128-byte row,
+// so its step is v -> v * x^(8*128) (slicing-by-4 tables of that shift, same
+// lane-private layout), and the lanes are combined with shifts x^(-32*2^k).
+constexpr int kColWords = 4 * 256 * 32;          // 128 KiB
+constexpr int kColFoldWords = kFoldLevels * 8 * 16;  // 2.5 KiB
 constexpr int kTabOff = 0;
 constexpr int kHornerOff = kTabOff + kTabWords;
 constexpr int kFoldOff = kHornerOff + kHornerWords;
 constexpr int kPosOff = kFoldOff + kFoldWords;
 constexpr int kUnitOff = kPosOff + kPosWords;
-constexpr int kTableWords = kUnitOff + kUnitWords;
+constexpr int kColOff = kUnitOff + kUnitWords;
+constexpr int kColFoldOff = kColOff + kColWords;
+constexpr int kTableWords = kColFoldOff + kColFoldWords;
 static_assert((kPosOff * 4) % 16 == 0 && (kFoldOff * 4 + kFoldWords * 4) % 16 == 0, "bulk-copy alignment");
 
 // Constants the table builder needs (computed on the host).
@@ -141,6 +148,8 @@ struct TableParams {
   uint32_t horner;             // x^(8 * (kRoundBytes - kSegBytes)) mod P
   uint32_t lanepow[32];        // x^(8 * 128 * (31 - l)) mod P
   uint32_t unitpow[16];        // x^(8 * 4096 * k) mod P
+  uint32_t col_shift;          // x^(8 * 128) mod P
+  uint32_t col_fold[kFoldLevels];  // x^(-32 * 2^k) mod P
 };
 
 // Parameters of one launch over the chunk range [c0, c1) of `desc`. Payload byte
@@ -162,6 +171,16 @@ struct LaunchParams {
   // pinned host memory) from its last CTA and resets status to {~0, 0, 0}; nullptr:
   // status is left as accumulated
   unsigned long long* status_host;
+  // the image is a peer GPU's memory (NVLink): no bulk (TMA) loads from it
+  int image_remote;
+  // diagnostics (CHECL_WARP_TRACE): per warp {start, tables ready, end, smid}
+  unsigned long long* warp_trace;
+  // balanced / TMA kernels: the first static_permille/1000 of the rounds go to the
+  // warps in equal contiguous stretches, the rest in blocks of dyn_block rounds to
+  // whichever warp is free, from the counter work[0] (work[1] counts finished CTAs;
+  // the last one resets both: zero between launches). work == nullptr: all static.
+  unsigned long long* work;
+  uint32_t static_permille, dyn_block;
   // sweep kernel (one 4 KiB unit per warp-iteration)
   unsigned long long* unit_acc;  // per chunk: low 32 = XOR of unit terms, high = finished-unit mask (zeroed)
 };

@@ -300,6 +300,17 @@ __device__ __forceinline__ void publish_status(const LaunchParams& p) {
   }
 }
 
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// diagnostics: lane 0 of every warp records {start, tables ready, end}
+__device__ __forceinline__ void warp_trace(const LaunchParams& p, int k, unsigned long long t) {
+  if (p.warp_trace && (threadIdx.x & 31) == 0)
+    p.warp_trace[((uint64_t)blockIdx.x * kWarpsPerCta + (threadIdx.x >> 5)) * 4 + k] = t;
+}
+
 template <int kOp>
 __device__ __forceinline__ void chunk_ptrs(const LaunchParams& p, const ChunkDesc& d, const uint8_t*& src,
                                            uint8_t*& dst, int& mode) {
@@ -390,6 +401,68 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
   publish_status<kOp>(p);
 }
 
+// ---- work of the balanced and TMA kernels --------------------------------------
+// The rounds [R0, R0 + R) of the launch's chunks (round_base) are handed out in two
+// phases (guided self-scheduling): the first Rs rounds in equal contiguous stretches,
+// one per warp, then blocks of B rounds taken from a launch-wide counter by whichever
+// warp is free. Measured (CHECL_WARP_TRACE): with static stretches only, warps on the
+// 3-warp SM sub-partitions finish ~8 us after those on 2-warp ones, and bulk-copy
+// throughput differs by SM position by up to 25%; the dynamic tail absorbs both.
+struct Sched {
+  uint64_t R0, R, Rs, nblk;
+  uint32_t B;
+};
+
+__device__ __forceinline__ Sched make_sched(const LaunchParams& p) {
+  Sched s;
+  s.R0 = p.round_base[p.c0];
+  s.R = p.round_base[p.c1] - s.R0;
+  s.B = p.dyn_block ? p.dyn_block : 1u;
+  s.Rs = p.work ? s.R * p.static_permille / 1000u : s.R;
+  s.nblk = (s.R - s.Rs + s.B - 1) / s.B;
+  return s;
+}
+
+// The chunk holding round g: the last c in [c0, c1) with round_base[c] <= g, by a
+// 32-way search (one probe per lane: 3 dependent loads for C2, 4 for 1 M chunks).
+__device__ __forceinline__ uint64_t find_chunk(const LaunchParams& p, uint64_t g, int lane) {
+  uint64_t lo = p.c0, hi = p.c1;  // invariant: round_base[lo] <= g, answer in [lo, hi)
+  while (hi - lo > 1) {
+    const uint64_t step = (hi - lo + 31) / 32, idx = lo + lane * step;
+    const unsigned m = __ballot_sync(0xFFFFFFFFu, idx < hi && p.round_base[idx] <= g);
+    lo += (uint64_t)(31 - __clz(m)) * step;
+    hi = hi < lo + step ? hi : lo + step;
+  }
+  return lo;
+}
+
+// Next dynamic block [g, ge) and its first chunk; false when the counter ran out.
+__device__ __forceinline__ bool next_block(const LaunchParams& p, const Sched& s, int lane, uint64_t& g, uint64_t& ge,
+                                           uint64_t& c) {
+  if (!p.work) return false;
+  unsigned long long b = 0;
+  if (lane == 0) b = atomicAdd(&p.work[0], 1ull);
+  b = __shfl_sync(0xFFFFFFFFu, b, 0);
+  if (b >= s.nblk) return false;
+  g = s.R0 + s.Rs + b * s.B;
+  ge = g + s.B < s.R0 + s.R ? g + s.B : s.R0 + s.R;
+  c = find_chunk(p, g, lane);
+  return true;
+}
+
+// End of a scheduled launch: the last CTA resets the work counter for the next one.
+__device__ __forceinline__ void release_work(const LaunchParams& p) {
+  if (!p.work) return;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    if (atomicAdd(&p.work[1], 1ull) == gridDim.x - 1) {
+      atomicExch(&p.work[0], 0ull);
+      atomicExch(&p.work[1], 0ull);
+    }
+  }
+}
+
 // ---- balanced kernel: an equal contiguous stretch of rounds per warp ---------
 //
 // The rounds of the launch's chunks, enumerated in order (round_base), are split
@@ -415,6 +488,7 @@ template <int kOp>
 __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const LaunchParams p) {
   using O = OpT<kOp>;
   extern __shared__ __align__(128) uint8_t smem[];
+  const unsigned long long t_start = gtimer();
   if (O::kCrc) {
     const TableCopy cp[2] = {{0u, (uint32_t)kTabOff, (uint32_t)kSnapTabWords * 4u},
                              {(uint32_t)kBalUnitOff, (uint32_t)kUnitOff, (uint32_t)kUnitWords * 4u}};
@@ -435,18 +509,20 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
   uint8_t* tile_w = stage + s_lane * kRowPitch + g_lane * 16;
 
   const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta, wid = (uint64_t)blockIdx.x * kWarpsPerCta + warp;
-  const uint64_t R0 = p.round_base[p.c0], R = p.round_base[p.c1] - R0;
-  uint64_t g = R0 + R * wid / nw;
-  const uint64_t g_end = R0 + R * (wid + 1) / nw;
-  // the chunk holding round g: the last c in [c0, c1) with round_base[c] <= g, by a
-  // 32-way search (one probe per lane: 3 dependent loads for C2, 4 for 1 M chunks)
-  uint64_t lo = p.c0, hi = p.c1;  // invariant: round_base[lo] <= g, answer in [lo, hi)
-  while (hi - lo > 1) {
-    const uint64_t step = (hi - lo + 31) / 32, idx = lo + lane * step;
-    const unsigned m = __ballot_sync(full, idx < hi && p.round_base[idx] <= g);
-    lo += (uint64_t)(31 - __clz(m)) * step;
-    hi = hi < lo + step ? hi : lo + step;
-  }
+  const Sched sc = make_sched(p);
+  uint64_t g = sc.R0 + sc.Rs * wid / nw, g_end = sc.R0 + sc.Rs * (wid + 1) / nw;
+  uint64_t lo = g < g_end ? find_chunk(p, g, lane) : p.c0;
+  for (bool more = true; more;) {
+  // the next dynamic block is fetched (and its chunk found) while the first loads of
+  // this stretch are in flight
+  uint64_t ng = 0, nge = 0, nlo = 0;
+  bool fetched = false, nmore = false;
+  auto prefetch = [&]() {
+    if (!fetched) {
+      fetched = true;
+      nmore = next_block(p, sc, lane, ng, nge, nlo);
+    }
+  };
   for (uint64_t cur = lo; g < g_end; ++cur) {
     const uint64_t rb = p.round_base[cur];
     const ChunkDesc d = p.desc[cur];
@@ -493,7 +569,9 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
     if (!tables_ready) {  // the first loads are in flight; the tables have landed by now
       wait_tables(reinterpret_cast<uint64_t*>(smem + kBalMbarOff));
       tables_ready = true;
+      warp_trace(p, 1, gtimer());
     }
+    prefetch();
     for (int r = r0; r < r1; ++r) round(v, r);
 #endif
     uint32_t f = ch;
@@ -522,8 +600,233 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
       finish_chunk<kOp>(p, cur, src, dst, len, pad, nrounds, (uint32_t)now, lane);
     }
   }
+  prefetch();
+  more = nmore;
+  g = ng;
+  g_end = nge;
+  lo = nlo;
+  }
   // a warp without rounds still waits: the CTA must not exit under the table copy
   if (!tables_ready) wait_tables(reinterpret_cast<uint64_t*>(smem + kBalMbarOff));
+  release_work(p);
+  warp_trace(p, 0, t_start);
+  warp_trace(p, 2, gtimer());
+  {
+    unsigned smid;
+    asm("mov.u32 %0, %%smid;" : "=r"(smid));
+    warp_trace(p, 3, smid);
+  }
+  publish_status<kOp>(p);
+}
+
+// ---- TMA kernel: bulk copies through a contiguous tile, column CRC -----------
+//
+// Same work split as balanced_kernel (equal stretches of 4 KiB rounds per warp,
+// split chunks combined through the atomic accumulator), different data path: a
+// full round of a 16-byte-aligned source is moved global -> shared by one bulk
+// copy (cp.async.bulk, mbarrier completion) and shared -> global by one bulk store,
+// two tiles per warp (the next round's copy is in flight during this round's CRC);
+// the LSU carries only the CRC's shared loads. Partial, misaligned or remote rounds
+// take the register path (16-byte loads, stores from registers, exact tails) and
+// are written into the same tile. The tile is contiguous, so the CRC reads it by
+// columns: lane l chains word l of every 128-byte row (conflict-free LDS.32), a
+// chain of stride 128 B that runs across rounds unchanged:
+//   h <- (h ^ w) * x^(8*128)           (slicing-by-4 over tables of that shift)
+// With D = the part's bytes zero-padded to whole rounds, n = |D|, word i = l + 32k,
+//   R(D, s) = XOR_i R(w_i, 0) x^(8(n - 4i - 4)) = XOR_l h_l x^(-32 l),
+// (s folded into lane 0's first word), the lanes combined by a shuffle tree with
+// shifts x^(-32*2^k). The rest (zero-padding correction, split-chunk terms) is the
+// balanced kernel's.
+constexpr int kTmaTiles = 2;
+constexpr size_t kTmaColOff = 0;
+constexpr size_t kTmaFoldOff = (size_t)kColWords * 4;
+constexpr size_t kTmaUnitOff = kTmaFoldOff + (size_t)kColFoldWords * 4;
+constexpr size_t kTmaTileOff = (kTmaUnitOff + (size_t)kUnitWords * 4 + 127) / 128 * 128;
+constexpr size_t kTmaMbarOff = kTmaTileOff + (size_t)kWarpsPerCta * kTmaTiles * kRoundBytes;
+constexpr size_t kTmaSmemBytes = kTmaMbarOff + (size_t)(kWarpsPerCta * kTmaTiles + 1) * 8;
+static_assert(kTmaSmemBytes <= 232448, "fits the 227 KiB opt-in shared memory");
+static_assert(kColFoldOff == kColOff + kColWords, "column tables and their fold tables are contiguous");
+
+__device__ __forceinline__ void mbar_init(uint32_t mb) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint32_t mb, uint32_t parity) {
+  asm volatile(
+      "{\n .reg .pred p;\n TW_%=:\n"
+      " mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n"
+      " @!p bra TW_%=;\n}" ::"r"(mb),
+      "r"(parity)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_load(uint32_t dst, const void* src, uint32_t bytes, uint32_t mb) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(bytes) : "memory");
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(mb)
+               : "memory");
+}
+__device__ __forceinline__ void bulk_store(void* dst, uint32_t src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(dst), "r"(src), "r"(bytes)
+               : "memory");
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+}
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+
+template <int kOp>
+__global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchParams p) {
+  using O = OpT<kOp>;
+  extern __shared__ __align__(128) uint8_t smem[];
+  const unsigned long long t_start = gtimer();
+  uint64_t* mbars = reinterpret_cast<uint64_t*>(smem + kTmaMbarOff);  // [warp][tile], then the tables'
+  if (threadIdx.x == 0)
+    for (int i = 0; i < kWarpsPerCta * kTmaTiles; ++i) mbar_init(smem_addr(mbars + i));
+  {  // (load_tables fences the barrier initialisations and synchronises the CTA)
+    const TableCopy cp[2] = {{(uint32_t)kTmaColOff, (uint32_t)kColOff, (uint32_t)(kColWords + kColFoldWords) * 4u},
+                             {(uint32_t)kTmaUnitOff, (uint32_t)kUnitOff, (uint32_t)kUnitWords * 4u}};
+    load_tables<2, false>(smem, p.tables, cp, mbars + kWarpsPerCta * kTmaTiles);
+  }
+  bool tables_ready = false;
+  const uint8_t* tb = smem + kTmaColOff;
+  const uint32_t* ftab = reinterpret_cast<const uint32_t*>(smem + kTmaFoldOff);
+  const uint32_t* utab = reinterpret_cast<const uint32_t*>(smem + kTmaUnitOff);
+
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint8_t* tiles = smem + kTmaTileOff + (size_t)warp * kTmaTiles * kRoundBytes;
+  const uint32_t tile_sa = smem_addr(tiles), mb_sa = smem_addr(mbars + warp * kTmaTiles);
+  uint32_t phase = 0;  // bit t: parity of tile t's next completion
+  const uint32_t l4 = (uint32_t)lane * 4u;
+  const unsigned full = 0xFFFFFFFFu;
+  // register path: instruction i of a round = 512 contiguous bytes; lane l moves
+  // the 16 bytes at lane_off + 512 i (the same offset in the contiguous tile)
+  const uint32_t lane_off = (uint32_t)(lane >> 3) * kSegBytes + (uint32_t)(lane & 7) * 16;
+
+  const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta, wid = (uint64_t)blockIdx.x * kWarpsPerCta + warp;
+  const Sched sc = make_sched(p);
+  uint64_t g = sc.R0 + sc.Rs * wid / nw, g_end = sc.R0 + sc.Rs * (wid + 1) / nw;
+  uint64_t lo = g < g_end ? find_chunk(p, g, lane) : p.c0;
+  int t = 0;  // tile of the round being consumed
+  for (bool more = true; more;) {
+  uint64_t ng = 0, nge = 0, nlo = 0;
+  bool fetched = false, nmore = false;
+  auto prefetch = [&]() {
+    if (!fetched) {
+      fetched = true;
+      nmore = next_block(p, sc, lane, ng, nge, nlo);
+    }
+  };
+  for (uint64_t cur = lo; g < g_end; ++cur) {
+    const uint64_t rb = p.round_base[cur];
+    const ChunkDesc d = p.desc[cur];
+    const uint32_t len = desc_len(d), pad = desc_pad(d);
+    const uint8_t* src;
+    uint8_t* dst;
+    int mode;
+    chunk_ptrs<kOp>(p, d, src, dst, mode);
+    const int nrounds = (int)((len + kRoundBytes - 1) / kRoundBytes);
+    const int r0 = (int)(g - rb);
+    const int r1 = (int)(g_end - rb < (uint64_t)nrounds ? g_end - rb : (uint64_t)nrounds);
+    g = rb + (uint64_t)r1;
+    uint32_t ch = (lane == 0 && r0 == 0) ? 0xFFFFFFFFu : 0u;
+    const bool bulk_ok = mode == 0 && ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) &&
+                         (!O::kStore || (reinterpret_cast<uintptr_t>(dst) & 15u) == 0) &&
+                         !(O::kSrcImg && p.image_remote);
+    auto is_bulk = [&](int r) { return bulk_ok && (uint32_t)(r + 1) * kRoundBytes <= len; };
+    uint4 v[8];
+    auto issue = [&](int r, int tt) {
+      if (is_bulk(r)) {
+        if (lane == 0) bulk_load(tile_sa + tt * kRoundBytes, src + (size_t)r * kRoundBytes, kRoundBytes, mb_sa + tt * 8);
+      } else {
+        load_round(v, src, len, mode, r, lane_off);
+      }
+    };
+    issue(r0, t);
+    if (!tables_ready) {
+      wait_tables(mbars + kWarpsPerCta * kTmaTiles);
+      tables_ready = true;
+      warp_trace(p, 1, gtimer());
+    }
+    prefetch();
+    for (int r = r0; r < r1; ++r) {
+      uint8_t* tile = tiles + t * kRoundBytes;
+      // the bulk stores of earlier rounds have finished reading their tiles
+      if (lane == 0) bulk_wait_read();
+      __syncwarp();
+      const bool bulk = is_bulk(r);
+      if (!bulk) {  // register round: into the tile, and to the destination from registers
+#pragma unroll
+        for (int i = 0; i < 8; ++i) *reinterpret_cast<uint4*>(tile + lane_off + i * 512) = v[i];
+        if (O::kStore) {
+          const uint32_t base = (uint32_t)r * kRoundBytes + lane_off;
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const uint32_t o = base + (uint32_t)i * 512;
+            if (o < len) {
+              if (!O::kExactTail || o + 16 <= len)
+                st_stream_v4(dst + o, v[i]);  // image destination: zeros past len are owned padding
+              else
+                st_partial(dst + o, v[i], len - o);
+            }
+          }
+        }
+        __syncwarp();
+      }
+      if (r + 1 < r1) issue(r + 1, t ^ 1);
+      if (bulk) {
+        mbar_wait(mb_sa + t * 8, (phase >> t) & 1u);
+        phase ^= 1u << t;
+        if (O::kStore && lane == 0) bulk_store(dst + (size_t)r * kRoundBytes, tile_sa + t * kRoundBytes, kRoundBytes);
+      }
+      if (O::kCrc) {
+#pragma unroll
+        for (int q = 0; q < 32; ++q)
+          ch = crc_step4(ch, *reinterpret_cast<const uint32_t*>(tile + q * kSegBytes + l4), tb, l4);
+      }
+      fence_proxy_async();  // this round's shared reads before the next bulk copy into the tile
+      __syncwarp();
+      t ^= 1;
+    }
+    uint32_t f = ch;
+    if (O::kCrc) {
+#pragma unroll
+      for (int k = 0; k < kFoldLevels; ++k) {
+        const uint32_t o = __shfl_down_sync(full, f, 1 << k);
+        if ((lane & ((2 << k) - 1)) == 0) f ^= fold_mul(o, ftab + k * 128);
+      }
+    }
+    if (!O::kCrc || (r0 == 0 && r1 == nrounds)) {
+      if (O::kCrc || r1 == nrounds) finish_chunk<kOp>(p, cur, src, dst, len, pad, nrounds, f, lane);
+      continue;
+    }
+    f = __shfl_sync(full, f, 0);
+    const int k = nrounds - r1;
+    const uint32_t term = warp_xor(((f >> (31 - lane)) & 1u) ? utab[k * 32 + lane] : 0u);
+    const unsigned long long mine =
+        (unsigned long long)term | ((((1ull << (r1 - r0)) - 1ull) << r0) << 32);
+    unsigned long long old = 0;
+    if (lane == 0) old = atomicXor(&p.unit_acc[cur - p.c0], mine);
+    const unsigned long long now = __shfl_sync(full, old, 0) ^ mine;
+    if ((now >> 32) == (1ull << nrounds) - 1) {
+      if (lane == 0) p.unit_acc[cur - p.c0] = 0ull;
+      finish_chunk<kOp>(p, cur, src, dst, len, pad, nrounds, (uint32_t)now, lane);
+    }
+  }
+  prefetch();
+  more = nmore;
+  g = ng;
+  g_end = nge;
+  lo = nlo;
+  }
+  if (!tables_ready) wait_tables(mbars + kWarpsPerCta * kTmaTiles);
+  if (lane == 0) bulk_wait_all();  // the bulk stores have landed before the kernel ends
+  release_work(p);
+  warp_trace(p, 0, t_start);
+  warp_trace(p, 2, gtimer());
+  {
+    unsigned smid;
+    asm("mov.u32 %0, %%smid;" : "=r"(smid));
+    warp_trace(p, 3, smid);
+  }
   publish_status<kOp>(p);
 }
 
@@ -697,6 +1000,20 @@ __global__ void build_tables_kernel(const TableParams tp, uint32_t* __restrict__
     uint32_t b = tp.unitpow[t >> 5];
     for (int m = 0; m < (t & 31); ++m) b = gf_mulx(b);
     out[kUnitOff + t] = b;
+  }
+  // column tables (TMA kernel): C_j[e] = (e << 8j) * x^(8*128), byte j of the
+  // register, in the super-table layout (A = [C_0 | C_1], B = [C_2 | C_3]); fold
+  // tables of the shifts x^(-32*2^k)
+  __syncthreads();
+  for (int e = threadIdx.x; e < 1024; e += blockDim.x) scratch[e] = gf_mul((uint32_t)(e & 255) << (8 * (e >> 8)), tp.col_shift);
+  __syncthreads();
+  for (int i = threadIdx.x; i < 1024 * 32; i += blockDim.x) {
+    const int h = i >> 5, st = h >> 9, e = (h >> 1) & 255, half = h & 1;
+    out[kColOff + i] = scratch[(2 * st + half) * 256 + e];
+  }
+  for (int i = threadIdx.x; i < kColFoldWords; i += blockDim.x) {
+    const int lvl = i >> 7, j = (i >> 4) & 7, v = i & 15;
+    out[kColFoldOff + i] = gf_mul((uint32_t)v << (4 * j), tp.col_fold[lvl]);
   }
 }
 
@@ -894,6 +1211,9 @@ static cudaError_t configure_op() {
     e = cudaFuncSetAttribute(sweep_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kSmemBytes);
   if (e == cudaSuccess)
     e = cudaFuncSetAttribute(balanced_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBalSmemBytes);
+  if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck)
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(tma_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmemBytes);
   return e;
 }
 
@@ -914,7 +1234,13 @@ cudaError_t launch_build_tables(const TableParams& tp, uint32_t* out, cudaStream
 
 template <int kOp>
 static void launch_op(const LaunchParams& p, unsigned ctas, cudaStream_t s, int kernel) {
-  if (kernel == 3)
+  if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck) {
+    if (kernel == 4) {
+      tma_kernel<kOp><<<ctas, kThreadsPerCta, kTmaSmemBytes, s>>>(p);
+      return;
+    }
+  }
+  if (kernel == 3 || kernel == 4)
     balanced_kernel<kOp><<<ctas, kThreadsPerCta, kBalSmemBytes, s>>>(p);
   else if (kernel == 2)
     sweep_kernel<kOp><<<ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
@@ -929,7 +1255,7 @@ static void launch_op(const LaunchParams& p, unsigned ctas, cudaStream_t s, int 
 cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel, uint64_t rounds) {
   const uint64_t chunks = p.c1 - p.c0;
   if (chunks == 0) return cudaSuccess;
-  const uint64_t units = kernel == 3 ? rounds : kernel == 2 ? chunks * 16 : chunks;
+  const uint64_t units = kernel >= 3 ? rounds : kernel == 2 ? chunks * 16 : chunks;
   uint64_t ctas = (units + kWarpsPerCta - 1) / kWarpsPerCta;
   if (ctas > (uint64_t)n_sms) ctas = (uint64_t)n_sms;
   switch (op) {

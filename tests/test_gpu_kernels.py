@@ -1,8 +1,9 @@
 """-m gpu: every kernel shape of the data path produces the same bytes.
 
-libchecl dispatches a launch to one of three kernels: 1 grid-stride
+libchecl dispatches a launch to one of four kernels: 1 grid-stride
 warp per chunk, 2 grid-stride 4 KiB units, 3 balanced stretches of rounds (partial
-chunks combined through the atomic CRC accumulator). CHECL_KERNEL=k forces one;
+chunks combined through the atomic CRC accumulator), 4 the same split with bulk
+(TMA) copies, the column CRC and a dynamic tail. CHECL_KERNEL=k forces one;
 each run here (a subprocess: the choice is read once per device) checkpoints a
 registry with ragged, misaligned, multi-chunk and zero-size buffers, in one launch
 and through small staging slots, compares the image with the oracle byte for byte,
@@ -60,9 +61,14 @@ print("kernel ok")
 """
 
 
-@pytest.mark.parametrize("kernel", ["1", "2", "3"])
+@pytest.mark.parametrize("kernel", ["1", "2", "3", "4", "4:0:1", "4:500:3", "4:900:16"])
 def test_forced_kernel_shapes_bit_exact(kernel):
-    env = dict(os.environ, CHECL_KERNEL=kernel)
+    """kernel "4:S:B" = the TMA kernel with the dynamic tail forced on at this size:
+    static share S permille, dynamic blocks of B rounds (S = 0: every round dynamic)."""
+    k, *dyn = kernel.split(":")
+    env = dict(os.environ, CHECL_KERNEL=k)
+    if dyn:
+        env.update(CHECL_STATIC_PERMILLE=dyn[0], CHECL_DYN_BLOCK=dyn[1], CHECL_DYN_MIN_ROUNDS="0")
     r = subprocess.run([sys.executable, "-c", SCRIPT % ROOT], capture_output=True, text=True, env=env, cwd=ROOT,
                        timeout=600)
     assert r.returncode == 0 and "kernel ok" in r.stdout, r.stdout + r.stderr
