@@ -946,7 +946,9 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
     const char* e = std::getenv("CHECL_DYN_MIN_ROUNDS");
     return e ? (uint64_t)std::strtoull(e, nullptr, 10) : ~0ull;
   }();
-  const uint64_t min_rounds = dyn_min != ~0ull ? dyn_min : (uint64_t)ds.n_sms * kWarpsPerCta * 8;
+  // (a dynamic tail pays when a warp has tens of rounds: measured 64 MiB launches (11
+  // rounds per warp) 37 -> 49 us with it, 463 MB (76 per warp) 169 -> 164 us)
+  const uint64_t min_rounds = dyn_min != ~0ull ? dyn_min : (uint64_t)ds.n_sms * kWarpsPerCta * 48;
   if (kernel == 4 && static_pm < 1000 && chunks * (kChunkBytes / kRoundBytes) >= min_rounds) {
     p.work = ds.work.p;
     p.static_permille = static_pm;

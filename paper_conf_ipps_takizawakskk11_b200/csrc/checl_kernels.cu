@@ -38,9 +38,12 @@ constexpr size_t kMbarOff = kTileOff + (size_t)kWarpsPerCta * kStageBytes;
 constexpr size_t kSmemBytes = kMbarOff + 16;
 static_assert(kSmemBytes <= 232448, "fits the 227 KiB opt-in shared memory");
 
+// Global loads are volatile asm: a plain asm has no side effects for the compiler,
+// which then may execute it speculatively outside its branch (it hoisted the next
+// part's first loads above their `if`, with a null source: an illegal address).
 __device__ __forceinline__ uint4 ld_stream_v4(const void* p) {
   uint4 r;
-  asm("ld.global.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+  asm volatile("ld.global.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
       : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
       : "l"(p));
   return r;
@@ -55,7 +58,7 @@ __device__ __forceinline__ void st_stream_v4(void* p, uint4 v) {
 
 __device__ __forceinline__ uint32_t ld_stream_u32(const void* p) {
   uint32_t r;
-  asm("ld.global.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+  asm volatile("ld.global.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
   return r;
 }
 
@@ -701,58 +704,88 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
   // the 16 bytes at lane_off + 512 i (the same offset in the contiguous tile)
   const uint32_t lane_off = (uint32_t)(lane >> 3) * kSegBytes + (uint32_t)(lane & 7) * 16;
 
+  // A part = the rounds [r0, r1) of one chunk inside a stretch. The first round of
+  // the next part (next chunk of the stretch, or first chunk of the next stretch) is
+  // issued during this part's last round, so a warp's copy pipeline never drains at
+  // chunk or stretch boundaries.
+  struct Part {
+    uint64_t c, rb;  // chunk, its round_base
+    const uint8_t* src;
+    uint8_t* dst;
+    uint32_t len, pad;
+    int mode, nrounds, r0, r1;
+    bool bulk_ok;
+  };
+  auto open_part = [&](uint64_t c, uint64_t rb, const ChunkDesc d, uint64_t g, uint64_t ge) {
+    Part q;
+    q.c = c;
+    q.rb = rb;
+    q.len = desc_len(d);
+    q.pad = desc_pad(d);
+    chunk_ptrs<kOp>(p, d, q.src, q.dst, q.mode);
+    q.nrounds = (int)((q.len + kRoundBytes - 1) / kRoundBytes);
+    q.r0 = (int)(g - rb);
+    q.r1 = (int)(ge - rb < (uint64_t)q.nrounds ? ge - rb : (uint64_t)q.nrounds);
+    q.bulk_ok = q.mode == 0 && ((reinterpret_cast<uintptr_t>(q.src) & 15u) == 0) &&
+                (!O::kStore || (reinterpret_cast<uintptr_t>(q.dst) & 15u) == 0) && !(O::kSrcImg && p.image_remote);
+    return q;
+  };
+  auto is_bulk = [&](const Part& q, int r) { return q.bulk_ok && (uint32_t)(r + 1) * kRoundBytes <= q.len; };
+  uint4 v[8];  // the register path's round in flight
+  auto issue = [&](const Part& q, int r, int tt) {
+    if (is_bulk(q, r)) {
+      if (lane == 0) bulk_load(tile_sa + tt * kRoundBytes, q.src + (size_t)r * kRoundBytes, kRoundBytes, mb_sa + tt * 8);
+    } else {
+      load_round(v, q.src, q.len, q.mode, r, lane_off);
+    }
+  };
+
   const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta, wid = (uint64_t)blockIdx.x * kWarpsPerCta + warp;
   const Sched sc = make_sched(p);
-  uint64_t g = sc.R0 + sc.Rs * wid / nw, g_end = sc.R0 + sc.Rs * (wid + 1) / nw;
-  uint64_t lo = g < g_end ? find_chunk(p, g, lane) : p.c0;
-  int t = 0;  // tile of the round being consumed
-  for (bool more = true; more;) {
-  uint64_t ng = 0, nge = 0, nlo = 0;
-  bool fetched = false, nmore = false;
-  auto prefetch = [&]() {
+  uint64_t g = sc.R0 + sc.Rs * wid / nw, g_end = sc.R0 + sc.Rs * (wid + 1) / nw, c = 0;
+  bool have = g < g_end, fetched = false, nmore = false;
+  if (have) {
+    c = find_chunk(p, g, lane);
+  } else {  // no static rounds: straight to the dynamic blocks
+    fetched = true;
+    have = next_block(p, sc, lane, g, g_end, c);
+  }
+  uint64_t ng = 0, nge = 0, nlo = 0;  // the next stretch (dynamic block), once fetched
+  int t = 0;                          // tile of the round being consumed
+  Part cur{};
+  if (have) {
+    cur = open_part(c, p.round_base[c], p.desc[c], g, g_end);
+    issue(cur, cur.r0, t);
+  }
+  if (!tables_ready) {
+    wait_tables(mbars + kWarpsPerCta * kTmaTiles);
+    tables_ready = true;
+    warp_trace(p, 1, gtimer());
+  }
+  while (have) {
+    // the next dynamic block, fetched (and its chunk found) while this stretch's first
+    // round is in flight
     if (!fetched) {
       fetched = true;
       nmore = next_block(p, sc, lane, ng, nge, nlo);
     }
-  };
-  for (uint64_t cur = lo; g < g_end; ++cur) {
-    const uint64_t rb = p.round_base[cur];
-    const ChunkDesc d = p.desc[cur];
-    const uint32_t len = desc_len(d), pad = desc_pad(d);
-    const uint8_t* src;
-    uint8_t* dst;
-    int mode;
-    chunk_ptrs<kOp>(p, d, src, dst, mode);
-    const int nrounds = (int)((len + kRoundBytes - 1) / kRoundBytes);
-    const int r0 = (int)(g - rb);
-    const int r1 = (int)(g_end - rb < (uint64_t)nrounds ? g_end - rb : (uint64_t)nrounds);
-    g = rb + (uint64_t)r1;
-    uint32_t ch = (lane == 0 && r0 == 0) ? 0xFFFFFFFFu : 0u;
-    const bool bulk_ok = mode == 0 && ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) &&
-                         (!O::kStore || (reinterpret_cast<uintptr_t>(dst) & 15u) == 0) &&
-                         !(O::kSrcImg && p.image_remote);
-    auto is_bulk = [&](int r) { return bulk_ok && (uint32_t)(r + 1) * kRoundBytes <= len; };
-    uint4 v[8];
-    auto issue = [&](int r, int tt) {
-      if (is_bulk(r)) {
-        if (lane == 0) bulk_load(tile_sa + tt * kRoundBytes, src + (size_t)r * kRoundBytes, kRoundBytes, mb_sa + tt * 8);
-      } else {
-        load_round(v, src, len, mode, r, lane_off);
-      }
-    };
-    issue(r0, t);
-    if (!tables_ready) {
-      wait_tables(mbars + kWarpsPerCta * kTmaTiles);
-      tables_ready = true;
-      warp_trace(p, 1, gtimer());
+    const uint64_t cur_end = cur.rb + (uint64_t)cur.r1;
+    const bool same = cur_end < g_end, succ = same || nmore;
+    const uint64_t s_c = same ? cur.c + 1 : nlo, s_g = same ? cur_end : ng, s_ge = same ? g_end : nge;
+    ChunkDesc sd{};
+    uint64_t srb = 0;
+    if (succ) {  // loads in flight during this part's rounds
+      sd = p.desc[s_c];
+      srb = p.round_base[s_c];
     }
-    prefetch();
-    for (int r = r0; r < r1; ++r) {
+    Part nxt = cur;
+    uint32_t ch = (lane == 0 && cur.r0 == 0) ? 0xFFFFFFFFu : 0u;
+    for (int r = cur.r0; r < cur.r1; ++r) {
       uint8_t* tile = tiles + t * kRoundBytes;
       // the bulk stores of earlier rounds have finished reading their tiles
       if (lane == 0) bulk_wait_read();
       __syncwarp();
-      const bool bulk = is_bulk(r);
+      const bool bulk = is_bulk(cur, r);
       if (!bulk) {  // register round: into the tile, and to the destination from registers
 #pragma unroll
         for (int i = 0; i < 8; ++i) *reinterpret_cast<uint4*>(tile + lane_off + i * 512) = v[i];
@@ -761,21 +794,27 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
             const uint32_t o = base + (uint32_t)i * 512;
-            if (o < len) {
-              if (!O::kExactTail || o + 16 <= len)
-                st_stream_v4(dst + o, v[i]);  // image destination: zeros past len are owned padding
+            if (o < cur.len) {
+              if (!O::kExactTail || o + 16 <= cur.len)
+                st_stream_v4(cur.dst + o, v[i]);  // image destination: zeros past len are owned padding
               else
-                st_partial(dst + o, v[i], len - o);
+                st_partial(cur.dst + o, v[i], cur.len - o);
             }
           }
         }
         __syncwarp();
       }
-      if (r + 1 < r1) issue(r + 1, t ^ 1);
+      if (r + 1 < cur.r1) {
+        issue(cur, r + 1, t ^ 1);
+      } else if (succ) {
+        nxt = open_part(s_c, srb, sd, s_g, s_ge);
+        issue(nxt, nxt.r0, t ^ 1);
+      }
       if (bulk) {
         mbar_wait(mb_sa + t * 8, (phase >> t) & 1u);
         phase ^= 1u << t;
-        if (O::kStore && lane == 0) bulk_store(dst + (size_t)r * kRoundBytes, tile_sa + t * kRoundBytes, kRoundBytes);
+        if (O::kStore && lane == 0)
+          bulk_store(cur.dst + (size_t)r * kRoundBytes, tile_sa + t * kRoundBytes, kRoundBytes);
       }
       if (O::kCrc) {
 #pragma unroll
@@ -794,28 +833,30 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
         if ((lane & ((2 << k) - 1)) == 0) f ^= fold_mul(o, ftab + k * 128);
       }
     }
-    if (!O::kCrc || (r0 == 0 && r1 == nrounds)) {
-      if (O::kCrc || r1 == nrounds) finish_chunk<kOp>(p, cur, src, dst, len, pad, nrounds, f, lane);
-      continue;
+    if (!O::kCrc || (cur.r0 == 0 && cur.r1 == cur.nrounds)) {
+      if (O::kCrc || cur.r1 == cur.nrounds)
+        finish_chunk<kOp>(p, cur.c, cur.src, cur.dst, cur.len, cur.pad, cur.nrounds, f, lane);
+    } else {
+      f = __shfl_sync(full, f, 0);
+      const int k = cur.nrounds - cur.r1;
+      const uint32_t term = warp_xor(((f >> (31 - lane)) & 1u) ? utab[k * 32 + lane] : 0u);
+      const unsigned long long mine =
+          (unsigned long long)term | ((((1ull << (cur.r1 - cur.r0)) - 1ull) << cur.r0) << 32);
+      unsigned long long old = 0;
+      if (lane == 0) old = atomicXor(&p.unit_acc[cur.c - p.c0], mine);
+      const unsigned long long now = __shfl_sync(full, old, 0) ^ mine;
+      if ((now >> 32) == (1ull << cur.nrounds) - 1) {
+        if (lane == 0) p.unit_acc[cur.c - p.c0] = 0ull;
+        finish_chunk<kOp>(p, cur.c, cur.src, cur.dst, cur.len, cur.pad, cur.nrounds, (uint32_t)now, lane);
+      }
     }
-    f = __shfl_sync(full, f, 0);
-    const int k = nrounds - r1;
-    const uint32_t term = warp_xor(((f >> (31 - lane)) & 1u) ? utab[k * 32 + lane] : 0u);
-    const unsigned long long mine =
-        (unsigned long long)term | ((((1ull << (r1 - r0)) - 1ull) << r0) << 32);
-    unsigned long long old = 0;
-    if (lane == 0) old = atomicXor(&p.unit_acc[cur - p.c0], mine);
-    const unsigned long long now = __shfl_sync(full, old, 0) ^ mine;
-    if ((now >> 32) == (1ull << nrounds) - 1) {
-      if (lane == 0) p.unit_acc[cur - p.c0] = 0ull;
-      finish_chunk<kOp>(p, cur, src, dst, len, pad, nrounds, (uint32_t)now, lane);
+    if (!succ) break;
+    if (!same) {  // into the next stretch: its successor is fetched at the top
+      g_end = nge;
+      fetched = false;
+      nmore = false;
     }
-  }
-  prefetch();
-  more = nmore;
-  g = ng;
-  g_end = nge;
-  lo = nlo;
+    cur = nxt;
   }
   if (!tables_ready) wait_tables(mbars + kWarpsPerCta * kTmaTiles);
   if (lane == 0) bulk_wait_all();  // the bulk stores have landed before the kernel ends
