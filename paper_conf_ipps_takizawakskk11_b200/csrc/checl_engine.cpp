@@ -926,9 +926,10 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
   if (kernel == 4 && op != kOpPack && op != kOpVerify && op != kOpCrc && op != kOpCheck) kernel = 3;
   if (kernel >= 3 && !p.round_base) kernel = 0;
   const bool small = chunks * 2 <= (uint64_t)ds.n_sms * kWarpsPerCta;
-  if (!kernel)
-    kernel = p.round_base ? ((op == kOpPack || op == kOpVerify || op == kOpCrc || op == kOpCheck) ? 4 : 3)
-                          : (small ? 2 : 1);
+  // (below 16 MiB of rounds the bulk-copy path measured no better, and with a dirty
+  // L2 worse: C1 pack 16.5 -> 21 us)
+  const bool tma_op = op == kOpPack || op == kOpVerify || op == kOpCrc || op == kOpCheck;
+  if (!kernel) kernel = p.round_base ? (tma_op && chunks * (kChunkBytes / kRoundBytes) >= 4096 ? 4 : 3) : (small ? 2 : 1);
   if (kernel < 3) p.round_base = nullptr;
   // balanced / TMA launches large enough to have a tail: static stretches for the
   // first part of the rounds, dynamic blocks for the rest (DESIGN.md §5 "Work split");

@@ -21,5 +21,5 @@ timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > $O/bench_ref
 CHECL_TRACE=1 timeout 120 python tools/trace_step.py > $O/trace.log 2>&1
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,temperature.gpu,power.draw --format=csv > $O/nvsmi.txt
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 300 --csv --log-file $O/launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline > $O/launches.log 2>&1
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:"snapshot_kernel|balanced_kernel" -s 2 -c 2 -o $O/prof -f python tools/profile_step.py --reps 2 > $O/ncu_full.log 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:"snapshot_kernel|balanced_kernel|tma_kernel" -s 2 -c 2 -o $O/prof -f python tools/profile_step.py --reps 2 > $O/ncu_full.log 2>&1
 tail -1 $O/ncu_full.log
