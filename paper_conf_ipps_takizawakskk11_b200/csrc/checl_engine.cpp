@@ -971,11 +971,18 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
     ck(cudaMemsetAsync(ds.warp_trace.p, 0, n_tr * 8, s));
     p.warp_trace = ds.warp_trace.p;
   }
+  static const bool host_tr = std::getenv("CHECL_TRACE") != nullptr;
+  const double h0 = host_tr ? now_ms() : 0;
   cudaEvent_t a = ds.events.get(), b = ds.events.get();
   ck(cudaEventRecord(a, s));
+  const double h1 = host_tr ? now_ms() : 0;
   ck(launch_snapshot(op, p, ds.n_sms, s, kernel, chunks * (kChunkBytes / kRoundBytes)));
+  const double h2 = host_tr ? now_ms() : 0;
   ck(cudaEventRecord(b, s));
   kt.spans.push_back({a, b});
+  if (host_tr)
+    std::fprintf(stderr, "[checl] timed_launch op %d kernel %d: record %.1f launch %.1f record %.1f us\n", op, kernel,
+                 (h1 - h0) * 1e3, (h2 - h1) * 1e3, (now_ms() - h2) * 1e3);
   if (p.warp_trace) {
     std::vector<unsigned long long> h(n_tr);
     ck(cudaMemcpyAsync(h.data(), p.warp_trace, n_tr * 8, cudaMemcpyDeviceToHost, s));
