@@ -506,6 +506,9 @@ struct checl_image {
   size_t d_payload_cap = 0;
   uint32_t* d_crc = nullptr;
   size_t d_crc_cap = 0;
+  // device address of host_mut (mapped pinned memory), cached: nullptr = not known yet
+  const uint8_t* mapped_for = nullptr;
+  uint8_t* mapped_dev = nullptr;
 
   void free_device() {
     if (device >= 0 && (d_payload || d_crc)) {
@@ -1092,11 +1095,16 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
     lp.crc = img->d_crc;
     // the host mirror's CRC table is written by the kernel itself through the
     // mapped pinned mirror (no D2H copy after the kernel); plain copy if unmapped
-    void* mirror = nullptr;
-    if (cudaHostGetDevicePointer(&mirror, img->host_mut + P.crc_off, 0) != cudaSuccess) {
-      cudaGetLastError();
-      mirror = nullptr;
+    if (img->mapped_for != img->host_mut) {
+      void* dp = nullptr;
+      if (cudaHostGetDevicePointer(&dp, img->host_mut, 0) != cudaSuccess) {
+        cudaGetLastError();
+        dp = nullptr;
+      }
+      img->mapped_for = img->host_mut;
+      img->mapped_dev = static_cast<uint8_t*>(dp);
     }
+    void* mirror = img->mapped_dev ? img->mapped_dev + P.crc_off : nullptr;
     lp.crc_mirror = static_cast<uint32_t*>(mirror);
     tr("mirror");
     if (P.n_chunks) timed_launch(ds, kt, kOpPack, lp, ds.compute);

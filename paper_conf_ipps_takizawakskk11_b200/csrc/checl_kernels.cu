@@ -757,24 +757,21 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
     cur = open_part(c, p.round_base[c], p.desc[c], g, g_end);
     issue(cur, cur.r0, t);
   }
-  if (!tables_ready) {
-    wait_tables(mbars + kWarpsPerCta * kTmaTiles);
-    tables_ready = true;
-    warp_trace(p, 1, gtimer());
-  }
+  // (the tables are waited for just before the first CRC: by then the first two rounds
+  // are in flight)
   while (have) {
-    // the next dynamic block, fetched (and its chunk found) while this stretch's first
-    // round is in flight
-    if (!fetched) {
-      fetched = true;
-      nmore = next_block(p, sc, lane, ng, nge, nlo);
-    }
+    // successor inside this stretch: its descriptor loads fly during this part's rounds
     const uint64_t cur_end = cur.rb + (uint64_t)cur.r1;
-    const bool same = cur_end < g_end, succ = same || nmore;
-    const uint64_t s_c = same ? cur.c + 1 : nlo, s_g = same ? cur_end : ng, s_ge = same ? g_end : nge;
+    const bool same = cur_end < g_end;
+    bool succ = same, s_known = same || fetched;
+    uint64_t s_c = cur.c + 1, s_g = cur_end, s_ge = g_end;
     ChunkDesc sd{};
     uint64_t srb = 0;
-    if (succ) {  // loads in flight during this part's rounds
+    if (!same && fetched && nmore) {
+      succ = true;
+      s_c = nlo, s_g = ng, s_ge = nge;
+    }
+    if (succ) {
       sd = p.desc[s_c];
       srb = p.round_base[s_c];
     }
@@ -804,11 +801,30 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
         }
         __syncwarp();
       }
-      if (r + 1 < cur.r1) {
-        issue(cur, r + 1, t ^ 1);
-      } else if (succ) {
+      if (r + 1 < cur.r1) issue(cur, r + 1, t ^ 1);
+      // the next dynamic block, fetched (and its chunk found) once per stretch while
+      // this stretch's first rounds are in flight
+      if (!fetched) {
+        fetched = true;
+        nmore = next_block(p, sc, lane, ng, nge, nlo);
+      }
+      if (!s_known) {  // the successor is the next block's first part
+        s_known = true;
+        if (nmore) {
+          succ = true;
+          s_c = nlo, s_g = ng, s_ge = nge;
+          sd = p.desc[s_c];
+          srb = p.round_base[s_c];
+        }
+      }
+      if (r + 1 == cur.r1 && succ) {
         nxt = open_part(s_c, srb, sd, s_g, s_ge);
         issue(nxt, nxt.r0, t ^ 1);
+      }
+      if (!tables_ready) {
+        wait_tables(mbars + kWarpsPerCta * kTmaTiles);
+        tables_ready = true;
+        warp_trace(p, 1, gtimer());
       }
       if (bulk) {
         mbar_wait(mb_sa + t * 8, (phase >> t) & 1u);
