@@ -455,7 +455,7 @@ def main():
             ctx.checkpoint(dev, epoch=i + 1, into=img)
             tc = ctx.last_timing(raw=True)
             coordinate(True, i + 1)
-            ctx.restore(img, dev)
+            ctx.restore(img, dev, report=False)
             tr = ctx.last_timing(raw=True)
             if collect is not None:
                 collect.append((tc, tr))

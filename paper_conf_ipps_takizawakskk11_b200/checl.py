@@ -392,8 +392,13 @@ class Context:
         _check(st, "checl_restore_chain", rep)
         return rep
 
-    def restore(self, image: Image, device: int, stream=None) -> Report:
-        """Restart steps 2-3 (L16): verify every chunk, then rebind every handle."""
+    def restore(self, image: Image, device: int, stream=None, report: bool = True) -> Optional[Report]:
+        """Restart steps 2-3 (L16): verify every chunk, then rebind every handle.
+        report=False passes no report (the call's status alone; a hot loop skips
+        building the Report)."""
+        if not report:
+            _check(lib.checl_restore(self._p, image.handle, device, _stream_ptr(stream), None), "checl_restore")
+            return None
         r = _Report()
         st = lib.checl_restore(self._p, image.handle, device, _stream_ptr(stream), C.byref(r))
         rep = Report._from(r)
