@@ -16,7 +16,7 @@ src, dst = sys.argv[1], sys.argv[2]
 os.makedirs(dst, exist_ok=True)
 import glob  # noqa: E402
 for f in sorted(glob.glob(os.path.join(src, "bench*.json"))) + [
-        os.path.join(src, f) for f in ("pytest_gpu.log", "smoke.log", "nvsmi.txt", "trace.log", "sanitizer.txt")]:
+        os.path.join(src, f) for f in ("pytest_gpu.log", "smoke.log", "nvsmi.txt", "trace.log", "trace_c3.log", "sanitizer.txt")]:
     if os.path.exists(f):
         shutil.copy(f, os.path.join(dst, os.path.basename(f)))
 lines = []
