@@ -57,6 +57,16 @@ def workload(cfg: str, rank: int, c4_scale: float):
     return w
 
 
+def init_dist(dist, torch, dev):
+    """One process per GPU over NCCL. CHECL_BENCH_DIST_BACKEND=gloo is for exercising
+    the multi-rank code path with several ranks on one GPU (timings meaningless)."""
+    backend = os.environ.get("CHECL_BENCH_DIST_BACKEND", "nccl")
+    if backend == "nccl":
+        dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+    else:
+        dist.init_process_group(backend)
+
+
 def peaks():
     try:
         return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -396,10 +406,10 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     world = int(os.environ.get("WORLD_SIZE", "1"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    dev = local
+    dev = local % max(torch.cuda.device_count(), 1)  # (== local on a box with a GPU per rank)
     torch.cuda.set_device(dev)
     if world > 1:
-        dist.init_process_group("nccl", device_id=torch.device("cuda", dev))
+        init_dist(dist, torch, dev)
     w = workload(a.config, rank, a.c4_scale)
     kind = {"random": checl.FILL_RANDOM, "float": checl.FILL_FLOAT, "zeros": checl.FILL_ZEROS}[a.kind]
 
@@ -423,19 +433,18 @@ def main():
             f, _, _, same, _ = agree(not ok, len(handles), S, epoch, None, dev)
             assert f == 0 and same
 
-    def max_over_ranks(x: float) -> float:
+    def over_ranks(x: float, op) -> float:
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        t = torch.tensor([x], dtype=torch.float64, device=dev if dist.get_backend() == "nccl" else "cpu")
+        dist.all_reduce(t, op=op)
         return float(t.item())
 
+    def max_over_ranks(x: float) -> float:
+        return over_ranks(x, dist.ReduceOp.MAX)
+
     def sum_over_ranks(x: float) -> float:
-        if world == 1:
-            return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.SUM)
-        return float(t.item())
+        return over_ranks(x, dist.ReduceOp.SUM)
 
     # inputs smaller than L2: every timed step starts from a flushed L2 (a 2x-L2
     # buffer written between steps, outside the timed spans)
