@@ -41,6 +41,9 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--c4-scale", type=float, default=1.0)
+    ap.add_argument("--restart", action="store_true",
+                    help="every step releases all handles between checkpoint and restore (the restarted process "
+                         "holds only the image; automatic when buffers + image + restored copy exceed HBM)")
     ap.add_argument("--c5-large", action="store_true", help="C5 with 16 x 1 GiB instead of the C2 set")
     ap.add_argument("--mode", default="snapshot", choices=["snapshot", "incremental"],
                     help="incremental: checl_checkpoint_incremental with --dirty of the chunks rewritten per step")
@@ -387,6 +390,24 @@ def run_incremental(a):
     ctx.close()
 
 
+def restart_samples_bad(ctx, handles, w, kind: str, per_buffer: int = 8) -> int:
+    """Restart mode: sampled 64 KiB chunks (random ones + each buffer's last) of the
+    restored buffers vs the synth generator's bytes; the number that differ."""
+    import numpy as np
+    import synth
+    rng = np.random.default_rng(w.seed)
+    bad = 0
+    for h, b in zip(handles, w.buffers):
+        nch = (b.size + 65535) // 65536
+        if nch == 0:
+            continue
+        t = ctx.tensor(h)
+        for k in [int(x) for x in rng.integers(0, nch, per_buffer)] + [nch - 1]:
+            lo, n = k * 65536, min(65536, b.size - k * 65536)
+            bad += int(not np.array_equal(t[lo:lo + n].cpu().numpy(), synth.fill_slice(lo, n, w.seed, b.stream, kind)))
+    return bad
+
+
 def main():
     a = parse()
     if a.mode == "incremental":
@@ -422,6 +443,11 @@ def main():
     handles = [ctx.register(t, b.flags) for t, b in zip(tensors, w.buffers)]
     S = w.total_bytes
     n_chunks = sum((b.size + 65535) // 65536 for b in w.buffers)
+    # Restart mode (L16 restart steps 2-3: the new process re-creates every object from
+    # the image). The application's buffers are dropped after the first checkpoint and
+    # every timed step releases all handles before restoring, so HBM holds one image
+    # plus one copy of the buffers: C4 at full size (64 GiB x 3 does not fit 179 GiB).
+    restart = a.restart or 3 * S + (4 << 30) > torch.cuda.get_device_properties(dev).total_memory
 
     def barrier():
         if world > 1:
@@ -464,6 +490,9 @@ def main():
             ctx.checkpoint(dev, epoch=i + 1, into=img)
             tc = ctx.last_timing(raw=True)
             coordinate(True, i + 1)
+            if restart:
+                for h in handles:
+                    ctx.release(h)
             ctx.restore(img, dev, report=False)
             tr = ctx.last_timing(raw=True)
             if collect is not None:
@@ -480,6 +509,16 @@ def main():
 
     # -- value: device-resident image (HBM) --------------------------------------
     dimg = ctx.checkpoint_device(dev, epoch=0)
+    crc0 = None
+    if restart:
+        import numpy as np
+        hd = dimg.header()
+        crc0 = np.array(dimg.view()[hd["crc_off"]:hd["crc_off"] + 4 * n_chunks])
+        for h in handles:
+            ctx.release(h)
+        del tensors[:]  # the user's buffers are gone; only the image survives the restart
+        torch.cuda.empty_cache()
+        ctx.restore(dimg, dev, report=False)
     run(dimg, a.warmup, None)
     phases = []
     barrier()
@@ -494,6 +533,13 @@ def main():
     for h, t in zip(handles, tensors):
         ptr, nb, d = ctx.translate(h)
         n_diff += checl.debug_compare(dev, ptr, t.data_ptr(), nb) if nb else 0
+    if restart:
+        # no original left to compare with: the last image's CRC table must equal the
+        # first one's (taken from the application's buffers), and sampled chunks of the
+        # restored buffers must equal the synth generator's bytes
+        hd = dimg.header()
+        n_diff += int(not (dimg.view()[hd["crc_off"]:hd["crc_off"] + 4 * n_chunks] == crc0).all())
+        n_diff += restart_samples_bad(ctx, handles, w, a.kind)
     pack_ms = statistics.mean(p[0]["kernel_ms"] for p in phases)
     verify_ms = statistics.mean(p[1]["kernel_ms"] for p in phases)
     ck_ms = statistics.mean(p[0]["total_ms"] for p in phases)
@@ -563,6 +609,8 @@ def main():
             "config": {"workload": w.name, "payload_bytes_per_gpu": S, "n_buffers": len(w.buffers),
                        "n_chunks": n_chunks, "fill": a.kind,
                        "image": "device-resident (HBM), reused across steps",
+                       "step": ("checkpoint -> release every handle (restart) -> restore re-creates them" if restart
+                                else "checkpoint -> restore (rebind)"),
                        "l2": ("inputs larger than L2" if S > L2_BYTES
                               else "inputs smaller than L2: L2 flushed (252 MB write) before every timed step"),
                        "parallelism": f"independent snapshot per rank, {world} rank(s)"},

@@ -20,7 +20,8 @@ timeout 300 python bench.py --mode incremental --dirty 0.1 > $O/bench_incrementa
 timeout 600 python bench.py --impl reference --steps 3 --warmup 3 > $O/bench_reference.json 2> $O/bench_ref.err
 CHECL_TRACE=1 timeout 120 python tools/trace_step.py > $O/trace.log 2>&1
 CHECL_TRACE=1 timeout 300 python tools/trace_step.py C3 6 > $O/trace_c3.log 2>&1
-timeout 900 python bench.py --config C4 --c4-scale 0.5 --no-cpu-baseline --steps 3 --warmup 3 > $O/bench_c4_half.json 2> $O/bench_c4.err
+timeout 300 python bench.py --restart --no-cpu-baseline > $O/bench_c2_restart.json 2> $O/bench_c2_restart.err
+timeout 1200 python bench.py --config C4 --steps 3 --warmup 3 > $O/bench_c4.json 2> $O/bench_c4.err
 nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm,temperature.gpu,power.draw --format=csv > $O/nvsmi.txt
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 300 --csv --log-file $O/launches.csv python bench.py --steps 2 --warmup 1 --no-cpu-baseline > $O/launches.log 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on -k regex:"snapshot_kernel|balanced_kernel|tma_kernel" -s 2 -c 2 -o $O/prof -f python tools/profile_step.py --reps 2 > $O/ncu_full.log 2>&1
