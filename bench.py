@@ -516,7 +516,7 @@ def main():
         crc0 = np.array(dimg.view()[hd["crc_off"]:hd["crc_off"] + 4 * n_chunks])
         for h in handles:
             ctx.release(h)
-        del tensors[:]  # the user's buffers are gone; only the image survives the restart
+        del tensors[:], t  # the user's buffers are gone (t: the fill loop's last one); only the image survives
         torch.cuda.empty_cache()
         ctx.restore(dimg, dev, report=False)
     run(dimg, a.warmup, None)
