@@ -253,6 +253,29 @@ def test_restore_twice_and_release_owned(ctx):
         ctx.translate(ds.handles[0])
 
 
+def test_restart_loop_release_all_then_restore(ctx):
+    """bench.py restart mode (L16 restart steps 2-3): checkpoint -> release every
+    handle -> restore re-creates them, repeated on one device image. Every image equals
+    the oracle's (same ids, flags, bytes) and the re-created buffers hold the bytes."""
+    ds = make_set(ctx, RAGGED, seed=21, offsets=[3] * len(RAGGED))
+    want = O.checkpoint(oracle_entries(ds), device=DEV, epoch=1)
+    img = ctx.checkpoint_device(DEV, epoch=1)
+    assert np.array_equal(img.to_host().view(), want)
+    for h in ds.handles:
+        ctx.release(h)
+    del ds.views[:], ds.bases[:]  # the application's buffers are gone
+    for epoch in (2, 3, 4):
+        rep = ctx.restore(img, DEV)
+        assert rep.n_bad_chunks == 0 and rep.n_buffers == len(RAGGED)
+        for h, b in zip(ds.handles, ds.host):
+            assert np.array_equal(bound_bytes(ctx, h), b)
+        ctx.checkpoint(DEV, epoch=epoch, into=img)
+        assert np.array_equal(img.to_host().view(), O.checkpoint(oracle_entries(ds), device=DEV, epoch=epoch))
+        for h in ds.handles:
+            ctx.release(h)
+    assert ctx.count(DEV)[0] == 0
+
+
 def test_checkpoint_into_reuses_and_grows(ctx):
     ds = make_set(ctx, [1000, 70000], seed=12)
     img = ctx.checkpoint(DEV, epoch=1)

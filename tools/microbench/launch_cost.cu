@@ -2,6 +2,7 @@
 // 320 threads, 217 KB dynamic smem) from an idle GPU, with and without a 135 KB
 // bulk-copied table prologue, to separate the fixed per-launch cost of the
 // snapshot kernels from their streaming time. Not part of the library.
+#include <chrono>
 #include <cstdint>
 #include <cstdio>
 #include <cuda_runtime.h>
@@ -64,6 +65,64 @@ int main() {
     }
     const char* name[] = {"empty 217KB smem", "135KB table prologue", "empty no smem", "2x table prologue"};
     printf("%-22s mean %.2f us  min %.2f us\n", name[mode], tot / 15 * 1e3, mn * 1e3);
+  }
+  // graph of [event a, kernel, event b]: the GPU receives the three together, so the
+  // span no longer contains the host's launch latency. Host cost measured per call:
+  // (g) launch only, (u) kernel-node parameter + both event updates, then launch.
+  {
+    cudaStream_t s;
+    cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
+    cudaGraph_t g;
+    cudaGraphCreate(&g, 0);
+    cudaGraphNode_t na, nk, nb;
+    cudaGraphAddEventRecordNode(&na, g, nullptr, 0, a);
+    const uint8_t* tp = tab;
+    uint32_t by = 135680;
+    int* sk = nullptr;
+    void* args[] = {&tp, &by, &sk};
+    cudaKernelNodeParams kp = {};
+    kp.func = (void*)k<true>;
+    kp.gridDim = dim3(148);
+    kp.blockDim = dim3(320);
+    kp.sharedMemBytes = (unsigned)smem;
+    kp.kernelParams = args;
+    cudaGraphAddKernelNode(&nk, g, &na, 1, &kp);
+    cudaGraphAddEventRecordNode(&nb, g, &nk, 1, b);
+    cudaGraphExec_t ge;
+    cudaGraphInstantiate(&ge, g, 0);
+    cudaEvent_t a2, b2;
+    cudaEventCreate(&a2);
+    cudaEventCreate(&b2);
+    for (int mode = 0; mode < 3; ++mode) {
+      float tot = 0, mn = 1e9;
+      double host = 0;
+      for (int r = 0; r < 40; ++r) {
+        cudaDeviceSynchronize();
+        auto t0 = std::chrono::steady_clock::now();
+        cudaEvent_t ea = a, eb = b;
+        if (mode == 0) {
+          cudaGraphLaunch(ge, s);
+        } else if (mode == 1) {
+          ea = (r & 1) ? a2 : a, eb = (r & 1) ? b2 : b;
+          cudaGraphExecKernelNodeSetParams(ge, nk, &kp);
+          cudaGraphExecEventRecordNodeSetEvent(ge, na, ea);
+          cudaGraphExecEventRecordNodeSetEvent(ge, nb, eb);
+          cudaGraphLaunch(ge, s);
+        } else {
+          cudaEventRecord(a, s);
+          k<true><<<148, 320, smem, s>>>(tab, 135680, nullptr);
+          cudaEventRecord(b, s);
+        }
+        auto t1 = std::chrono::steady_clock::now();
+        cudaEventSynchronize(eb);
+        float ms;
+        cudaEventElapsedTime(&ms, ea, eb);
+        if (r >= 10) tot += ms, mn = ms < mn ? ms : mn, host += std::chrono::duration<double, std::micro>(t1 - t0).count();
+      }
+      const char* name[] = {"graph [ev,k,ev]", "graph + node updates", "stream record/launch/record"};
+      printf("%-28s span mean %.2f us  min %.2f us  host %.2f us/call\n", name[mode], tot / 30 * 1e3, mn * 1e3,
+             host / 30);
+    }
   }
   return 0;
 }
