@@ -35,6 +35,8 @@ namespace checl {
 size_t snapshot_smem_bytes();
 cudaError_t snapshot_configure();
 cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel, uint64_t rounds);
+cudaError_t snapshot_launch_config(int op, const LaunchParams& p, int n_sms, int kernel, uint64_t rounds,
+                                   const void** fn, unsigned* ctas, size_t* smem);
 cudaError_t launch_build_tables(const TableParams& tp, uint32_t* out, cudaStream_t s);
 cudaError_t launch_fill(uint8_t* ptr, uint64_t bytes, uint64_t key, int kind, int n_sms, cudaStream_t s);
 cudaError_t launch_compare(const uint8_t* a, const uint8_t* b, uint64_t bytes, unsigned long long* n_diff, int n_sms,
@@ -253,6 +255,19 @@ TableParams table_params() {
 
 // ---- per-device resources ---------------------------------------------------
 
+// One instantiated CUDA graph [event record a -> snapshot kernel -> event record b]
+// per (kernel function, grid): a timed launch updates the kernel node's parameters
+// and the two events and launches the graph, so the GPU receives the three together
+// (the host's launch latency is no longer inside the kernel's event span) and the
+// host spends one graph launch instead of record + launch + record
+// (profiles/r01k/launch_graph.txt). CHECL_GRAPH=0 uses plain stream launches.
+struct LaunchGraph {
+  const void* fn = nullptr;
+  unsigned ctas = 0;
+  cudaGraphExec_t exec = nullptr;
+  cudaGraphNode_t ev_a = nullptr, kern = nullptr, ev_b = nullptr;
+};
+
 struct EventPool {
   std::vector<cudaEvent_t> ev;
   size_t used = 0;
@@ -370,6 +385,7 @@ struct DevState {
   PinnedBuf<unsigned long long> h_status;
   PinnedBuf<BufferRecord> h_recs;
   EventPool events;
+  std::vector<LaunchGraph> graphs;
   Plan plan;
 
   void init(int d) {
@@ -437,6 +453,8 @@ struct DevState {
     plan.d_desc.release();
     h_status.release();
     h_recs.release();
+    for (auto& g : graphs) cudaGraphExecDestroy(g.exec);
+    graphs.clear();
     for (auto e : events.ev) cudaEventDestroy(e);
     events.ev.clear();
     if (compute) cudaStreamDestroy(compute);
@@ -984,14 +1002,60 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
   static const bool host_tr = std::getenv("CHECL_TRACE") != nullptr;
   const double h0 = host_tr ? now_ms() : 0;
   cudaEvent_t a = ds.events.get(), b = ds.events.get();
-  ck(cudaEventRecord(a, s));
-  const double h1 = host_tr ? now_ms() : 0;
-  ck(launch_snapshot(op, p, ds.n_sms, s, kernel, chunks * (kChunkBytes / kRoundBytes)));
-  const double h2 = host_tr ? now_ms() : 0;
-  ck(cudaEventRecord(b, s));
+  static const bool use_graph = [] {
+    const char* e = std::getenv("CHECL_GRAPH");
+    return !e || std::atoi(e) != 0;
+  }();
+  const void* fn = nullptr;
+  unsigned ctas = 0;
+  size_t smem = 0;
+  if (use_graph)
+    ck(snapshot_launch_config(op, p, ds.n_sms, kernel, chunks * (kChunkBytes / kRoundBytes), &fn, &ctas, &smem));
+  double h1 = 0, h2 = 0;
+  if (fn) {
+    LaunchGraph* g = nullptr;
+    for (auto& x : ds.graphs)
+      if (x.fn == fn && x.ctas == ctas) g = &x;
+    void* args[] = {&p};
+    cudaKernelNodeParams kp = {};
+    kp.func = const_cast<void*>(fn);
+    kp.gridDim = dim3(ctas);
+    kp.blockDim = dim3(kThreadsPerCta);
+    kp.sharedMemBytes = (unsigned)smem;
+    kp.kernelParams = args;
+    if (!g) {
+      LaunchGraph n;
+      n.fn = fn;
+      n.ctas = ctas;
+      cudaGraph_t gr;
+      ck(cudaGraphCreate(&gr, 0));
+      ck(cudaGraphAddEventRecordNode(&n.ev_a, gr, nullptr, 0, a));
+      ck(cudaGraphAddKernelNode(&n.kern, gr, &n.ev_a, 1, &kp));
+      ck(cudaGraphAddEventRecordNode(&n.ev_b, gr, &n.kern, 1, b));
+      const cudaError_t e = cudaGraphInstantiate(&n.exec, gr, 0);
+      cudaGraphDestroy(gr);
+      ck(e);
+      ds.graphs.push_back(n);
+      g = &ds.graphs.back();
+    } else {
+      ck(cudaGraphExecKernelNodeSetParams(g->exec, g->kern, &kp));
+      ck(cudaGraphExecEventRecordNodeSetEvent(g->exec, g->ev_a, a));
+      ck(cudaGraphExecEventRecordNodeSetEvent(g->exec, g->ev_b, b));
+    }
+    h1 = host_tr ? now_ms() : 0;
+    ck(cudaGraphLaunch(g->exec, s));
+    h2 = host_tr ? now_ms() : 0;
+  } else {
+    ck(cudaEventRecord(a, s));
+    h1 = host_tr ? now_ms() : 0;
+    ck(launch_snapshot(op, p, ds.n_sms, s, kernel, chunks * (kChunkBytes / kRoundBytes)));
+    h2 = host_tr ? now_ms() : 0;
+    ck(cudaEventRecord(b, s));
+  }
   kt.spans.push_back({a, b});
   if (host_tr)
-    std::fprintf(stderr, "[checl] timed_launch op %d kernel %d: record %.1f launch %.1f record %.1f us\n", op, kernel,
+    std::fprintf(stderr, "[checl] timed_launch op %d kernel %d%s: record/update %.1f launch %.1f record %.1f us\n", op,
+                 kernel, fn ? " (graph)" : "",
                  (h1 - h0) * 1e3, (h2 - h1) * 1e3, (now_ms() - h2) * 1e3);
   if (p.warp_trace) {
     std::vector<unsigned long long> h(n_tr);

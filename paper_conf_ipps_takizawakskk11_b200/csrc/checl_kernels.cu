@@ -1305,16 +1305,56 @@ static void launch_op(const LaunchParams& p, unsigned ctas, cudaStream_t s, int 
     snapshot_kernel<kOp><<<ctas, kThreadsPerCta, kSmemBytes, s>>>(p);
 }
 
+template <int kOp>
+static const void* op_fn(int kernel, size_t* smem) {
+  if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck) {
+    if (kernel == 4) {
+      *smem = kTmaSmemBytes;
+      return reinterpret_cast<const void*>(tma_kernel<kOp>);
+    }
+  }
+  if (kernel == 3 || kernel == 4) {
+    *smem = kBalSmemBytes;
+    return reinterpret_cast<const void*>(balanced_kernel<kOp>);
+  }
+  *smem = kSmemBytes;
+  return kernel == 2 ? reinterpret_cast<const void*>(sweep_kernel<kOp>)
+                     : reinterpret_cast<const void*>(snapshot_kernel<kOp>);
+}
+
+static uint64_t snapshot_ctas(const LaunchParams& p, int n_sms, int kernel, uint64_t rounds) {
+  const uint64_t chunks = p.c1 - p.c0;
+  const uint64_t units = kernel >= 3 ? rounds : kernel == 2 ? chunks * 16 : chunks;
+  const uint64_t ctas = (units + kWarpsPerCta - 1) / kWarpsPerCta;
+  return ctas > (uint64_t)n_sms ? (uint64_t)n_sms : ctas;
+}
+
+// The kernel, grid and dynamic shared memory launch_snapshot would use (for a
+// kernel node of a CUDA graph); *fn = nullptr when the launch has no chunks.
+cudaError_t snapshot_launch_config(int op, const LaunchParams& p, int n_sms, int kernel, uint64_t rounds,
+                                   const void** fn, unsigned* ctas, size_t* smem) {
+  *fn = nullptr;
+  if (p.c1 == p.c0) return cudaSuccess;
+  *ctas = (unsigned)snapshot_ctas(p, n_sms, kernel, rounds);
+  switch (op) {
+    case kOpPack: *fn = op_fn<kOpPack>(kernel, smem); break;
+    case kOpVerify: *fn = op_fn<kOpVerify>(kernel, smem); break;
+    case kOpCrc: *fn = op_fn<kOpCrc>(kernel, smem); break;
+    case kOpCheck: *fn = op_fn<kOpCheck>(kernel, smem); break;
+    case kOpCopy: *fn = op_fn<kOpCopy>(kernel, smem); break;
+    case kOpScatter: *fn = op_fn<kOpScatter>(kernel, smem); break;
+    default: return cudaErrorInvalidValue;
+  }
+  return cudaSuccess;
+}
+
 // kernel 1 = warp per chunk (snapshot_kernel), 2 = 4 KiB units swept by the grid
 // (sweep_kernel; p.unit_acc must be zero for the chunk range when the op CRCs —
 // the kernel leaves it zero again)
 // (3 = balanced_kernel: needs p.round_base; `rounds` = the launch's round count)
 cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel, uint64_t rounds) {
-  const uint64_t chunks = p.c1 - p.c0;
-  if (chunks == 0) return cudaSuccess;
-  const uint64_t units = kernel >= 3 ? rounds : kernel == 2 ? chunks * 16 : chunks;
-  uint64_t ctas = (units + kWarpsPerCta - 1) / kWarpsPerCta;
-  if (ctas > (uint64_t)n_sms) ctas = (uint64_t)n_sms;
+  if (p.c1 == p.c0) return cudaSuccess;
+  const uint64_t ctas = snapshot_ctas(p, n_sms, kernel, rounds);
   switch (op) {
     case kOpPack: launch_op<kOpPack>(p, (unsigned)ctas, s, kernel); break;
     case kOpVerify: launch_op<kOpVerify>(p, (unsigned)ctas, s, kernel); break;
