@@ -264,6 +264,7 @@ TableParams table_params() {
 struct LaunchGraph {
   const void* fn = nullptr;
   unsigned ctas = 0;
+  cudaGraph_t graph = nullptr;  // kept: the exec updates name its nodes by these handles
   cudaGraphExec_t exec = nullptr;
   cudaGraphNode_t ev_a = nullptr, kern = nullptr, ev_b = nullptr;
 };
@@ -453,7 +454,10 @@ struct DevState {
     plan.d_desc.release();
     h_status.release();
     h_recs.release();
-    for (auto& g : graphs) cudaGraphExecDestroy(g.exec);
+    for (auto& g : graphs) {
+      cudaGraphExecDestroy(g.exec);
+      cudaGraphDestroy(g.graph);
+    }
     graphs.clear();
     for (auto e : events.ev) cudaEventDestroy(e);
     events.ev.clear();
@@ -936,6 +940,11 @@ LaunchParams base_params(DevState& ds) {
   return p;
 }
 
+void gck(const char* what, cudaError_t e) {
+  if (e != cudaSuccess && std::getenv("CHECL_TRACE")) std::fprintf(stderr, "[checl] %s: %s\n", what, cudaGetErrorName(e));
+  ck(e);
+}
+
 void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0, cudaStream_t s) {
   LaunchParams p = p0;
   // experiments only (tools/exp_run.py): CHECL_EXP_PACK_OP=2|4 replaces the pack
@@ -1027,23 +1036,23 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
       LaunchGraph n;
       n.fn = fn;
       n.ctas = ctas;
-      cudaGraph_t gr;
-      ck(cudaGraphCreate(&gr, 0));
-      ck(cudaGraphAddEventRecordNode(&n.ev_a, gr, nullptr, 0, a));
-      ck(cudaGraphAddKernelNode(&n.kern, gr, &n.ev_a, 1, &kp));
-      ck(cudaGraphAddEventRecordNode(&n.ev_b, gr, &n.kern, 1, b));
+      gck("cudaGraphCreate", cudaGraphCreate(&n.graph, 0));
+      cudaGraph_t gr = n.graph;
+      gck("cudaGraphAddEventRecordNode", cudaGraphAddEventRecordNode(&n.ev_a, gr, nullptr, 0, a));
+      gck("cudaGraphAddKernelNode", cudaGraphAddKernelNode(&n.kern, gr, &n.ev_a, 1, &kp));
+      gck("cudaGraphAddEventRecordNode", cudaGraphAddEventRecordNode(&n.ev_b, gr, &n.kern, 1, b));
       const cudaError_t e = cudaGraphInstantiate(&n.exec, gr, 0);
-      cudaGraphDestroy(gr);
-      ck(e);
+      if (e != cudaSuccess) cudaGraphDestroy(gr);
+      gck("cudaGraphInstantiate", e);
       ds.graphs.push_back(n);
       g = &ds.graphs.back();
     } else {
-      ck(cudaGraphExecKernelNodeSetParams(g->exec, g->kern, &kp));
-      ck(cudaGraphExecEventRecordNodeSetEvent(g->exec, g->ev_a, a));
-      ck(cudaGraphExecEventRecordNodeSetEvent(g->exec, g->ev_b, b));
+      gck("cudaGraphExecKernelNodeSetParams", cudaGraphExecKernelNodeSetParams(g->exec, g->kern, &kp));
+      gck("cudaGraphExecEventRecordNodeSetEvent", cudaGraphExecEventRecordNodeSetEvent(g->exec, g->ev_a, a));
+      gck("cudaGraphExecEventRecordNodeSetEvent", cudaGraphExecEventRecordNodeSetEvent(g->exec, g->ev_b, b));
     }
     h1 = host_tr ? now_ms() : 0;
-    ck(cudaGraphLaunch(g->exec, s));
+    gck("cudaGraphLaunch", cudaGraphLaunch(g->exec, s));
     h2 = host_tr ? now_ms() : 0;
   } else {
     ck(cudaEventRecord(a, s));

@@ -263,7 +263,7 @@ def test_restart_loop_release_all_then_restore(ctx):
     assert np.array_equal(img.to_host().view(), want)
     for h in ds.handles:
         ctx.release(h)
-    del ds.views[:], ds.bases[:]  # the application's buffers are gone
+    del ds.tensors[:], ds.bases[:]  # the application's buffers are gone
     for epoch in (2, 3, 4):
         rep = ctx.restore(img, DEV)
         assert rep.n_bad_chunks == 0 and rep.n_buffers == len(RAGGED)
