@@ -265,6 +265,8 @@ def run_migration(a):
         ptr, nb, d = ctx.translate(h)
         if d == dev:
             n_diff += checl.debug_compare(dev, ptr, t.data_ptr(), nb)
+        elif nb:  # the buffers now live on another GPU: bring them back (torch peer copy) to compare
+            n_diff += int(not torch.equal(ctx.tensor(h).to(dev), t))
     if world > 1:
         t = torch.tensor([ms], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
