@@ -1217,6 +1217,9 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       packed[i] = ds.events.get();
       drained[i] = ds.events.get();
     }
+    // diagnostics: CHECL_STAGE_TRACE=1 times every stage's D2H (events around it)
+    static const bool stage_tr = std::getenv("CHECL_STAGE_TRACE") != nullptr;
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> d2h;
     ck(cudaEventRecord(c_begin, ds.copy));
     for (size_t s = 0; s < P.stages.size(); ++s) {
       const Stage& S = P.stages[s];
@@ -1229,9 +1232,40 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       timed_launch(ds, kt, kOpPack, lp, ds.compute);
       ck(cudaEventRecord(packed[k], ds.compute));
       ck(cudaStreamWaitEvent(ds.copy, packed[k], 0));
+      if (stage_tr) {
+        d2h.push_back({ds.events.get(), ds.events.get()});
+        ck(cudaEventRecord(d2h.back().first, ds.copy));
+      }
       ck(cudaMemcpyAsync(img->host_mut + P.payload_off + S.img_lo, ds.slot(k), S.img_hi - S.img_lo,
                          cudaMemcpyDeviceToHost, ds.copy));
+      if (stage_tr) ck(cudaEventRecord(d2h.back().second, ds.copy));
       ck(cudaEventRecord(drained[k], ds.copy));
+    }
+    if (stage_tr && !d2h.empty()) {
+      ck(cudaStreamSynchronize(ds.copy));
+      double busy = 0, gap = 0, gap_max = 0, pk_to_start = 0;
+      for (size_t s = 0; s < d2h.size(); ++s) {
+        float a = 0, b = 0, k_end = 0;
+        cudaEventElapsedTime(&a, c_begin, d2h[s].first);
+        cudaEventElapsedTime(&b, c_begin, d2h[s].second);
+        cudaEventElapsedTime(&k_end, c_begin, kt.spans[s].second);
+        busy += b - a;
+        pk_to_start += a - k_end;
+        if (s) {
+          float pb = 0;
+          cudaEventElapsedTime(&pb, c_begin, d2h[s - 1].second);
+          gap += a - pb;
+          gap_max = std::max(gap_max, (double)(a - pb));
+        }
+      }
+      float tot = 0;
+      cudaEventElapsedTime(&tot, c_begin, d2h.back().second);
+      std::fprintf(stderr,
+                   "[checl] stages %zu: span %.3f ms, D2H busy %.3f ms (%.1f us each), gaps %.1f us total (max %.1f), "
+                   "first D2H starts %.1f us after begin, D2H start - pack end mean %.1f us\n",
+                   d2h.size(), tot, busy, busy / d2h.size() * 1e3, gap * 1e3, gap_max * 1e3,
+                   [&] { float a = 0; cudaEventElapsedTime(&a, c_begin, d2h[0].first); return a * 1e3; }(),
+                   pk_to_start / d2h.size() * 1e3);
     }
     if (P.n_chunks)
       ck(cudaMemcpyAsync(img->host_mut + P.crc_off, ds.crc_scratch.p, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.copy));
