@@ -8,6 +8,8 @@ byte for byte, the HBM image's metadata mirror equals it too, restore from both
 reproduces every buffer, a random single-bit payload flip is reported at the
 oracle's chunk, and an incremental image after random rewrites equals the
 oracle's delta."""
+import os
+
 import numpy as np
 import pytest
 
@@ -40,7 +42,8 @@ def _sizes(rng, n):
     return out
 
 
-@pytest.mark.parametrize("case", range(24))
+# CHECL_FUZZ_CASES widens the sweep (default 24 cases; profiles/ records a 400-case run)
+@pytest.mark.parametrize("case", range(int(os.environ.get("CHECL_FUZZ_CASES", "24"))))
 def test_random_registry(case):
     rng = np.random.default_rng(1000 + case)
     ctx = checl.Context()
