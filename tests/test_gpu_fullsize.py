@@ -88,6 +88,7 @@ def test_c4_full_size_device_image_restart_sampled():
     same samples."""
     w = synth.c4_md_rank(0)
     S = w.total_bytes
+    torch.cuda.empty_cache()  # what an earlier test's restore left in torch's cache
     free, _ = torch.cuda.mem_get_info(0)
     if free < 2 * S + (8 << 30):
         pytest.skip(f"needs {2 * S >> 30} GiB free on the device")
