@@ -75,7 +75,7 @@ def test_c4_md_rank_full_size_sampled():
 def _device_bytes(ptr: int, n: int) -> np.ndarray:
     """n bytes of device memory at ptr (a torch view, copied to the host)."""
     class _Iface:
-        __cuda_array_interface__ = {"shape": (n,), "typestr": "|u1", "data": (ptr, True), "version": 2,
+        __cuda_array_interface__ = {"shape": (n,), "typestr": "|u1", "data": (ptr, False), "version": 2,
                                     "strides": None}
     return torch.as_tensor(_Iface(), device="cuda:0").cpu().numpy()
 
