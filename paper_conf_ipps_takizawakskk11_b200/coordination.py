@@ -50,9 +50,11 @@ def agree(failed: bool, n_buffers: int, nbytes: int, epoch: int, group=None, dev
 
 
 def coordinated(take_local: Callable[[], Tuple[object, int, int]], epoch: int, group=None,
-                device: Optional[int] = None) -> GlobalSnapshot:
+                device: Optional[int] = None, keep=None) -> GlobalSnapshot:
     """Runs `take_local()` -> (image, n_buffers, bytes) on every rank, then the
-    status all-reduce; frees the local image if the global snapshot aborts."""
+    status all-reduce; frees the local image if the global snapshot aborts, unless it
+    is `keep` (a caller-owned image reused through checl_checkpoint_into: the caller
+    keeps it, and `committed` = False says its contents are not a global snapshot)."""
     img, n, b, failed = None, 0, 0, False
     try:
         img, n, b = take_local()
@@ -61,7 +63,8 @@ def coordinated(take_local: Callable[[], Tuple[object, int, int]], epoch: int, g
     f, tn, tb, same, ep = agree(failed, n, b, epoch, group, device)
     ok = f == 0 and same
     if not ok and img is not None:
-        img.free()
+        if img is not keep:
+            img.free()
         img = None
     return GlobalSnapshot(ok, img, f, tn, tb, ep, same)
 
@@ -74,4 +77,4 @@ def coordinated_checkpoint(ctx, device: int, epoch: int, group=None, stream=None
         if on_device:
             return ctx.checkpoint_device(device, stream, epoch), n, b
         return ctx.checkpoint(device, stream, epoch, into=into), n, b
-    return coordinated(local, epoch, group, device)
+    return coordinated(local, epoch, group, device, keep=into)

@@ -33,7 +33,7 @@ def _worker(rank, world, port, scenario, q):
     img = FakeImage()
 
     def local():
-        if scenario == "fail" and rank == world - 1:
+        if scenario in ("fail", "fail_keep") and rank == world - 1:
             raise RuntimeError("injected local checkpoint failure")
         return img, 3 + rank, 1000 * (rank + 1)
 
@@ -42,7 +42,7 @@ def _worker(rank, world, port, scenario, q):
         epoch = 7 + ((1 << 48) if rank == 1 else 0)
     if scenario == "epoch_big":  # equal, all 64 bits in use
         epoch = (1 << 63) - 3
-    g = coordinated(local, epoch)
+    g = coordinated(local, epoch, keep=img if scenario == "fail_keep" else None)
     q.put((rank, g.committed, g.failures, g.n_buffers, g.total_bytes, g.epochs_agree, img.freed, g.image is None))
     dist.destroy_process_group()
 
@@ -88,3 +88,10 @@ def test_epoch_agreement_exact_in_every_16_bit_part():
         assert not ok and not same and none
     for rank, ok, f, nb, tb, same, freed, none in _run(3, "epoch_big"):
         assert ok and same and not none
+
+
+def test_abort_keeps_caller_owned_reused_image():
+    """An image passed for reuse (checl_checkpoint_into) stays the caller's on abort:
+    not freed, not returned, committed = False."""
+    for rank, ok, f, nb, tb, same, freed, none in _run(2, "fail_keep"):
+        assert not ok and f == 1 and none and not freed
