@@ -177,7 +177,18 @@ def cpu_baseline(w, max_seconds: float = 20.0):
     sample = (f"{len(picked)}/{len(w.buffers)} buffers of {w.name} ({acc} of {total} B), "
               f"oracle checkpoint+restore, median of {len(times)}")
     return {"value": acc / t / 1e9, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample,
-            "ms_per_roundtrip": t * 1e3}
+            "ms_per_roundtrip": t * 1e3, "cpu_model": cpu_model()}
+
+
+def cpu_model() -> str:
+    """The host CPU's model name (/proc/cpuinfo), recorded beside the oracle's timing."""
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    return "unknown"
 
 
 def run_reference(a):
@@ -212,7 +223,8 @@ def run_reference(a):
         "warmup": a.warmup, "ms_per_step": dt / a.steps * 1e3, "higher_is_better": True, "scaling": "weak",
         "vs_baseline": None, "dtype": "u8", "data": "synthetic",
         "config": {"workload": w.name, "payload_bytes_per_gpu": w.total_bytes, "n_buffers": len(w.buffers)},
-        "cpu_baseline": {"value": value, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample},
+        "cpu_baseline": {"value": value, "unit": "GB/s", "cores": 1, "kind": "oracle", "sample": sample,
+                         "cpu_model": cpu_model()},
         "e2e": {"value": value, "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }))
 
