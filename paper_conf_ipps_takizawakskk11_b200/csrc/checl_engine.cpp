@@ -36,7 +36,7 @@ size_t snapshot_smem_bytes();
 cudaError_t snapshot_configure();
 cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream_t s, int kernel, uint64_t rounds);
 cudaError_t snapshot_launch_config(int op, const LaunchParams& p, int n_sms, int kernel, uint64_t rounds,
-                                   const void** fn, unsigned* ctas, size_t* smem);
+                                   const void** fn, unsigned* ctas, size_t* smem, unsigned* cluster);
 cudaError_t launch_build_tables(const TableParams& tp, uint32_t* out, cudaStream_t s);
 cudaError_t launch_fill(uint8_t* ptr, uint64_t bytes, uint64_t key, int kind, int n_sms, cudaStream_t s);
 cudaError_t launch_compare(const uint8_t* a, const uint8_t* b, uint64_t bytes, unsigned long long* n_diff, int n_sms,
@@ -1037,10 +1037,11 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
     return !e || std::atoi(e) != 0;
   }();
   const void* fn = nullptr;
-  unsigned ctas = 0;
+  unsigned ctas = 0, cluster = 1;
   size_t smem = 0;
   if (use_graph)
-    ck(snapshot_launch_config(op, p, ds.n_sms, kernel, chunks * (kChunkBytes / kRoundBytes), &fn, &ctas, &smem));
+    ck(snapshot_launch_config(op, p, ds.n_sms, kernel, chunks * (kChunkBytes / kRoundBytes), &fn, &ctas, &smem,
+                              &cluster));
   double h1 = 0, h2 = 0;
   if (fn) {
     LaunchGraph* g = nullptr;
@@ -1061,6 +1062,14 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
       cudaGraph_t gr = n.graph;
       gck("cudaGraphAddEventRecordNode", cudaGraphAddEventRecordNode(&n.ev_a, gr, nullptr, 0, a));
       gck("cudaGraphAddKernelNode", cudaGraphAddKernelNode(&n.kern, gr, &n.ev_a, 1, &kp));
+      if (cluster > 1) {  // kernel 4 as 2-CTA clusters (multicast table prologue)
+        cudaKernelNodeAttrValue v = {};
+        v.clusterDim.x = cluster;
+        v.clusterDim.y = 1;
+        v.clusterDim.z = 1;
+        gck("cudaGraphKernelNodeSetAttribute",
+            cudaGraphKernelNodeSetAttribute(n.kern, cudaLaunchAttributeClusterDimension, &v));
+      }
       gck("cudaGraphAddEventRecordNode", cudaGraphAddEventRecordNode(&n.ev_b, gr, &n.kern, 1, b));
       const cudaError_t e = cudaGraphInstantiate(&n.exec, gr, 0);
       if (e != cudaSuccess) cudaGraphDestroy(gr);

@@ -25,6 +25,8 @@
 // multiply by x^(-8 zp). The next round's loads are issued before the current
 // round's CRC so that HBM latency hides under the table lookups.
 // DESIGN.md §5 derives the resource budget and the GF(2) identities.
+#include <cstdlib>
+
 #include <cuda_runtime.h>
 
 #include "checl_internal.h"
@@ -676,7 +678,51 @@ __device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.w
 __device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 
-template <int kOp>
+__device__ __forceinline__ void cluster_sync() {
+  asm volatile("barrier.cluster.arrive.release.aligned;\nbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+
+// Table prologue of a 2-CTA cluster (kernel 4, CHECL_TABLE_MC): the table image is
+// cut into 32 KiB pieces and each CTA issues every other piece as one bulk copy
+// multicast to both CTAs (same shared offset in each), so L2 serves each table byte
+// once per SM pair instead of once per SM. Each CTA's table mbarrier expects all the
+// bytes; the cluster barrier orders both CTAs' barrier initialisations before any
+// multicast can complete on them (and synchronises the CTA like load_tables).
+template <int N>
+__device__ __forceinline__ void load_tables_mc(uint8_t* smem, const uint32_t* gtab, const TableCopy (&cp)[N],
+                                               uint64_t* mbar) {
+  const uint32_t mb = smem_addr(mbar);
+  uint32_t rank;
+  asm("mov.u32 %0, %%cluster_ctarank;" : "=r"(rank));
+  if (threadIdx.x == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mb) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  cluster_sync();
+  if (threadIdx.x == 0) {
+    uint32_t total = 0;
+#pragma unroll
+    for (int i = 0; i < N; ++i) total += cp[i].bytes;
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mb), "r"(total) : "memory");
+    const uint16_t both = 0x3;
+    uint32_t k = 0;
+#pragma unroll
+    for (int i = 0; i < N; ++i) {
+      for (uint32_t o = 0; o < cp[i].bytes; o += 32768u, ++k) {
+        if ((k & 1u) != rank) continue;
+        const uint32_t n = cp[i].bytes - o < 32768u ? cp[i].bytes - o : 32768u;
+        asm volatile(
+            "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1], %2, [%3], "
+            "%4;" ::"r"(smem_addr(smem + cp[i].dst_off + o)),
+            "l"(reinterpret_cast<const uint8_t*>(gtab + cp[i].src_word) + o), "r"(n), "r"(mb), "h"(both)
+            : "memory");
+      }
+    }
+  }
+}
+
+// kMc: launched as 2-CTA clusters; the table prologue is multicast (load_tables_mc)
+template <int kOp, bool kMc>
 __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchParams p) {
   using O = OpT<kOp>;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -687,7 +733,10 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
   {  // (load_tables fences the barrier initialisations and synchronises the CTA)
     const TableCopy cp[2] = {{(uint32_t)kTmaColOff, (uint32_t)kColOff, (uint32_t)(kColWords + kColFoldWords) * 4u},
                              {(uint32_t)kTmaUnitOff, (uint32_t)kUnitOff, (uint32_t)kUnitWords * 4u}};
-    load_tables<2, false>(smem, p.tables, cp, mbars + kWarpsPerCta * kTmaTiles);
+    if constexpr (kMc)
+      load_tables_mc<2>(smem, p.tables, cp, mbars + kWarpsPerCta * kTmaTiles);
+    else
+      load_tables<2, false>(smem, p.tables, cp, mbars + kWarpsPerCta * kTmaTiles);
   }
   bool tables_ready = false;
   const uint8_t* tb = smem + kTmaColOff;
@@ -877,6 +926,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
   if (!tables_ready) wait_tables(mbars + kWarpsPerCta * kTmaTiles);
   if (lane == 0) bulk_wait_all();  // the bulk stores have landed before the kernel ends
   release_work(p);
+  if constexpr (kMc) cluster_sync();  // neither CTA exits while a multicast it issued is in flight
   warp_trace(p, 0, t_start);
   warp_trace(p, 2, gtimer());
   {
@@ -1270,8 +1320,38 @@ static cudaError_t configure_op() {
     e = cudaFuncSetAttribute(balanced_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kBalSmemBytes);
   if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck)
     if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(tma_kernel<kOp>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmemBytes);
+      e = cudaFuncSetAttribute(tma_kernel<kOp, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmemBytes);
+  if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck)
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(tma_kernel<kOp, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmemBytes);
   return e;
+}
+
+// Kernel 4 as 2-CTA clusters with the multicast table prologue: CHECL_TABLE_MC=1
+// asks for it; used only if every SM can hold a CTA of a co-resident cluster.
+static bool g_table_mc = false;
+
+static bool table_mc_possible() {
+  int dev = 0, n_sms = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || cudaDeviceGetAttribute(&n_sms, cudaDevAttrMultiProcessorCount, dev))
+    return false;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(n_sms & ~1));
+  cfg.blockDim = dim3(kThreadsPerCta);
+  cfg.dynamicSmemBytes = kTmaSmemBytes;
+  cudaLaunchAttribute at[1];
+  at[0].id = cudaLaunchAttributeClusterDimension;
+  at[0].val.clusterDim.x = 2;
+  at[0].val.clusterDim.y = 1;
+  at[0].val.clusterDim.z = 1;
+  cfg.attrs = at;
+  cfg.numAttrs = 1;
+  int n = 0;
+  if (cudaOccupancyMaxActiveClusters(&n, tma_kernel<kOpPack, true>, &cfg) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return 2 * n >= (n_sms & ~1);
 }
 
 cudaError_t snapshot_configure() {
@@ -1281,6 +1361,10 @@ cudaError_t snapshot_configure() {
   if (e == cudaSuccess) e = configure_op<kOpCheck>();
   if (e == cudaSuccess) e = configure_op<kOpCopy>();
   if (e == cudaSuccess) e = configure_op<kOpScatter>();
+  if (e == cudaSuccess) {
+    const char* m = std::getenv("CHECL_TABLE_MC");
+    g_table_mc = m && std::atoi(m) != 0 && table_mc_possible();
+  }
   return e;
 }
 
@@ -1293,7 +1377,23 @@ template <int kOp>
 static void launch_op(const LaunchParams& p, unsigned ctas, cudaStream_t s, int kernel) {
   if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck) {
     if (kernel == 4) {
-      tma_kernel<kOp><<<ctas, kThreadsPerCta, kTmaSmemBytes, s>>>(p);
+      if (!g_table_mc) {
+        tma_kernel<kOp, false><<<ctas, kThreadsPerCta, kTmaSmemBytes, s>>>(p);
+        return;
+      }
+      cudaLaunchConfig_t cfg = {};
+      cfg.gridDim = dim3(ctas);
+      cfg.blockDim = dim3(kThreadsPerCta);
+      cfg.dynamicSmemBytes = kTmaSmemBytes;
+      cfg.stream = s;
+      cudaLaunchAttribute at[1];
+      at[0].id = cudaLaunchAttributeClusterDimension;
+      at[0].val.clusterDim.x = 2;
+      at[0].val.clusterDim.y = 1;
+      at[0].val.clusterDim.z = 1;
+      cfg.attrs = at;
+      cfg.numAttrs = 1;
+      cudaLaunchKernelEx(&cfg, tma_kernel<kOp, true>, p);
       return;
     }
   }
@@ -1310,7 +1410,8 @@ static const void* op_fn(int kernel, size_t* smem) {
   if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck) {
     if (kernel == 4) {
       *smem = kTmaSmemBytes;
-      return reinterpret_cast<const void*>(tma_kernel<kOp>);
+      return g_table_mc ? reinterpret_cast<const void*>(tma_kernel<kOp, true>)
+                        : reinterpret_cast<const void*>(tma_kernel<kOp, false>);
     }
   }
   if (kernel == 3 || kernel == 4) {
@@ -1325,15 +1426,18 @@ static const void* op_fn(int kernel, size_t* smem) {
 static uint64_t snapshot_ctas(const LaunchParams& p, int n_sms, int kernel, uint64_t rounds) {
   const uint64_t chunks = p.c1 - p.c0;
   const uint64_t units = kernel >= 3 ? rounds : kernel == 2 ? chunks * 16 : chunks;
-  const uint64_t ctas = (units + kWarpsPerCta - 1) / kWarpsPerCta;
-  return ctas > (uint64_t)n_sms ? (uint64_t)n_sms : ctas;
+  uint64_t ctas = (units + kWarpsPerCta - 1) / kWarpsPerCta;
+  ctas = ctas > (uint64_t)n_sms ? (uint64_t)n_sms : ctas;
+  if (kernel == 4 && g_table_mc) ctas = ctas < 2 ? 2 : ctas & ~1ull;  // whole 2-CTA clusters
+  return ctas;
 }
 
 // The kernel, grid and dynamic shared memory launch_snapshot would use (for a
 // kernel node of a CUDA graph); *fn = nullptr when the launch has no chunks.
 cudaError_t snapshot_launch_config(int op, const LaunchParams& p, int n_sms, int kernel, uint64_t rounds,
-                                   const void** fn, unsigned* ctas, size_t* smem) {
+                                   const void** fn, unsigned* ctas, size_t* smem, unsigned* cluster) {
   *fn = nullptr;
+  *cluster = kernel == 4 && g_table_mc && (op == kOpPack || op == kOpVerify || op == kOpCrc || op == kOpCheck) ? 2 : 1;
   if (p.c1 == p.c0) return cudaSuccess;
   *ctas = (unsigned)snapshot_ctas(p, n_sms, kernel, rounds);
   switch (op) {
