@@ -795,8 +795,8 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
   bool have = g < g_end, fetched = false, nmore = false;
   if (have) {
     c = find_chunk(p, g, lane);
-  } else {  // no static rounds: straight to the dynamic blocks
-    fetched = true;
+  } else {  // no static rounds: straight to the dynamic blocks (the block taken here is
+            // the current stretch; its successor is fetched during its first round)
     have = next_block(p, sc, lane, g, g_end, c);
   }
   uint64_t ng = 0, nge = 0, nlo = 0;  // the next stretch (dynamic block), once fetched

@@ -61,12 +61,17 @@ print("kernel ok")
 """
 
 
-@pytest.mark.parametrize("kernel", ["1", "2", "3", "4", "4:0:1", "4:500:3", "4:900:16"])
+@pytest.mark.parametrize("kernel", ["1", "2", "3", "4", "4:0:1", "4:500:3", "4:900:16", "4:0:1:mc", "4:500:3:mc"])
 def test_forced_kernel_shapes_bit_exact(kernel):
     """kernel "4:S:B" = the TMA kernel with the dynamic tail forced on at this size:
-    static share S permille, dynamic blocks of B rounds (S = 0: every round dynamic)."""
+    static share S permille, dynamic blocks of B rounds (S = 0: every round dynamic;
+    with ":mc" the grid is rounded down to whole 2-CTA clusters, so the 3-chunk stages
+    have more blocks than warps: every warp must keep fetching)."""
     k, *dyn = kernel.split(":")
     env = dict(os.environ, CHECL_KERNEL=k)
+    if dyn and dyn[-1] == "mc":  # 2-CTA clusters with the multicast table prologue (even grids)
+        env.update(CHECL_TABLE_MC="1")
+        dyn = dyn[:-1]
     if dyn:
         env.update(CHECL_STATIC_PERMILLE=dyn[0], CHECL_DYN_BLOCK=dyn[1], CHECL_DYN_MIN_ROUNDS="0")
     r = subprocess.run([sys.executable, "-c", SCRIPT % ROOT], capture_output=True, text=True, env=env, cwd=ROOT,
