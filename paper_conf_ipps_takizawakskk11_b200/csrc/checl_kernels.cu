@@ -428,10 +428,21 @@ __device__ __forceinline__ Sched make_sched(const LaunchParams& p) {
   return s;
 }
 
-// The chunk holding round g: the last c in [c0, c1) with round_base[c] <= g, by a
-// 32-way search (one probe per lane: 3 dependent loads for C2, 4 for 1 M chunks).
-__device__ __forceinline__ uint64_t find_chunk(const LaunchParams& p, uint64_t g, int lane) {
-  uint64_t lo = p.c0, hi = p.c1;  // invariant: round_base[lo] <= g, answer in [lo, hi)
+// The chunk holding round g: the last c in [c0, c1) with round_base[c] <= g. A chunk
+// has at most 16 rounds, so round_base[c] <= R0 + 16 (c - c0) and the answer is at
+// least c0 + (g - R0) / 16: the first probe reads the 32 chunks from there (one
+// coalesced load), which settles it whenever fewer than ~31 short chunks precede g
+// (C2, C4: one dependent load instead of three or four); otherwise a 32-way search
+// (one probe per lane) continues above them.
+__device__ __forceinline__ uint64_t find_chunk(const LaunchParams& p, uint64_t g, uint64_t R0, int lane) {
+  constexpr uint64_t kRoundsPerChunk = kChunkBytes / kRoundBytes;
+  uint64_t lo = p.c0 + (g - R0) / kRoundsPerChunk, hi = p.c1;  // invariant: round_base[lo] <= g, answer in [lo, hi)
+  {
+    const uint64_t idx = lo + (uint64_t)lane;
+    const unsigned m = __ballot_sync(0xFFFFFFFFu, idx < hi && p.round_base[idx] <= g);
+    if (m != 0xFFFFFFFFu) return lo + (uint64_t)(31 - __clz(m));
+    lo += 31;
+  }
   while (hi - lo > 1) {
     const uint64_t step = (hi - lo + 31) / 32, idx = lo + lane * step;
     const unsigned m = __ballot_sync(0xFFFFFFFFu, idx < hi && p.round_base[idx] <= g);
@@ -451,7 +462,7 @@ __device__ __forceinline__ bool next_block(const LaunchParams& p, const Sched& s
   if (b >= s.nblk) return false;
   g = s.R0 + s.Rs + b * s.B;
   ge = g + s.B < s.R0 + s.R ? g + s.B : s.R0 + s.R;
-  c = find_chunk(p, g, lane);
+  c = find_chunk(p, g, s.R0, lane);
   return true;
 }
 
@@ -516,7 +527,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
   const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta, wid = (uint64_t)blockIdx.x * kWarpsPerCta + warp;
   const Sched sc = make_sched(p);
   uint64_t g = sc.R0 + sc.Rs * wid / nw, g_end = sc.R0 + sc.Rs * (wid + 1) / nw;
-  uint64_t lo = g < g_end ? find_chunk(p, g, lane) : p.c0;
+  uint64_t lo = g < g_end ? find_chunk(p, g, sc.R0, lane) : p.c0;
   for (bool more = true; more;) {
   // the next dynamic block is fetched (and its chunk found) while the first loads of
   // this stretch are in flight
@@ -794,7 +805,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
   uint64_t g = sc.R0 + sc.Rs * wid / nw, g_end = sc.R0 + sc.Rs * (wid + 1) / nw, c = 0;
   bool have = g < g_end, fetched = false, nmore = false;
   if (have) {
-    c = find_chunk(p, g, lane);
+    c = find_chunk(p, g, sc.R0, lane);
   } else {  // no static rounds: straight to the dynamic blocks (the block taken here is
             // the current stretch; its successor is fetched during its first round)
     have = next_block(p, sc, lane, g, g_end, c);
@@ -806,6 +817,9 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
     cur = open_part(c, p.round_base[c], p.desc[c], g, g_end);
     issue(cur, cur.r0, t);
   }
+#ifdef CHECL_TRACE_SETUP  // experiment: slot 1 = first round issued (schedule set up)
+  warp_trace(p, 1, gtimer());
+#endif
   // (the tables are waited for just before the first CRC: by then the first two rounds
   // are in flight)
   while (have) {
@@ -873,7 +887,9 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
       if (!tables_ready) {
         wait_tables(mbars + kWarpsPerCta * kTmaTiles);
         tables_ready = true;
+#ifndef CHECL_TRACE_SETUP
         warp_trace(p, 1, gtimer());
+#endif
       }
       if (bulk) {
         mbar_wait(mb_sa + t * 8, (phase >> t) & 1u);
