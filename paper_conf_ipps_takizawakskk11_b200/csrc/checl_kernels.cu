@@ -416,6 +416,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
 struct Sched {
   uint64_t R0, R, Rs, nblk;
   uint32_t B;
+  bool near;  // few short chunks: find_chunk's first probe settles every search
 };
 
 __device__ __forceinline__ Sched make_sched(const LaunchParams& p) {
@@ -425,19 +426,24 @@ __device__ __forceinline__ Sched make_sched(const LaunchParams& p) {
   s.B = p.dyn_block ? p.dyn_block : 1u;
   s.Rs = p.work ? s.R * p.static_permille / 1000u : s.R;
   s.nblk = (s.R - s.Rs + s.B - 1) / s.B;
+  // rounds missing against 16 per chunk; below 16 * 30 the chunk holding any round is
+  // within 31 chunks of find_chunk's lower bound
+  s.near = (p.c1 - p.c0) * (kChunkBytes / kRoundBytes) - s.R < 16 * 30;
   return s;
 }
 
 // The chunk holding round g: the last c in [c0, c1) with round_base[c] <= g. A chunk
 // has at most 16 rounds, so round_base[c] <= R0 + 16 (c - c0) and the answer is at
-// least c0 + (g - R0) / 16: the first probe reads the 32 chunks from there (one
-// coalesced load), which settles it whenever fewer than ~31 short chunks precede g
-// (C2, C4: one dependent load instead of three or four); otherwise a 32-way search
-// (one probe per lane) continues above them.
-__device__ __forceinline__ uint64_t find_chunk(const LaunchParams& p, uint64_t g, uint64_t R0, int lane) {
+// least lo = c0 + (g - R0) / 16, and at most ~(missing rounds) / 16 chunks above it.
+// With few short chunks (s.near: C1, C2, C4) one coalesced probe of the 32 chunks from
+// lo settles it (one dependent load instead of three or four); otherwise a 32-way
+// search over [c0, c1) (one probe per lane; with 10 000 short chunks the first probe
+// would only add a load: C3 measured 8-12 us slower with it).
+__device__ __forceinline__ uint64_t find_chunk(const LaunchParams& p, uint64_t g, const Sched& s, int lane) {
   constexpr uint64_t kRoundsPerChunk = kChunkBytes / kRoundBytes;
-  uint64_t lo = p.c0 + (g - R0) / kRoundsPerChunk, hi = p.c1;  // invariant: round_base[lo] <= g, answer in [lo, hi)
-  {
+  uint64_t lo = p.c0, hi = p.c1;  // invariant: round_base[lo] <= g, answer in [lo, hi)
+  if (s.near) {
+    lo += (g - s.R0) / kRoundsPerChunk;
     const uint64_t idx = lo + (uint64_t)lane;
     const unsigned m = __ballot_sync(0xFFFFFFFFu, idx < hi && p.round_base[idx] <= g);
     if (m != 0xFFFFFFFFu) return lo + (uint64_t)(31 - __clz(m));
@@ -462,7 +468,7 @@ __device__ __forceinline__ bool next_block(const LaunchParams& p, const Sched& s
   if (b >= s.nblk) return false;
   g = s.R0 + s.Rs + b * s.B;
   ge = g + s.B < s.R0 + s.R ? g + s.B : s.R0 + s.R;
-  c = find_chunk(p, g, s.R0, lane);
+  c = find_chunk(p, g, s, lane);
   return true;
 }
 
@@ -527,7 +533,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
   const uint64_t nw = (uint64_t)gridDim.x * kWarpsPerCta, wid = (uint64_t)blockIdx.x * kWarpsPerCta + warp;
   const Sched sc = make_sched(p);
   uint64_t g = sc.R0 + sc.Rs * wid / nw, g_end = sc.R0 + sc.Rs * (wid + 1) / nw;
-  uint64_t lo = g < g_end ? find_chunk(p, g, sc.R0, lane) : p.c0;
+  uint64_t lo = g < g_end ? find_chunk(p, g, sc, lane) : p.c0;
   for (bool more = true; more;) {
   // the next dynamic block is fetched (and its chunk found) while the first loads of
   // this stretch are in flight
@@ -805,7 +811,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
   uint64_t g = sc.R0 + sc.Rs * wid / nw, g_end = sc.R0 + sc.Rs * (wid + 1) / nw, c = 0;
   bool have = g < g_end, fetched = false, nmore = false;
   if (have) {
-    c = find_chunk(p, g, sc.R0, lane);
+    c = find_chunk(p, g, sc, lane);
   } else {  // no static rounds: straight to the dynamic blocks (the block taken here is
             // the current stretch; its successor is fetched during its first round)
     have = next_block(p, sc, lane, g, g_end, c);
