@@ -490,11 +490,14 @@ def main():
     # buffer written between steps, outside the timed spans)
     flush = torch.empty(2 * L2_BYTES, dtype=torch.uint8, device=dev) if S <= L2_BYTES else None
 
-    def run(img, steps, collect):
-        """steps x (checkpoint_into img -> coordinate -> restore img); returns device ms."""
+    def run(img, steps, collect: bool):
+        """steps x (checkpoint_into img -> coordinate -> restore img); returns device ms
+        and, with collect, the library's cumulative per-call timing of those steps
+        (checl_stats: kernel spans from its CUDA events, read after the timed region)."""
         cur = torch.cuda.current_stream(dev)
         total = 0.0
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        ctx.reset_stats()
         if flush is None:
             e0.record(cur)
         for i in range(steps):
@@ -502,15 +505,11 @@ def main():
                 flush.fill_(i & 0xFF)
                 e0.record(cur)
             ctx.checkpoint(dev, epoch=i + 1, into=img)
-            tc = ctx.last_timing(raw=True)
             coordinate(True, i + 1)
             if restart:
                 for h in handles:
                     ctx.release(h)
             ctx.restore(img, dev, report=False)
-            tr = ctx.last_timing(raw=True)
-            if collect is not None:
-                collect.append((tc, tr))
             if flush is not None:
                 e1.record(cur)
                 e1.synchronize()
@@ -519,7 +518,21 @@ def main():
             e1.record(cur)
             e1.synchronize()
             total = e0.elapsed_time(e1)
-        return total
+        if not collect:
+            return total, None
+        st = (ctx.stats(checl.STATS_CHECKPOINT), ctx.stats(checl.STATS_RESTORE))
+        assert st[0]["n_calls"] == steps and st[1]["n_calls"] == steps
+        return total, st
+
+    def detail(img):
+        """One more (untimed) step: the per-phase timing of a checkpoint and a restore."""
+        ctx.checkpoint(dev, epoch=a.steps + 1, into=img)
+        tc = ctx.last_timing()
+        if restart:
+            for h in handles:
+                ctx.release(h)
+        ctx.restore(img, dev, report=False)
+        return tc, ctx.last_timing()
 
     # -- value: device-resident image (HBM) --------------------------------------
     dimg = ctx.checkpoint_device(dev, epoch=0)
@@ -533,13 +546,12 @@ def main():
         del tensors[:], t  # the user's buffers are gone (t: the fill loop's last one); only the image survives
         torch.cuda.empty_cache()
         ctx.restore(dimg, dev, report=False)
-    run(dimg, a.warmup, None)
-    phases = []
+    run(dimg, a.warmup, False)
     barrier()
     with ClockSampler(dev) as clk:
-        ms = run(dimg, a.steps, phases)
+        ms, (sck, srs) = run(dimg, a.steps, True)
     barrier()
-    phases = [(checl.timing_dict(c), checl.timing_dict(r)) for c, r in phases]
+    last_ck, last_rs = detail(dimg)
     ms_max = max_over_ranks(ms)
     value = sum_over_ranks(S * a.steps) / (ms_max * 1e-3) / 1e9
     # correctness of the last restore: every handle's new buffer == the application's bytes
@@ -554,11 +566,11 @@ def main():
         hd = dimg.header()
         n_diff += int(not (dimg.view()[hd["crc_off"]:hd["crc_off"] + 4 * n_chunks] == crc0).all())
         n_diff += restart_samples_bad(ctx, handles, w, a.kind)
-    pack_ms = statistics.mean(p[0]["kernel_ms"] for p in phases)
-    verify_ms = statistics.mean(p[1]["kernel_ms"] for p in phases)
-    ck_ms = statistics.mean(p[0]["total_ms"] for p in phases)
-    rs_ms = statistics.mean(p[1]["total_ms"] for p in phases)
-    launches = sum(p[0]["n_kernels"] + p[1]["n_kernels"] for p in phases)
+    pack_ms = sck["kernel_ms"] / sck["n_calls"]
+    verify_ms = srs["kernel_ms"] / srs["n_calls"]
+    ck_ms = sck["total_ms"] / sck["n_calls"]
+    rs_ms = srs["total_ms"] / srs["n_calls"]
+    launches = sck["n_kernels"] + srs["n_kernels"]
     pk = peaks()
     hbm_peak = pk.get("hbm_gbs")
     peak_src = "MEASURED_PEAKS.json hbm_gbs (measured copy)" if hbm_peak else "fallback 6650 GB/s (B200_PROFILING.md)"
@@ -582,18 +594,16 @@ def main():
         pcie = pcie_probe(dev)
         himg = ctx.checkpoint(dev, epoch=0)
         payload_span = himg.info()["image_bytes"]
-        run(himg, a.warmup, None)
-        ph2 = []
+        run(himg, a.warmup, False)
         barrier()
-        ms2 = run(himg, a.steps, ph2)
-        ph2 = [(checl.timing_dict(c), checl.timing_dict(r)) for c, r in ph2]
+        ms2, (eck, ers) = run(himg, a.steps, True)
         barrier()
         ms2_max = max_over_ranks(ms2)
         E = sum_over_ranks(S * a.steps) / (ms2_max * 1e-3) / 1e9
-        ck2 = statistics.mean(p[0]["total_ms"] for p in ph2)
-        rs2 = statistics.mean(p[1]["total_ms"] for p in ph2)
-        drain = statistics.mean(p[0]["copy_ms"] for p in ph2)
-        fill = statistics.mean(p[1]["copy_ms"] for p in ph2)
+        ck2 = eck["total_ms"] / eck["n_calls"]
+        rs2 = ers["total_ms"] / ers["n_calls"]
+        drain = eck["copy_ms"] / eck["n_calls"]
+        fill = ers["copy_ms"] / ers["n_calls"]
         himg.free()
         pay = S  # payload bytes carried each way (+ padding, tables below)
         e2e = {
@@ -606,7 +616,7 @@ def main():
             "pcie_measured_GBs": pcie,
             "drain_frac_of_pcie": (pay / (drain * 1e-3) / 1e9) / pcie["d2h"],
             "fill_frac_of_pcie": (pay / (fill * 1e-3) / 1e9) / pcie["h2d"],
-            "gpu_launches": sum(p[0]["n_kernels"] + p[1]["n_kernels"] for p in ph2),
+            "gpu_launches": eck["n_kernels"] + ers["n_kernels"],
             "image": "pinned host memory (cudaHostAlloc), reused across steps",
         }
 
@@ -635,7 +645,7 @@ def main():
             "phases": {"checkpoint_ms": ck_ms, "restore_ms": rs_ms, "checkpoint_GBs": S / (ck_ms * 1e-3) / 1e9,
                        "restore_GBs": S / (rs_ms * 1e-3) / 1e9,
                        "pack_GBs_2S": 2 * S / (pack_ms * 1e-3) / 1e9, "verify_GBs_2S": 2 * S / (verify_ms * 1e-3) / 1e9,
-                       "checkpoint_detail": phases[-1][0], "restore_detail": phases[-1][1]},
+                       "checkpoint_detail": last_ck, "restore_detail": last_rs},
             "verified": n_diff == 0,
             "gpu_launches": launches,
             "clocks": clk.summary(),

@@ -46,7 +46,7 @@ EXPORTS = (
     "checl_version", "checl_debug_fill", "checl_debug_compare", "checl_debug_corrupt",
     "checl_checkpoint_incremental", "checl_restore_chain", "checl_image_merge",
     "checl_request_checkpoint", "checl_checkpoint_pending", "checl_install_signal", "checl_sync_point",
-    "checl_image_write", "checl_image_read", "checl_trim",
+    "checl_image_write", "checl_image_read", "checl_trim", "checl_stats_get", "checl_stats_reset",
 )
 
 
@@ -65,6 +65,14 @@ class _Timing(C.Structure):
     _fields_ = [("sync_ms", C.c_double), ("plan_ms", C.c_double), ("alloc_ms", C.c_double),
                 ("kernel_ms", C.c_double), ("copy_ms", C.c_double), ("commit_ms", C.c_double),
                 ("total_ms", C.c_double), ("n_stages", C.c_uint64), ("n_kernels", C.c_uint64)]
+
+
+class _Stats(C.Structure):
+    _fields_ = [("n_calls", C.c_uint64), ("total_ms", C.c_double), ("kernel_ms", C.c_double),
+                ("copy_ms", C.c_double), ("n_kernels", C.c_uint64)]
+
+
+STATS_CHECKPOINT, STATS_RESTORE, STATS_INCREMENTAL, STATS_CHAIN = 0, 1, 2, 3
 
 
 def _load() -> C.CDLL:
@@ -93,6 +101,8 @@ def _load() -> C.CDLL:
         "checl_restore": [P, P, C.c_int, V, C.POINTER(_Report)],
         "checl_migrate": [P, C.c_int, C.c_int, V, C.POINTER(_Report)],
         "checl_last_timing": [P, C.POINTER(_Timing)],
+        "checl_stats_get": [P, C.c_int, C.POINTER(_Stats)],
+        "checl_stats_reset": [P],
         "checl_debug_fill": [C.c_int, V, SZ, U64, U64, C.c_int, V],
         "checl_debug_compare": [C.c_int, V, V, SZ, C.POINTER(U64)],
         "checl_debug_corrupt": [P, U64, C.c_uint8],
@@ -444,6 +454,19 @@ class Context:
         t = _Timing()
         _check(lib.checl_last_timing(self._p, C.byref(t)), "checl_last_timing")
         return t if raw else timing_dict(t)
+
+    def stats(self, kind: int) -> dict:
+        """Cumulative timing of one kind of call (STATS_*) since creation / reset_stats."""
+        t = _Stats()
+        _check(lib.checl_stats_get(self._p, kind, C.byref(t)), "checl_stats_get")
+        return _stats_dict(t)
+
+    def reset_stats(self):
+        _check(lib.checl_stats_reset(self._p), "checl_stats_reset")
+
+
+def _stats_dict(t) -> dict:
+    return {n: (float(getattr(t, n)) if ty is C.c_double else int(getattr(t, n))) for n, ty in _Stats._fields_}
 
 
 def timing_dict(t) -> dict:

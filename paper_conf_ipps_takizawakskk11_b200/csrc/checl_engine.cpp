@@ -269,21 +269,33 @@ struct LaunchGraph {
   cudaGraphNode_t ev_a = nullptr, kern = nullptr, ev_b = nullptr;
 };
 
+// Two halves used by alternate calls on a device: the event spans of a call stay
+// readable during the next call, which reads them while its own kernel runs
+// (deferred timing, see PendingTiming).
 struct EventPool {
-  std::vector<cudaEvent_t> ev;
+  std::vector<cudaEvent_t> ev[2];
   size_t used = 0;
+  int active = 0;
   cudaEvent_t get() {
-    if (used == ev.size()) {
+    std::vector<cudaEvent_t>& v = ev[active];
+    if (used == v.size()) {
       cudaEvent_t e;
       ck(cudaEventCreate(&e));
-      ev.push_back(e);
+      v.push_back(e);
     }
-    return ev[used++];
+    return v[used++];
   }
-  void reset() { used = 0; }
-  ~EventPool() {
-    for (auto e : ev) cudaEventDestroy(e);
+  void reset() {
+    active ^= 1;
+    used = 0;
   }
+  void destroy_all() {
+    for (auto& v : ev) {
+      for (auto e : v) cudaEventDestroy(e);
+      v.clear();
+    }
+  }
+  ~EventPool() { destroy_all(); }
 };
 
 template <typename T>
@@ -459,8 +471,7 @@ struct DevState {
       cudaGraphDestroy(g.graph);
     }
     graphs.clear();
-    for (auto e : events.ev) cudaEventDestroy(e);
-    events.ev.clear();
+    events.destroy_all();
     if (compute) cudaStreamDestroy(compute);
     if (copy) cudaStreamDestroy(copy);
     if (prev >= 0) cudaSetDevice(prev);
@@ -501,16 +512,8 @@ struct Entry {
 };
 
 // Phase-time events for checl_timing.
-struct KernelTimer {
+struct KernelTimer {  // the event pair around every timed launch of a call
   std::vector<std::pair<cudaEvent_t, cudaEvent_t>> spans;
-  double sum_ms() const {
-    double t = 0;
-    for (auto& s : spans) {
-      float ms = 0;
-      if (cudaEventElapsedTime(&ms, s.first, s.second) == cudaSuccess) t += ms;
-    }
-    return t;
-  }
 };
 
 }  // namespace
@@ -602,7 +605,23 @@ struct checl_ctx {
   DevState* devs[kMaxDevices] = {};
   size_t slot_bytes = kDefaultSlotBytes;
   uint32_t n_slots = 2;
-  checl_timing last{};
+  // timing of the last call; its CUDA-event spans are read lazily (PendingTiming)
+  mutable checl_timing last{};
+  // The last call's kernel / copy spans, not read yet: cudaEventElapsedTime costs
+  // ~3 us of host time per call on this pool (profiles/r01o/launch_cost_events.txt),
+  // so a call leaves its spans here and the next call reads them while its own kernel
+  // runs; checl_last_timing / checl_stats_get read them on demand.
+  struct PendingTiming {
+    bool on = false;
+    int kind = 0;
+    const EventPool* pool = nullptr;
+    int half = 0;
+    std::vector<std::pair<cudaEvent_t, cudaEvent_t>> spans;
+    cudaEvent_t c_begin = nullptr, c_end = nullptr;
+  };
+  mutable PendingTiming pend;
+  mutable checl_stats stats[CHECL_STATS_KINDS] = {};
+  mutable std::mutex tmu;
   checl_image* mig_img[kMaxDevices] = {};  // migration images, reused (HBM of the source)
   // the last allocation a commit released on each device, kept for the next restore
   // of (nearly) the same size: skips an allocator round trip per restore (a
@@ -1146,6 +1165,61 @@ void finalize_meta(uint8_t* host, const Plan& P, uint64_t epoch) {
   put_u32(host + 124, meta_crc(host, P.payload_off));
 }
 
+// -- deferred timing (checl_ctx::PendingTiming) -----------------------------------
+
+// Reads the pending spans of the last call into ctx->last and its statistics slot.
+void settle(const checl_ctx* ctx) {
+  std::lock_guard<std::mutex> lk(ctx->tmu);
+  auto& q = ctx->pend;
+  if (!q.on) return;
+  double k = 0;
+  for (auto& sp : q.spans) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, sp.first, sp.second) == cudaSuccess) k += ms;
+  }
+  float c = 0;
+  if (q.c_begin && cudaEventElapsedTime(&c, q.c_begin, q.c_end) != cudaSuccess) c = 0;
+  cudaGetLastError();
+  ctx->last.kernel_ms = k;
+  ctx->last.copy_ms = c;
+  ctx->stats[q.kind].kernel_ms += k;
+  ctx->stats[q.kind].copy_ms += c;
+  q.on = false;
+}
+
+// End of a call: its host-clock timing now, its event spans when next needed.
+void defer_timing(checl_ctx* ctx, const DevState& ds, const checl_timing& tm, const KernelTimer& kt,
+                  cudaEvent_t c_begin, cudaEvent_t c_end, int kind) {
+  settle(ctx);  // (normally done already, during this call's kernel)
+  std::lock_guard<std::mutex> lk(ctx->tmu);
+  ctx->last = tm;
+  ctx->last.kernel_ms = ctx->last.copy_ms = 0;
+  checl_stats& st = ctx->stats[kind];
+  st.n_calls++;
+  st.total_ms += tm.total_ms;
+  st.n_kernels += tm.n_kernels;
+  auto& q = ctx->pend;
+  q.on = true;
+  q.kind = kind;
+  q.pool = &ds.events;
+  q.half = ds.events.active;
+  q.spans = kt.spans;
+  q.c_begin = c_begin;
+  q.c_end = c_end;
+}
+
+// Start of a call on ds: switch its event pool to the other half, reading first the
+// pending spans if they live in that half.
+void begin_events(checl_ctx* ctx, DevState& ds) {
+  bool need = false;
+  {
+    std::lock_guard<std::mutex> lk(ctx->tmu);
+    need = ctx->pend.on && ctx->pend.pool == &ds.events && ctx->pend.half != ds.events.active;
+  }
+  if (need) settle(ctx);
+  ds.events.reset();
+}
+
 checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t epoch, checl_image* img,
                            bool to_device) {
   (void)stream;
@@ -1154,7 +1228,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
   const uint64_t aux0 = ds.aux_launches;
-  ds.events.reset();
+  begin_events(ctx, ds);
   KernelTimer kt;
   checl_timing tm{};
   tr("setup");
@@ -1227,6 +1301,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       c_begin = c_end = nullptr;  // nothing copied
     }
     tm.n_stages = 1;
+    settle(ctx);  // the previous call's spans, read while K1 runs
     ck(cudaStreamSynchronize(ds.compute));
     tr("wait");
   } else {
@@ -1300,6 +1375,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       ck(cudaMemcpyAsync(img->host_mut + P.crc_off, ds.crc_scratch.p, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.copy));
     ck(cudaEventRecord(c_end, ds.copy));
     tm.n_stages = P.stages.size();
+    settle(ctx);  // the previous call's spans, read while the pipeline runs
     ck(cudaStreamSynchronize(ds.copy));
   }
   // a5: header, manifest and meta CRC (the CRC table has landed)
@@ -1309,12 +1385,9 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
   tr("finalize");
   img->image_bytes = P.image_bytes;
   img->payload_off = P.payload_off;
-  float cms = 0;
-  if (c_begin && cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
-  tm.kernel_ms = kt.sum_ms();
   tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tm.total_ms = now_ms() - t0;
-  ctx->last = tm;
+  defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_CHECKPOINT);
   return CHECL_SUCCESS;
 }
 
@@ -1521,7 +1594,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
   const uint64_t aux0 = ds.aux_launches;
-  ds.events.reset();
+  begin_events(ctx, ds);
   KernelTimer kt;
   checl_timing tm{};
   if (rep) std::memset(rep, 0, sizeof(*rep)), rep->first_bad_chunk = ~0ull;
@@ -1656,20 +1729,19 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     ds.h_status.p[0] = ~0ull;
     ds.h_status.p[1] = 0;
   }
+  settle(ctx);  // the previous call's spans, read while K2 runs
   ck(cudaStreamSynchronize(ds.compute));
   ck(cudaStreamSynchronize(ds.copy));
   tr("wait");
   ds.status_clean = nch ? lp.status_host != nullptr : was_clean;
   const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
-  float cms = 0;
-  if (c_begin && cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
-  tm.kernel_ms = kt.sum_ms();
   tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tmp_payload.release();
   tmp_crc.release();
   if (rep) set_report(rep, P, n_bad, first_bad);
   if (n_bad) {
-    ctx->last = tm;
+    tm.total_ms = now_ms() - t0;
+    defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_RESTORE);
     return CHECL_ERR_CRC_MISMATCH;  // arena freed by its destructor; nothing rebound
   }
   // r5: rebind every handle (all-or-nothing)
@@ -1682,7 +1754,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   tr("adopt");
   tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
-  ctx->last = tm;
+  defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_RESTORE);
   return CHECL_SUCCESS;
 }
 
@@ -1711,7 +1783,7 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
     Plan& P0 = get_plan(ctx, ds, device);
     if (!same_layout(base->host, B, P0, device)) return do_checkpoint(ctx, device, stream, epoch, img, false);
   }
-  ds.events.reset();
+  begin_events(ctx, ds);
   KernelTimer kt;
   checl_timing tm{};
 
@@ -1828,12 +1900,9 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   tm.commit_ms = now_ms() - tf;
   img->image_bytes = image_bytes;
   img->payload_off = payload_off;
-  float cms = 0;
-  if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
-  tm.kernel_ms = kt.sum_ms();
   tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tm.total_ms = now_ms() - t0;
-  ctx->last = tm;
+  defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_INCREMENTAL);
   return CHECL_SUCCESS;
 }
 
@@ -1868,7 +1937,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
   const uint64_t aux0 = ds.aux_launches;
-  ds.events.reset();
+  begin_events(ctx, ds);
   KernelTimer kt;
   checl_timing tm{};
   const double ts = now_ms();
@@ -1999,21 +2068,19 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   ck(cudaStreamSynchronize(ds.copy));
   ds.status_clean = nch && lp.status_host;
   const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
-  float cms = 0;
-  if (cudaEventElapsedTime(&cms, c_begin, c_end) == cudaSuccess) tm.copy_ms = cms;
-  tm.kernel_ms = kt.sum_ms();
   tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tm.n_stages = dst.size() + 1;
   if (rep) set_report(rep, Z, n_bad, first_bad);
   if (n_bad) {
-    ctx->last = tm;
+    tm.total_ms = now_ms() - t0;
+    defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_CHAIN);
     return CHECL_ERR_CRC_MISMATCH;
   }
   const double tc = now_ms();
   commit(ctx, Z, device, arena);
   tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
-  ctx->last = tm;
+  defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_CHAIN);
   return CHECL_SUCCESS;
 }
 
@@ -2305,8 +2372,11 @@ checl_status checl_migrate(checl_ctx* ctx, int src_device, int dst_device, void*
     if (!ctx->mig_img[src_device]) ctx->mig_img[src_device] = new checl_image();
     checl_image& img = *ctx->mig_img[src_device];
     checl_status st = do_checkpoint(ctx, src_device, cuda_stream, 0, &img, true);
+    settle(ctx);
     checl_timing ck_t = ctx->last;
     if (st == CHECL_SUCCESS) st = do_restore(ctx, &img, dst_device, cuda_stream, rep, true);
+    settle(ctx);
+    std::lock_guard<std::mutex> lk(ctx->tmu);
     checl_timing& t = ctx->last;
     t.sync_ms += ck_t.sync_ms;
     t.plan_ms += ck_t.plan_ms;
@@ -2624,7 +2694,25 @@ checl_status checl_trim(checl_ctx* ctx) {
 
 checl_status checl_last_timing(const checl_ctx* ctx, checl_timing* out) {
   if (!ctx || !out) return CHECL_ERR_INVALID_VALUE;
+  settle(ctx);
+  std::lock_guard<std::mutex> lk(ctx->tmu);
   *out = ctx->last;
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_stats_get(const checl_ctx* ctx, int kind, checl_stats* out) {
+  if (!ctx || !out || kind < 0 || kind >= CHECL_STATS_KINDS) return CHECL_ERR_INVALID_VALUE;
+  settle(ctx);
+  std::lock_guard<std::mutex> lk(ctx->tmu);
+  *out = ctx->stats[kind];
+  return CHECL_SUCCESS;
+}
+
+checl_status checl_stats_reset(checl_ctx* ctx) {
+  if (!ctx) return CHECL_ERR_INVALID_VALUE;
+  settle(ctx);
+  std::lock_guard<std::mutex> lk(ctx->tmu);
+  for (auto& st : ctx->stats) st = checl_stats{};
   return CHECL_SUCCESS;
 }
 

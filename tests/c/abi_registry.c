@@ -60,6 +60,10 @@ int main(void) {
   CHECK(checl_image_free(NULL) == CHECL_SUCCESS);
   checl_timing t;
   CHECK(checl_last_timing(ctx, &t) == CHECL_SUCCESS);
+  checl_stats st;
+  CHECK(checl_stats_get(ctx, CHECL_STATS_RESTORE, &st) == CHECL_SUCCESS && st.n_calls == 0 && st.kernel_ms == 0.0);
+  CHECK(checl_stats_get(ctx, CHECL_STATS_KINDS, &st) == CHECL_ERR_INVALID_VALUE);
+  CHECK(checl_stats_reset(ctx) == CHECL_SUCCESS);
   CHECK(checl_destroy(ctx) == CHECL_SUCCESS);
   printf("abi_registry ok\n");
   return 0;

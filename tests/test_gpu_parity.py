@@ -276,6 +276,37 @@ def test_restart_loop_release_all_then_restore(ctx):
     assert ctx.count(DEV)[0] == 0
 
 
+def test_stats_accumulate_deferred_event_spans(ctx):
+    """Event spans are read lazily (next call / query): per-call timings and the
+    cumulative checl_stats agree, with or without a query after every call."""
+    make_set(ctx, [1 << 22, 12345, 0], seed=31)
+    img = ctx.checkpoint_device(DEV, epoch=1)
+    ctx.reset_stats()
+    ks, rs = [], []
+    for e in range(3):
+        ctx.checkpoint(DEV, epoch=e, into=img)
+        ks.append(ctx.last_timing())
+        ctx.restore(img, DEV)
+        rs.append(ctx.last_timing())
+    s0, s1 = ctx.stats(checl.STATS_CHECKPOINT), ctx.stats(checl.STATS_RESTORE)
+    assert s0["n_calls"] == 3 and s1["n_calls"] == 3
+    assert all(t["kernel_ms"] > 0 and t["n_kernels"] >= 1 for t in ks + rs)
+    assert s0["kernel_ms"] == pytest.approx(sum(t["kernel_ms"] for t in ks), rel=1e-12)
+    assert s1["kernel_ms"] == pytest.approx(sum(t["kernel_ms"] for t in rs), rel=1e-12)
+    assert s0["n_kernels"] == sum(t["n_kernels"] for t in ks)
+    ctx.reset_stats()
+    for e in range(4):  # no query in between: each call reads the previous call's spans
+        ctx.checkpoint(DEV, epoch=e, into=img)
+        ctx.restore(img, DEV)
+    last = ctx.last_timing()
+    s0, s1 = ctx.stats(checl.STATS_CHECKPOINT), ctx.stats(checl.STATS_RESTORE)
+    assert s0["n_calls"] == 4 and s1["n_calls"] == 4 and last["kernel_ms"] > 0
+    assert s0["kernel_ms"] > 0 and s1["kernel_ms"] >= last["kernel_ms"]
+    assert ctx.stats(checl.STATS_INCREMENTAL)["n_calls"] == 0
+    with pytest.raises(checl.CheclError):
+        ctx.stats(4)
+
+
 def test_checkpoint_into_reuses_and_grows(ctx):
     ds = make_set(ctx, [1000, 70000], seed=12)
     img = ctx.checkpoint(DEV, epoch=1)

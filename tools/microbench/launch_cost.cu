@@ -119,6 +119,15 @@ int main() {
         cudaEventElapsedTime(&ms, ea, eb);
         if (r >= 10) tot += ms, mn = ms < mn ? ms : mn, host += std::chrono::duration<double, std::micro>(t1 - t0).count();
       }
+      // host cost of reading the span back (cudaEventElapsedTime after completion)
+      {
+        auto q0 = std::chrono::steady_clock::now();
+        float x = 0;
+        for (int i = 0; i < 100; ++i) cudaEventElapsedTime(&x, mode == 1 ? a2 : a, mode == 1 ? b2 : b);
+        auto q1 = std::chrono::steady_clock::now();
+        printf("  cudaEventElapsedTime after mode %d: %.2f us/call\n", mode,
+               std::chrono::duration<double, std::micro>(q1 - q0).count() / 100);
+      }
       const char* name[] = {"graph [ev,k,ev]", "graph + node updates", "stream record/launch/record"};
       printf("%-28s span mean %.2f us  min %.2f us  host %.2f us/call\n", name[mode], tot / 30 * 1e3, mn * 1e3,
              host / 30);
