@@ -825,8 +825,10 @@ void chunk_span(const std::vector<BufRec>& bufs, size_t b, uint64_t j, uint64_t 
 
 bool bit_set(const uint8_t* map, uint64_t k) { return (map[k >> 3] >> (k & 7)) & 1u; }
 
-checl_status parse_image(const uint8_t* img, size_t len, bool meta_only, Parsed* out) {
+checl_status parse_image(const uint8_t* img, size_t len, bool meta_only, Parsed* out, bool check_meta_crc = true) {
   // meta_only: `len` covers [0, payload_off) only (device image mirror)
+  // check_meta_crc = false: the caller checks the meta CRC itself (do_restore, while
+  // its kernel runs); every structural check is made here
   if (!img || len < kHeaderBytes) return CHECL_ERR_BAD_IMAGE;
   if (std::memcmp(img, "CHECLIM1", 8) != 0) return CHECL_ERR_BAD_IMAGE;
   const uint32_t flags = get_u32(img + 84);
@@ -854,7 +856,7 @@ checl_status parse_image(const uint8_t* img, size_t len, bool meta_only, Parsed*
   uint64_t want;
   if (!add_ok(L.payload_off, L.payload_bytes, &want) || want != L.image_bytes) return CHECL_ERR_BAD_IMAGE;
   if ((uint64_t)len < (meta_only ? L.payload_off : L.image_bytes)) return CHECL_ERR_BAD_IMAGE;
-  if (get_u32(img + 124) != meta_crc(img, L.payload_off)) return CHECL_ERR_BAD_IMAGE;
+  if (check_meta_crc && get_u32(img + 124) != meta_crc(img, L.payload_off)) return CHECL_ERR_BAD_IMAGE;
   for (uint64_t i = L.crc_off + 4 * nch + map_bytes; i < L.payload_off; ++i)
     if (img[i]) return CHECL_ERR_BAD_IMAGE;
   const int device = (int32_t)get_u32(img + 80);
@@ -1605,11 +1607,14 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   tm.sync_ms = now_ms() - ts;
   tr("sync");
 
-  // r1: validate header + manifest (+ meta CRC over the CRC table)
+  // r1: validate header + manifest here; the meta CRC (over header, manifest and CRC
+  // table) is checked while K2 runs, and decides before anything is rebound: every
+  // structural check has passed, so K2 only reads inside the image and writes inside
+  // the new allocation, which an invalid image leaves unbound and frees
   const double tp = now_ms();
   Parsed P;
   const bool dev_img = img->location == CHECL_IMAGE_DEVICE;
-  checl_status st = parse_image(img->host, dev_img ? img->payload_off : img->image_bytes, dev_img, &P);
+  checl_status st = parse_image(img->host, dev_img ? img->payload_off : img->image_bytes, dev_img, &P, false);
   if (st) return st;
   if (P.flags != 0) return CHECL_ERR_BAD_IMAGE;  // a delta restores only as part of a chain
   if (rep) set_report(rep, P, 0, 0);
@@ -1618,7 +1623,9 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   // r2: re-create the buffers: one allocation laid out like the payload
   const double ta = now_ms();
   auto arena = new_arena(ctx, device, stream, P.L.payload_bytes);
-  if (!arena) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
+  if (!arena)  // (an invalid image still reports BAD_IMAGE first)
+    return get_u32(img->host + 124) == meta_crc(img->host, P.L.payload_off) ? CHECL_ERR_OUT_OF_DEVICE_MEMORY
+                                                                           : CHECL_ERR_BAD_IMAGE;
   tm.alloc_ms = now_ms() - ta;
   tr("alloc");
   const uint64_t nch = P.L.n_chunks;
@@ -1729,6 +1736,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     ds.h_status.p[0] = ~0ull;
     ds.h_status.p[1] = 0;
   }
+  const bool meta_ok = get_u32(img->host + 124) == meta_crc(img->host, P.L.payload_off);  // r1, under K2
   settle(ctx);  // the previous call's spans, read while K2 runs
   ck(cudaStreamSynchronize(ds.compute));
   ck(cudaStreamSynchronize(ds.copy));
@@ -1738,6 +1746,12 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
   tmp_payload.release();
   tmp_crc.release();
+  if (!meta_ok) {  // as if validation had failed first: no report, nothing rebound
+    if (rep) std::memset(rep, 0, sizeof(*rep)), rep->first_bad_chunk = ~0ull;
+    tm.total_ms = now_ms() - t0;
+    defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_RESTORE);
+    return CHECL_ERR_BAD_IMAGE;
+  }
   if (rep) set_report(rep, P, n_bad, first_bad);
   if (n_bad) {
     tm.total_ms = now_ms() - t0;
