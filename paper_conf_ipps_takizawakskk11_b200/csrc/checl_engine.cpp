@@ -1609,11 +1609,9 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   checl_timing tm{};
   if (rep) std::memset(rep, 0, sizeof(*rep)), rep->first_bad_chunk = ~0ull;
 
-  // quiesce the target (its old buffers may be freed at commit)
-  const double ts = now_ms();
-  ck(cudaDeviceSynchronize());
-  tm.sync_ms = now_ms() - ts;
-  tr("sync");
+  // (the target is quiesced before anything is rebound — its old buffers may be
+  // freed at commit — by the device-wide wait for K2 below; nothing before it touches
+  // memory the application may still be using: tm.sync_ms stays 0)
 
   // r1: validate header + manifest here; the meta CRC (over header, manifest and CRC
   // table) is checked while K2 runs, and decides before anything is rebound: every
@@ -1746,8 +1744,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   }
   const bool meta_ok = get_u32(img->host + 124) == meta_crc(img->host, P.L.payload_off);  // r1, under K2
   settle(ctx);  // the previous call's spans, read while K2 runs
-  ck(cudaStreamSynchronize(ds.compute));
-  ck(cudaStreamSynchronize(ds.copy));
+  ck(cudaDeviceSynchronize());  // K2, the copies, and every queue of the target (quiesce, L16)
   tr("wait");
   ds.status_clean = nch ? lp.status_host != nullptr : was_clean;
   const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
