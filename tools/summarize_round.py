@@ -5,6 +5,7 @@ import csv
 import io
 import json
 import os
+import re
 import shutil
 import sys
 from collections import defaultdict
@@ -51,8 +52,11 @@ if os.path.exists(rep):
         lines.append("")
         rd = float(d["dram__bytes_read.sum"][0]) * (1e6 if "Mbyte" in d["dram__bytes_read.sum"][1] else 1e9 if "Gbyte" in d["dram__bytes_read.sum"][1] else 1)
         wr = float(d["dram__bytes_write.sum"][0]) * (1e6 if "Mbyte" in d["dram__bytes_write.sum"][1] else 1e9 if "Gbyte" in d["dram__bytes_write.sum"][1] else 1)
-        key = "K2" if "<1>" in name or "(bool)1" in name else "K1"
-        traffic[key] = rd + wr
+        # first template argument = the kOp (checl_internal.h): 0 pack (K1), 1 verify (K2)
+        m = re.search(r"<\s*(\d+)", name)
+        op = int(m.group(1)) if m else -1
+        if op in (0, 1):
+            traffic["K1" if op == 0 else "K2"] = rd + wr
 if os.path.exists(os.path.join(src, "bench.json")):
     try:
         b = json.loads(open(os.path.join(src, "bench.json")).read().strip().splitlines()[-1])
