@@ -1692,7 +1692,10 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
       ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
     } else {  // nothing to copy: the kernel reads the image where it is
       c_begin = c_end = nullptr;
-      lp.image_remote = img->device != device;
+      // CHECL_FORCE_IMAGE_REMOTE=1 (tests): treat a same-device image as a peer GPU's,
+      // so the one-GPU test box runs K2's peer-read path (register loads for every round)
+      static const bool force_remote = std::getenv("CHECL_FORCE_IMAGE_REMOTE") != nullptr;
+      lp.image_remote = img->device != device || force_remote;
     }
     lp.c0 = 0;
     lp.c1 = nch;

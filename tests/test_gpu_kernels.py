@@ -56,19 +56,32 @@ for slot in (None, 196608):
         raise SystemExit("corruption not detected")
     except checl.CheclError as e:
         assert e.report.first_bad_chunk == rep_o["first_bad_chunk"]
+    # a corrupted HBM image (K2 reads it in place; with CHECL_FORCE_IMAGE_REMOTE as a peer's)
+    dimg.corrupt(poff + 65536 * 16 + 5, 1)
+    try:
+        ctx.restore(dimg, 0)
+        raise SystemExit("device image corruption not detected")
+    except checl.CheclError as e:
+        assert e.report.first_bad_chunk == rep_o["first_bad_chunk"] and e.report.n_bad_chunks == 1
     ctx.close()
 print("kernel ok")
 """
 
 
-@pytest.mark.parametrize("kernel", ["1", "2", "3", "4", "4:0:1", "4:500:3", "4:900:16", "4:0:1:mc", "4:500:3:mc"])
+@pytest.mark.parametrize("kernel", ["1", "2", "3", "4", "4:0:1", "4:500:3", "4:900:16", "4:0:1:mc", "4:500:3:mc",
+                                    "0:remote", "4:remote", "4:0:1:remote"])
 def test_forced_kernel_shapes_bit_exact(kernel):
     """kernel "4:S:B" = the TMA kernel with the dynamic tail forced on at this size:
     static share S permille, dynamic blocks of B rounds (S = 0: every round dynamic;
     with ":mc" the grid is rounded down to whole 2-CTA clusters, so the 3-chunk stages
-    have more blocks than warps: every warp must keep fetching)."""
+    have more blocks than warps: every warp must keep fetching). ":remote": restores
+    from the HBM image read it as a peer GPU's image (the migration i -> j path, which a
+    one-GPU box cannot reach otherwise); kernel "0" = the default dispatch."""
     k, *dyn = kernel.split(":")
     env = dict(os.environ, CHECL_KERNEL=k)
+    if dyn and dyn[-1] == "remote":  # K2 on an HBM image takes the peer-GPU read path (migration i -> j)
+        env.update(CHECL_FORCE_IMAGE_REMOTE="1")
+        dyn = dyn[:-1]
     if dyn and dyn[-1] == "mc":  # 2-CTA clusters with the multicast table prologue (even grids)
         env.update(CHECL_TABLE_MC="1")
         dyn = dyn[:-1]
