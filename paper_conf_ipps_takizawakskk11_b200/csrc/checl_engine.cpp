@@ -1418,6 +1418,10 @@ void set_report(checl_report* rep, const Parsed& P, uint64_t n_bad, uint64_t fir
 }
 
 bool ensure_peer(int dev, int peer) {
+  // CHECL_FORCE_NO_PEER=1 (tests): report no peer access, so the one-GPU test box runs
+  // the migration fallback (cudaMemcpyPeerAsync into a local copy, then K2 on it)
+  static const bool force_no_peer = std::getenv("CHECL_FORCE_NO_PEER") != nullptr;
+  if (force_no_peer) return false;
   if (dev == peer) return true;
   int can = 0;
   if (cudaDeviceCanAccessPeer(&can, dev, peer) != cudaSuccess || !can) {

@@ -47,6 +47,10 @@ for slot in (None, 196608):
         assert rep.n_bad_chunks == 0
         for h, b in zip(ds.handles, ds.host):
             assert np.array_equal(bound_bytes(ctx, h), b)
+    rep = ctx.migrate(0, 0)  # K1 into an HBM image, K2 from it (peer path / fallback per env)
+    assert rep.n_bad_chunks == 0
+    for h, b in zip(ds.handles, ds.host):
+        assert np.array_equal(bound_bytes(ctx, h), b), "migrate"
     bad = img.view().copy()
     poff = int(img.header()["payload_off"])
     bad[poff + 65536 * 16 + 5] ^= 1
@@ -69,18 +73,23 @@ print("kernel ok")
 
 
 @pytest.mark.parametrize("kernel", ["1", "2", "3", "4", "4:0:1", "4:500:3", "4:900:16", "4:0:1:mc", "4:500:3:mc",
-                                    "0:remote", "4:remote", "4:0:1:remote"])
+                                    "0:remote", "4:remote", "4:0:1:remote", "0:nopeer", "4:nopeer"])
 def test_forced_kernel_shapes_bit_exact(kernel):
     """kernel "4:S:B" = the TMA kernel with the dynamic tail forced on at this size:
     static share S permille, dynamic blocks of B rounds (S = 0: every round dynamic;
     with ":mc" the grid is rounded down to whole 2-CTA clusters, so the 3-chunk stages
     have more blocks than warps: every warp must keep fetching). ":remote": restores
     from the HBM image read it as a peer GPU's image (the migration i -> j path, which a
-    one-GPU box cannot reach otherwise); kernel "0" = the default dispatch."""
+    one-GPU box cannot reach otherwise); ":nopeer": the fallback when peer access is
+    unavailable (cudaMemcpyPeerAsync of the image, then K2 on the copy); kernel "0" =
+    the default dispatch."""
     k, *dyn = kernel.split(":")
     env = dict(os.environ, CHECL_KERNEL=k)
     if dyn and dyn[-1] == "remote":  # K2 on an HBM image takes the peer-GPU read path (migration i -> j)
         env.update(CHECL_FORCE_IMAGE_REMOTE="1")
+        dyn = dyn[:-1]
+    if dyn and dyn[-1] == "nopeer":  # no peer access: the image is copied to a local buffer first
+        env.update(CHECL_FORCE_NO_PEER="1")
         dyn = dyn[:-1]
     if dyn and dyn[-1] == "mc":  # 2-CTA clusters with the multicast table prologue (even grids)
         env.update(CHECL_TABLE_MC="1")
