@@ -1008,7 +1008,12 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
   // (below 16 MiB of rounds the bulk-copy path measured no better, and with a dirty
   // L2 worse: C1 pack 16.5 -> 21 us)
   const bool tma_op = op == kOpPack || op == kOpVerify || op == kOpCrc || op == kOpCheck;
-  if (!kernel) kernel = p.round_base ? (tma_op && chunks * (kChunkBytes / kRoundBytes) >= 4096 ? 4 : 3) : (small ? 2 : 1);
+  // launches of at most 128 chunks (<= 8 MiB) take the 4 KiB-unit sweep even with a
+  // round_base: no stretch search and a smaller table prologue; measured C1 (3 x 1 MiB,
+  // 48 chunks, `profiles/r01r/c1_kernels.txt`) pack 15.9 -> 14.6 us, verify 15.7 -> 12.8 us
+  if (!kernel)
+    kernel = p.round_base ? (chunks <= 128 ? 2 : tma_op && chunks * (kChunkBytes / kRoundBytes) >= 4096 ? 4 : 3)
+                          : (small ? 2 : 1);
   if (kernel < 3) p.round_base = nullptr;
   // balanced / TMA launches large enough to have a tail: static stretches for the
   // first part of the rounds, dynamic blocks for the rest (DESIGN.md §5 "Work split");
