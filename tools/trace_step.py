@@ -1,5 +1,5 @@
 """CHECL_TRACE=1 host phase trace of checkpoint_into + restore on a device image.
-usage: CHECL_TRACE=1 python tools/trace_step.py [config] [reps]"""
+usage: CHECL_TRACE=1 python tools/trace_step.py [config] [reps] [host]  (host: pinned host image)"""
 import os
 import sys
 
@@ -19,7 +19,7 @@ torch.cuda.synchronize()
 ctx = checl.Context()
 for t in ts:
     ctx.register(t)
-img = ctx.checkpoint_device(0)
+img = ctx.checkpoint(0) if len(sys.argv) > 3 and sys.argv[3] == "host" else ctx.checkpoint_device(0)
 for i in range(reps):
     ctx.checkpoint(0, epoch=i, into=img)
     ctx.restore(img, 0)
