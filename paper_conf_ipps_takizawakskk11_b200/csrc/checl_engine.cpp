@@ -1328,10 +1328,40 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       img->location = CHECL_IMAGE_HOST;
       img->device = -1;
     }
-    img->ensure_host(P.image_bytes, true);
+    img->ensure_host(P.image_bytes + kSlotSlack, true);
     ds.ensure_slots(ctx->slot_bytes, ctx->n_slots);
     ds.crc_scratch.ensure(std::max<uint64_t>(P.n_chunks, 1));
     lp.crc = ds.crc_scratch.p;
+    // small images (<= 128 chunks, i.e. the sweep kernel with its register stores and
+    // exact tails; payload <= CHECL_ZERO_COPY_MAX, default 8 MiB): K1 stores the payload and
+    // the CRC table straight into the mapped pinned image over PCIe, so there is no
+    // staging slot and no D2H copy; the drain span is K1's own
+    static const uint64_t zc_max = [] {
+      const char* e = std::getenv("CHECL_ZERO_COPY_MAX");
+      return e ? (uint64_t)std::strtoull(e, nullptr, 10) : (8ull << 20);
+    }();
+    uint8_t* mapped = nullptr;
+    // (not under a forced kernel 4: its bulk stores are for device memory)
+    if (P.n_chunks && P.n_chunks <= 128 && P.stages.size() == 1 && P.payload_bytes <= zc_max && ds.kernel != 4) {
+      void* dp = nullptr;
+      if (cudaHostGetDevicePointer(&dp, img->host_mut, 0) == cudaSuccess)
+        mapped = static_cast<uint8_t*>(dp);
+      else
+        cudaGetLastError();
+    }
+    if (mapped) {
+      lp.c0 = 0;
+      lp.c1 = P.n_chunks;
+      lp.image = mapped + P.payload_off;
+      lp.image_base = 0;
+      lp.crc_mirror = reinterpret_cast<uint32_t*>(mapped + P.crc_off);
+      ck(cudaEventRecord(c_begin, ds.compute));
+      timed_launch(ds, kt, kOpPack, lp, ds.compute);
+      ck(cudaEventRecord(c_end, ds.compute));
+      tm.n_stages = 1;
+      settle(ctx);  // the previous call's spans, read while K1 runs
+      ck(cudaStreamSynchronize(ds.compute));
+    } else {
     std::vector<cudaEvent_t> packed(ds.n_slots), drained(ds.n_slots);
     for (uint32_t i = 0; i < ds.n_slots; ++i) {
       packed[i] = ds.events.get();
@@ -1392,6 +1422,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
     tm.n_stages = P.stages.size();
     settle(ctx);  // the previous call's spans, read while the pipeline runs
     ck(cudaStreamSynchronize(ds.copy));
+    }
   }
   // a5: header, manifest and meta CRC (the CRC table has landed)
   const double tf = now_ms();
@@ -1715,6 +1746,34 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     tm.n_stages = 1;
     tr("launch");
   } else {
+    // small pinned images (<= 128 chunks, payload <= CHECL_ZERO_COPY_MAX): K2 reads the
+    // payload and the CRC table straight from the mapped pinned image over PCIe (exact
+    // register loads), so there is no staging slot and no H2D copy
+    static const uint64_t zc_max = [] {
+      const char* e = std::getenv("CHECL_ZERO_COPY_MAX");
+      return e ? (uint64_t)std::strtoull(e, nullptr, 10) : (8ull << 20);
+    }();
+    const uint8_t* mapped = nullptr;
+    if (nch && nch <= 128 && img->pinned && img->host_cap >= P.L.image_bytes && P.L.payload_bytes <= zc_max &&
+        P.L.payload_bytes <= ctx->slot_bytes) {
+      void* dp = nullptr;
+      if (cudaHostGetDevicePointer(&dp, const_cast<uint8_t*>(img->host), 0) == cudaSuccess)
+        mapped = static_cast<const uint8_t*>(dp);
+      else
+        cudaGetLastError();
+    }
+    if (mapped) {
+      ck(cudaEventRecord(c_begin, ds.compute));
+      lp.c0 = 0;
+      lp.c1 = nch;
+      lp.image = const_cast<uint8_t*>(mapped + P.L.payload_off);
+      lp.image_base = 0;
+      lp.image_remote = 1;  // not HBM: register loads only
+      lp.crc = reinterpret_cast<uint32_t*>(const_cast<uint8_t*>(mapped + P.L.crc_off));
+      timed_launch(ds, kt, kOpVerify, lp, ds.compute);
+      ck(cudaEventRecord(c_end, ds.compute));
+      tm.n_stages = 1;
+    } else {
     // r3 + r4: fill slot s % n_slots over PCIe while the previous slot is verified
     ck(cudaEventRecord(c_begin, ds.copy));
     ds.ensure_slots(ctx->slot_bytes, ctx->n_slots);
@@ -1747,6 +1806,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     ck(cudaEventRecord(c_end, ds.copy));
     if (stages.empty()) ck(cudaStreamWaitEvent(ds.compute, c_end, 0));
     tm.n_stages = stages.size();
+    }
   }
   if (nch && !lp.status_host) {
     ck(cudaMemcpyAsync(ds.h_status.p, ds.status.p, 16, cudaMemcpyDeviceToHost, ds.compute));
