@@ -73,7 +73,7 @@ print("kernel ok")
 
 
 @pytest.mark.parametrize("kernel", ["1", "2", "3", "4", "4:0:1", "4:500:3", "4:900:16", "4:0:1:mc", "4:500:3:mc",
-                                    "0:remote", "4:remote", "4:0:1:remote", "0:nopeer", "4:nopeer"])
+                                    "0:remote", "4:remote", "4:0:1:remote", "0:nopeer", "4:nopeer", "0:nozc"])
 def test_forced_kernel_shapes_bit_exact(kernel):
     """kernel "4:S:B" = the TMA kernel with the dynamic tail forced on at this size:
     static share S permille, dynamic blocks of B rounds (S = 0: every round dynamic;
@@ -81,12 +81,16 @@ def test_forced_kernel_shapes_bit_exact(kernel):
     have more blocks than warps: every warp must keep fetching). ":remote": restores
     from the HBM image read it as a peer GPU's image (the migration i -> j path, which a
     one-GPU box cannot reach otherwise); ":nopeer": the fallback when peer access is
-    unavailable (cudaMemcpyPeerAsync of the image, then K2 on the copy); kernel "0" =
+    unavailable (cudaMemcpyPeerAsync of the image, then K2 on the copy); ":nozc": small
+    host images staged through a slot instead of the mapped pinned image; kernel "0" =
     the default dispatch."""
     k, *dyn = kernel.split(":")
     env = dict(os.environ, CHECL_KERNEL=k)
     if dyn and dyn[-1] == "remote":  # K2 on an HBM image takes the peer-GPU read path (migration i -> j)
         env.update(CHECL_FORCE_IMAGE_REMOTE="1")
+        dyn = dyn[:-1]
+    if dyn and dyn[-1] == "nozc":  # small host images through the staging slot, not zero copy
+        env.update(CHECL_ZERO_COPY_MAX="0")
         dyn = dyn[:-1]
     if dyn and dyn[-1] == "nopeer":  # no peer access: the image is copied to a local buffer first
         env.update(CHECL_FORCE_NO_PEER="1")
