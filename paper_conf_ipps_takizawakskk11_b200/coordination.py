@@ -69,12 +69,71 @@ def coordinated(take_local: Callable[[], Tuple[object, int, int]], epoch: int, g
     return GlobalSnapshot(ok, img, f, tn, tb, ep, same)
 
 
+class ImagePair:
+    """Two reusable host images for a loop of global snapshots (double buffering).
+
+    Each new local snapshot is written into the image that does NOT hold the last
+    committed global snapshot, so an aborted vote leaves the last committed one
+    intact: the rollback target of the two-phase commit (reading 16).
+    `committed` is that image (None before the first commit). Neither image is
+    re-pinned after its first use."""
+
+    def __init__(self):
+        self.images = [None, None]
+        self.last = -1  # index of the committed image
+
+    @property
+    def committed(self):
+        return self.images[self.last] if self.last >= 0 else None
+
+    def _slot(self) -> int:
+        return 0 if self.last != 0 else 1
+
+    def take(self, ctx, device: int, stream, epoch: int):
+        k = self._slot()
+        if self.images[k] is None:
+            self.images[k] = ctx.checkpoint(device, stream, epoch)
+        else:
+            ctx.checkpoint(device, stream, epoch, into=self.images[k])
+        return self.images[k]
+
+    def commit(self, img):
+        self.last = self.images.index(img)
+
+    def free(self):
+        for im in self.images:
+            if im is not None:
+                im.free()
+        self.images = [None, None]
+        self.last = -1
+
+
 def coordinated_checkpoint(ctx, device: int, epoch: int, group=None, stream=None, into=None,
                            on_device: bool = False) -> GlobalSnapshot:
-    """Local checl_checkpoint (host image, or HBM image with on_device) + commit barrier."""
+    """Local checl_checkpoint (host image, or HBM image with on_device) + commit barrier.
+
+    into=None: a new image; freed on abort. into=Image: written in place (no
+    re-pinning) and kept on abort, but its previous contents are overwritten before
+    the vote, so an abort leaves no committed snapshot to roll back to. into=ImagePair:
+    double-buffered, an abort keeps the last committed snapshot intact (snap.image is
+    then None and pair.committed is the previous global snapshot)."""
+    pair = into if isinstance(into, ImagePair) else None
+
     def local():
         n, b = ctx.count(device)
         if on_device:
             return ctx.checkpoint_device(device, stream, epoch), n, b
+        if pair is not None:
+            return pair.take(ctx, device, stream, epoch), n, b
         return ctx.checkpoint(device, stream, epoch, into=into), n, b
+
+    if pair is not None:
+        k = pair._slot()
+        target = pair.images[k]  # None: the slot's first snapshot (a new image, freed on abort)
+        snap = coordinated(local, epoch, group, device, keep=target)
+        if snap.committed:
+            pair.commit(snap.image)
+        elif target is None:
+            pair.images[k] = None
+        return snap
     return coordinated(local, epoch, group, device, keep=into)

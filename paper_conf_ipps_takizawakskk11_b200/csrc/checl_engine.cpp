@@ -481,7 +481,10 @@ struct DevState {
 
 // ---- library-owned memory (buffers re-created by restore / migrate) ----------
 
-struct Arena {  // one allocation holding every buffer of one restore (payload layout)
+// One allocation of re-created buffers: a *segment* of a restore, i.e. a run of
+// consecutive manifest records laid out like their part of the payload (buffer b
+// at base + off_b - lo). Freed when its last handle is released or rebound.
+struct Arena {
   checl_allocator alloc;
   int device;
   void* stream;
@@ -522,6 +525,11 @@ struct KernelTimer {  // the event pair around every timed launch of a call
 
 struct checl_image {
   int location = CHECL_IMAGE_HOST;
+  // device payload / CRC table from this allocator when set (the migration image
+  // comes from the context's allocator, so freeing it returns the memory to the
+  // caller's pool); cudaMalloc / cudaFree otherwise
+  checl_allocator dalloc{nullptr, nullptr, nullptr};
+  void* dstream = nullptr;
   int device = -1;  // device image: where payload and CRC table live
   bool owned = true;
   bool pinned = false;
@@ -537,13 +545,29 @@ struct checl_image {
   const uint8_t* mapped_for = nullptr;
   uint8_t* mapped_dev = nullptr;
 
+  void* dev_alloc(size_t n) {  // on the current device (= `device`); nullptr on failure
+    if (dalloc.alloc) return dalloc.alloc(n, device, dstream, dalloc.user);
+    void* p = nullptr;
+    if (cudaMalloc(&p, n) != cudaSuccess) {
+      cudaGetLastError();
+      return nullptr;
+    }
+    return p;
+  }
+  void dev_free(void* p) {
+    if (!p) return;
+    if (dalloc.free)
+      dalloc.free(p, device, dstream, dalloc.user);
+    else
+      cudaFree(p);
+  }
   void free_device() {
     if (device >= 0 && (d_payload || d_crc)) {
       int prev = -1;
       cudaGetDevice(&prev);
       cudaSetDevice(device);
-      if (d_payload) cudaFree(d_payload);
-      if (d_crc) cudaFree(d_crc);
+      dev_free(d_payload);
+      dev_free(d_crc);
       if (prev >= 0) cudaSetDevice(prev);
     }
     d_payload = nullptr;
@@ -622,11 +646,14 @@ struct checl_ctx {
   mutable PendingTiming pend;
   mutable checl_stats stats[CHECL_STATS_KINDS] = {};
   mutable std::mutex tmu;
-  checl_image* mig_img[kMaxDevices] = {};  // migration images, reused (HBM of the source)
-  // the last allocation a commit released on each device, kept for the next restore
-  // of (nearly) the same size: skips an allocator round trip per restore (a
-  // checkpoint/restore loop re-creates a same-sized arena every time)
-  std::shared_ptr<Arena> spare[kMaxDevices];
+  // the segments the last commit on each device released (bounded by
+  // CHECL_SPARE_BYTES, default 8 GiB), kept for the next restore of (nearly) the same
+  // layout: a checkpoint/restore loop re-creates same-sized segments every time and
+  // skips one allocator round trip per segment; checl_trim frees them
+  std::vector<std::shared_ptr<Arena>> spares[kMaxDevices];
+  // arenas whose last handle was released while a checkpoint / restore / migrate ran
+  // (its plan may still read them): freed when that call ends (BusyGuard)
+  std::vector<std::shared_ptr<Arena>> deferred;
 
   DevState& dev(int d) {
     if (!devs[d]) {
@@ -646,6 +673,23 @@ struct checl_ctx {
 
 namespace {
 
+// Frees arenas once their devices are idle (no kernel of any stream can still read
+// or write them).
+void free_arenas(std::vector<std::shared_ptr<Arena>>& v) {
+  bool synced[kMaxDevices] = {};
+  int prev = -1;
+  for (auto& a : v) {
+    if (a && a.use_count() == 1 && a->base && !synced[a->device]) {  // one wait per device
+      if (prev < 0) cudaGetDevice(&prev);
+      cudaSetDevice(a->device);
+      cudaDeviceSynchronize();
+      synced[a->device] = true;
+    }
+  }
+  if (prev >= 0) cudaSetDevice(prev);
+  v.clear();  // (the arenas free their allocations)
+}
+
 struct BusyGuard {
   checl_ctx* ctx;
   bool ok;
@@ -654,7 +698,15 @@ struct BusyGuard {
     ok = ctx->busy.compare_exchange_strong(expected, true);
   }
   ~BusyGuard() {
-    if (ok) ctx->busy.store(false);
+    if (!ok) return;
+    std::vector<std::shared_ptr<Arena>> d;
+    {
+      // (under the lock checl_release decides between freeing and deferring)
+      std::lock_guard<std::mutex> lk(ctx->mu);
+      ctx->busy.store(false);
+      d.swap(ctx->deferred);
+    }
+    free_arenas(d);
   }
 };
 
@@ -969,10 +1021,14 @@ LaunchParams base_params(DevState& ds) {
 void d2h_page_aligned(uint8_t* dst, const uint8_t* src, uint64_t n, cudaStream_t s) {
   const uintptr_t d0 = reinterpret_cast<uintptr_t>(dst), d1 = d0 + n;
   const uintptr_t a0 = (d0 + 4095) & ~static_cast<uintptr_t>(4095), a1 = d1 & ~static_cast<uintptr_t>(4095);
-  static const bool split = [] {  // CHECL_D2H_SPLIT=0: one copy per stage (A/B)
+#ifdef CHECL_EXPERIMENTS
+  static const bool split = [] {  // CHECL_D2H_SPLIT=0: one copy per stage (A/B, experiments build)
     const char* e = std::getenv("CHECL_D2H_SPLIT");
     return !e || std::atoi(e) != 0;
   }();
+#else
+  constexpr bool split = true;
+#endif
   if (!split || n < 4 * 4096 || (a0 == d0 && a1 == d1)) {
     ck(cudaMemcpyAsync(dst, src, n, cudaMemcpyDeviceToHost, s));
     return;
@@ -989,13 +1045,16 @@ void gck(const char* what, cudaError_t e) {
 
 void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0, cudaStream_t s) {
   LaunchParams p = p0;
-  // experiments only (tools/exp_run.py): CHECL_EXP_PACK_OP=2|4 replaces the pack
-  // launches by the CRC-only / copy-only op over the same plan (no valid image)
+#ifdef CHECL_EXPERIMENTS
+  // experiments build only (libchecl_exp.so, tools/exp_run.py): CHECL_EXP_PACK_OP=2|4
+  // replaces the pack launches by the CRC-only / copy-only op over the same plan (no
+  // valid image); the product library does not read it
   static const int exp_pack_op = [] {
     const char* e = std::getenv("CHECL_EXP_PACK_OP");
     return e ? std::atoi(e) : -1;
   }();
   if (op == kOpPack && (exp_pack_op == kOpCrc || exp_pack_op == kOpCopy)) op = exp_pack_op;
+#endif
   const uint64_t chunks = p.c1 - p.c0;
   // kernel 4 (bulk copies, column CRC; scheduled stretches of rounds) whenever the
   // chunk list has a round_base (kernel 3 for the ops kernel 4 does not implement);
@@ -1017,7 +1076,10 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
   if (kernel < 3) p.round_base = nullptr;
   // balanced / TMA launches large enough to have a tail: static stretches for the
   // first part of the rounds, dynamic blocks for the rest (DESIGN.md §5 "Work split");
-  // CHECL_STATIC_PERMILLE / CHECL_DYN_BLOCK override the defaults (experiments)
+  // the experiments build reads CHECL_STATIC_PERMILLE / CHECL_DYN_BLOCK /
+  // CHECL_DYN_MIN_ROUNDS overrides (sweeps, and the kernel-shape tests that force the
+  // tail on at small sizes)
+#ifdef CHECL_EXPERIMENTS
   static const uint32_t static_pm = [] {
     const char* e = std::getenv("CHECL_STATIC_PERMILLE");
     return e ? (uint32_t)std::min(1000, std::max(0, std::atoi(e))) : 750u;
@@ -1026,11 +1088,15 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
     const char* e = std::getenv("CHECL_DYN_BLOCK");
     return e ? (uint32_t)std::max(1, std::atoi(e)) : 8u;
   }();
-  // (kernel 3 keeps static stretches only: measured slower with the dynamic tail)
   static const uint64_t dyn_min = [] {
     const char* e = std::getenv("CHECL_DYN_MIN_ROUNDS");
     return e ? (uint64_t)std::strtoull(e, nullptr, 10) : ~0ull;
   }();
+#else
+  constexpr uint32_t static_pm = 750u, dyn_block = 8u;
+  constexpr uint64_t dyn_min = ~0ull;
+#endif
+  // (kernel 3 keeps static stretches only: measured slower with the dynamic tail)
   // (a dynamic tail pays when a warp has tens of rounds: measured 64 MiB launches (11
   // rounds per warp) 37 -> 49 us with it, 463 MB (76 per warp) 169 -> 164 us)
   const uint64_t min_rounds = dyn_min != ~0ull ? dyn_min : (uint64_t)ds.n_sms * kWarpsPerCta * 48;
@@ -1046,9 +1112,14 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
     }
     p.unit_acc = ds.unit_acc.p;
   }
-  // diagnostics: CHECL_WARP_TRACE=1 prints the warps' start / tables-ready / end
-  // times of every balanced or TMA launch (relative to the earliest start, us)
+  // diagnostics (experiments build): CHECL_WARP_TRACE=1 prints the warps' start /
+  // tables-ready / end times of every balanced or TMA launch (relative to the earliest
+  // start, us)
+#ifdef CHECL_EXPERIMENTS
   static const bool warp_tr = std::getenv("CHECL_WARP_TRACE") != nullptr;
+#else
+  constexpr bool warp_tr = false;
+#endif
   const uint64_t n_tr = (uint64_t)ds.n_sms * kWarpsPerCta * 4;
   if (warp_tr && kernel >= 3) {
     ds.warp_trace.ensure(n_tr);
@@ -1130,6 +1201,7 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
     std::fprintf(stderr, "[checl] timed_launch op %d kernel %d%s: record/update %.1f launch %.1f record %.1f us\n", op,
                  kernel, fn ? " (graph)" : "",
                  (h1 - h0) * 1e3, (h2 - h1) * 1e3, (now_ms() - h2) * 1e3);
+#ifdef CHECL_EXPERIMENTS
   if (p.warp_trace) {
     std::vector<unsigned long long> h(n_tr);
     ck(cudaMemcpyAsync(h.data(), p.warp_trace, n_tr * 8, cudaMemcpyDeviceToHost, s));
@@ -1156,7 +1228,8 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
                  "end min %.1f p10 %.1f p50 %.1f p90 %.1f max %.1f us\n",
                  op, kernel, st.size(), ms * 1e3, q(st, 0.5), q(st, 1.0), q(tb, 0.5), q(tb, 1.0), q(en, 0.0), q(en, 0.1),
                  q(en, 0.5), q(en, 0.9), q(en, 1.0));
-    if (std::atoi(std::getenv("CHECL_WARP_TRACE")) == 2) {  // raw end times, one line per CTA
+    const char* wt = std::getenv("CHECL_WARP_TRACE");
+    if (wt && std::atoi(wt) == 2) {  // raw end times, one line per CTA
       for (int c = 0; c < ds.n_sms; ++c) {
         std::string line = "[checl] cta " + std::to_string(c) + " sm " + std::to_string(h[4 * (uint64_t)c * kWarpsPerCta + 3]);
         for (int w = 0; w < kWarpsPerCta; ++w) {
@@ -1169,6 +1242,7 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
       }
     }
   }
+#endif
 }
 
 // Writes header + manifest + meta_crc into the image's host bytes [0, payload_off);
@@ -1235,6 +1309,31 @@ void begin_events(checl_ctx* ctx, DevState& ds) {
   ds.events.reset();
 }
 
+// The caller's stream, if it belongs to `device` (the allocator hands out memory that
+// is safe to use in the order of that stream); nullptr (the legacy default stream of
+// the current device) otherwise.
+void* stream_on(void* stream, int device) {
+  if (!stream) return nullptr;
+  int d = -1;
+  if (cudaStreamGetDevice(static_cast<cudaStream_t>(stream), &d) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return d == device ? stream : nullptr;
+}
+
+// New allocations are written by the library's own streams, but the allocator (the
+// PyTorch caching allocator) hands out blocks that are safe only in the order of the
+// stream they were requested on: a block the application freed while its kernels
+// were still pending could otherwise be overwritten by those kernels after K2. The
+// library's streams wait for everything queued on that stream so far.
+void order_after(DevState& ds, void* stream) {
+  cudaEvent_t ev = ds.events.get();
+  ck(cudaEventRecord(ev, static_cast<cudaStream_t>(stream)));
+  ck(cudaStreamWaitEvent(ds.compute, ev, 0));
+  ck(cudaStreamWaitEvent(ds.copy, ev, 0));
+}
+
 checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t epoch, checl_image* img,
                            bool to_device) {
   (void)stream;
@@ -1273,19 +1372,22 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
     img->location = CHECL_IMAGE_DEVICE;
     img->device = device;
     if (img->d_payload_cap < P.payload_bytes + kSlotSlack) {
-      if (img->d_payload) cudaFree(img->d_payload);
+      img->dev_free(img->d_payload);
       img->d_payload = nullptr;
       img->d_payload_cap = 0;
-      ck(cudaMalloc(&img->d_payload, P.payload_bytes + kSlotSlack));
+      img->d_payload = static_cast<uint8_t*>(img->dev_alloc(P.payload_bytes + kSlotSlack));
+      if (!img->d_payload) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
       img->d_payload_cap = P.payload_bytes + kSlotSlack;
     }
     if (img->d_crc_cap < std::max<uint64_t>(P.n_chunks, 1)) {
-      if (img->d_crc) cudaFree(img->d_crc);
+      img->dev_free(img->d_crc);
       img->d_crc = nullptr;
       img->d_crc_cap = 0;
-      ck(cudaMalloc(&img->d_crc, std::max<uint64_t>(P.n_chunks, 1) * 4));
+      img->d_crc = static_cast<uint32_t*>(img->dev_alloc(std::max<uint64_t>(P.n_chunks, 1) * 4));
+      if (!img->d_crc) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
       img->d_crc_cap = std::max<uint64_t>(P.n_chunks, 1);
     }
+    if (img->dalloc.alloc) order_after(ds, img->dstream);
     img->ensure_host(P.payload_off, true);
     lp.c0 = 0;
     lp.c1 = P.n_chunks;
@@ -1367,8 +1469,12 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       packed[i] = ds.events.get();
       drained[i] = ds.events.get();
     }
-    // diagnostics: CHECL_STAGE_TRACE=1 times every stage's D2H (events around it)
+    // diagnostics (experiments build): CHECL_STAGE_TRACE=1 times every stage's D2H
+#ifdef CHECL_EXPERIMENTS
     static const bool stage_tr = std::getenv("CHECL_STAGE_TRACE") != nullptr;
+#else
+    constexpr bool stage_tr = false;
+#endif
     std::vector<std::pair<cudaEvent_t, cudaEvent_t>> d2h;
     ck(cudaEventRecord(c_begin, ds.copy));
     for (size_t s = 0; s < P.stages.size(); ++s) {
@@ -1473,28 +1579,77 @@ bool ensure_peer(int dev, int peer) {
   return true;
 }
 
-// Largest allocation kept as a spare (CHECL_SPARE_BYTES, default 4 GiB): larger
-// re-creations amortise their allocator call anyway, and a spare holds HBM idle.
+// Bytes of segments kept as spares per device (CHECL_SPARE_BYTES, default 8 GiB):
+// larger re-creations amortise their allocator calls anyway, and a spare holds HBM idle
+// (checl_trim releases it).
 uint64_t spare_limit() {
   static const uint64_t v = [] {
     const char* e = std::getenv("CHECL_SPARE_BYTES");
-    return e ? (uint64_t)std::strtoull(e, nullptr, 10) : (4ull << 30);
+    return e ? (uint64_t)std::strtoull(e, nullptr, 10) : (8ull << 30);
   }();
   return v;
 }
 
-// r2: one allocation of `bytes` on `device` (through the context's allocator), or
-// the spare the last commit on this device released when it is large enough and
-// at most 1/8 larger. nullptr when the allocator fails.
-std::shared_ptr<Arena> new_arena(checl_ctx* ctx, int device, void* stream, uint64_t bytes) {
-  {
-    std::lock_guard<std::mutex> lk(ctx->mu);
-    std::shared_ptr<Arena>& sp = ctx->spare[device];
-    if (sp && bytes && sp->bytes >= bytes && sp->bytes - bytes <= bytes / 8) {
-      std::shared_ptr<Arena> a = std::move(sp);
-      return a;
+// Target size of one allocation of re-created buffers (CHECL_SEGMENT_BYTES, default
+// 64 MiB; 0 = one allocation per restore). Restore re-creates the objects of an image
+// as a few segments instead of one object at a time (10 000 allocator calls for C3)
+// or one block for all (which could not be returned until every handle is released).
+uint64_t segment_bytes() {
+  static const uint64_t v = [] {
+    const char* e = std::getenv("CHECL_SEGMENT_BYTES");
+    return e ? (uint64_t)std::strtoull(e, nullptr, 10) : (64ull << 20);
+  }();
+  return v;
+}
+
+// A segment: records [b0, b1), payload span [lo, hi) = from buffer b0's offset to the
+// next segment's first offset (or payload_bytes), so the padding a chunk owns lies
+// inside its segment.
+struct Segment {
+  size_t b0, b1;
+  uint64_t lo, hi;
+};
+
+// Consecutive records in manifest order; a segment is closed before a record that
+// would take it past segment_bytes(), so a buffer at least that large is alone.
+std::vector<Segment> plan_segments(const std::vector<BufRec>& bufs, uint64_t payload_bytes) {
+  std::vector<Segment> out;
+  if (bufs.empty()) return out;
+  const uint64_t T = segment_bytes();
+  size_t b0 = 0;
+  for (size_t b = 1; b < bufs.size(); ++b) {
+    if (T && bufs[b].off + bufs[b].size - bufs[b0].off > T) {
+      out.push_back(Segment{b0, b, bufs[b0].off, bufs[b].off});
+      b0 = b;
     }
   }
+  out.push_back(Segment{b0, bufs.size(), bufs[b0].off, payload_bytes});
+  return out;
+}
+
+// The re-created buffers of one restore (r2).
+struct RestoreAlloc {
+  std::vector<Segment> segs;
+  std::vector<std::shared_ptr<Arena>> arenas;  // one per segment (base nullptr when empty)
+  std::vector<uint32_t> seg_of;                // per record
+  // device address of record b (nullptr for a zero-size buffer)
+  uint8_t* buf(const std::vector<BufRec>& bufs, size_t b) const {
+    if (!bufs[b].size) return nullptr;
+    const uint32_t k = seg_of[b];
+    return static_cast<uint8_t*>(arenas[k]->base) + (bufs[b].off - segs[k].lo);
+  }
+  // device address of full-payload offset o (inside some segment's span)
+  uint8_t* at(uint64_t o) const {
+    size_t lo = 0, hi = segs.size();
+    while (hi - lo > 1) {
+      const size_t mid = (lo + hi) / 2;
+      (segs[mid].lo <= o ? lo : hi) = mid;
+    }
+    return static_cast<uint8_t*>(arenas[lo]->base) + (o - segs[lo].lo);
+  }
+};
+
+std::shared_ptr<Arena> alloc_arena(checl_ctx* ctx, int device, void* stream, uint64_t bytes) {
   auto arena = std::make_shared<Arena>();
   arena->alloc = ctx->alloc;
   arena->device = device;
@@ -1512,19 +1667,58 @@ std::shared_ptr<Arena> new_arena(checl_ctx* ctx, int device, void* stream, uint6
   return arena;
 }
 
-// Swaps every handle of the image to its new buffer (L15); frees library-owned
-// buffers previously bound to those handles (after their devices are idle).
-void commit(checl_ctx* ctx, const Parsed& P, int device, const std::shared_ptr<Arena>& arena) {
-  std::vector<std::shared_ptr<Arena>> dropped;  // distinct arenas that lost handles
+// r2: the segments of `bufs` on `device`, each from the spares the last commit on
+// this device released (best fit, at most 1/8 larger) or through the context's
+// allocator. false when the allocator fails (whatever was taken is freed).
+bool new_alloc(checl_ctx* ctx, int device, void* stream, const std::vector<BufRec>& bufs, uint64_t payload_bytes,
+               RestoreAlloc* out) {
+  out->segs = plan_segments(bufs, payload_bytes);
+  out->arenas.assign(out->segs.size(), nullptr);
+  out->seg_of.assign(bufs.size(), ~0u);
+  std::vector<size_t> need;  // segments the spares did not cover
   {
     std::lock_guard<std::mutex> lk(ctx->mu);
-    if (arena->base) ctx->by_addr[device][reinterpret_cast<uintptr_t>(arena->base)] = {arena->bytes, 0};
+    auto& sp = ctx->spares[device];
+    for (size_t k = 0; k < out->segs.size(); ++k) {
+      const uint64_t n = out->segs[k].hi - out->segs[k].lo;
+      size_t best = sp.size();
+      for (size_t i = 0; n && i < sp.size(); ++i)
+        if (sp[i]->bytes >= n && sp[i]->bytes - n <= n / 8 && (best == sp.size() || sp[i]->bytes < sp[best]->bytes))
+          best = i;
+      if (best != sp.size()) {
+        out->arenas[k] = std::move(sp[best]);
+        sp.erase(sp.begin() + (long)best);
+      } else {
+        need.push_back(k);
+      }
+    }
+  }
+  for (size_t k : need) {
+    out->arenas[k] = alloc_arena(ctx, device, stream, out->segs[k].hi - out->segs[k].lo);
+    if (!out->arenas[k]) {
+      out->arenas.clear();
+      return false;
+    }
+  }
+  for (size_t k = 0; k < out->segs.size(); ++k)
+    for (size_t b = out->segs[k].b0; b < out->segs[k].b1; ++b) out->seg_of[b] = (uint32_t)k;
+  return true;
+}
+
+// Swaps every handle of the image to its new buffer (L15); frees library-owned
+// buffers previously bound to those handles (after their devices are idle).
+void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A) {
+  std::vector<std::shared_ptr<Arena>> dropped;  // distinct arenas that lost their last handle
+  {
+    std::lock_guard<std::mutex> lk(ctx->mu);
+    for (auto& a : A.arenas)
+      if (a->base) ctx->by_addr[device][reinterpret_cast<uintptr_t>(a->base)] = {a->bytes, 0};
     uint64_t max_h = 0;
     // P.bufs ascend by handle, like the map: walk both in order (O(n), sequential)
     // instead of one O(log n) search per handle (C3: 10 000 handles)
     auto it = P.bufs.empty() ? ctx->entries.end() : ctx->entries.lower_bound(P.bufs.front().handle);
-    Arena* const na = arena.get();
-    for (const BufRec& b : P.bufs) {
+    for (size_t bi = 0; bi < P.bufs.size(); ++bi) {
+      const BufRec& b = P.bufs[bi];
       while (it != ctx->entries.end() && it->first < b.handle) ++it;
       const bool fresh = it == ctx->entries.end() || it->first != b.handle;
       if (fresh) it = ctx->entries.emplace_hint(it, b.handle, Entry{});
@@ -1541,39 +1735,46 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, const std::shared_ptr<A
       }
       ctx->n_live[device]++;
       e.device = device;
-      e.ptr = b.size ? static_cast<uint8_t*>(na->base) + b.off : nullptr;
+      e.ptr = A.buf(P.bufs, bi);
       e.bytes = b.size;
       e.flags = b.flags;
       e.owned = true;
-      e.arena = b.size ? na : nullptr;
-      if (b.size) na->n_handles++;
+      Arena* na = b.size ? A.arenas[A.seg_of[bi]].get() : nullptr;
+      e.arena = na;
+      if (na) na->n_handles++;
       max_h = std::max(max_h, b.handle);
     }
-    if (na->n_handles) ctx->arenas.emplace(na, arena);
+    for (auto& a : A.arenas)
+      if (a->n_handles) ctx->arenas.emplace(a.get(), a);
     ctx->version[device]++;
     ctx->next_id = std::max(ctx->next_id, max_h + 1);
     for (auto& a : dropped)
       if (a->base) ctx->by_addr[a->device].erase(reinterpret_cast<uintptr_t>(a->base));
   }
-  // arenas whose last handle moved away are freed here, outside the lock, once
-  // their device is idle (the restore quiesced `device` when it started and has
-  // synchronised its own streams since; another device is synchronised here)
+  // arenas whose last handle moved away are freed here, outside the lock, once their
+  // device is idle (the restore synchronised `device` after K2; another device is
+  // synchronised here); on this device they become the spares of the next restore
+  // (the previous spares are freed)
+  std::vector<std::shared_ptr<Arena>> keep, old;
+  uint64_t kept = 0;
+  bool other = false;
   for (auto& a : dropped) {
     if (a->device != device) {
-      DeviceGuard g(a->device);
-      ck(cudaDeviceSynchronize());
+      other = true;
+      continue;
     }
-    if (a.use_count() == 1 && a->base && a->bytes <= spare_limit()) {  // the device's spare (the previous is freed)
-      std::shared_ptr<Arena> old;
-      {
-        std::lock_guard<std::mutex> lk(ctx->mu);
-        old = std::move(ctx->spare[a->device]);
-        ctx->spare[a->device] = std::move(a);
-      }
-      old.reset();
+    if (a.use_count() == 1 && a->base && kept + a->bytes <= spare_limit()) {
+      kept += a->bytes;
+      keep.push_back(std::move(a));
     }
-    a.reset();
   }
+  if (!keep.empty()) {
+    std::lock_guard<std::mutex> lk(ctx->mu);
+    old.swap(ctx->spares[device]);
+    ctx->spares[device] = std::move(keep);
+  }
+  free_arenas(old);
+  if (other || !dropped.empty()) free_arenas(dropped);
 }
 
 // After a successful restore onto `device`, the chunk list it expanded for the new
@@ -1581,7 +1782,7 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, const std::shared_ptr<A
 // checkpoint of `device` needs when the device's live buffers are the image's: it
 // becomes that plan (buffers swapped, no re-expansion), so a checkpoint right
 // after a restore or migration skips the plan rebuild.
-void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, uint8_t* abase, uint64_t rounds) {
+void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, const RestoreAlloc& A) {
   std::lock_guard<std::mutex> lk(ctx->mu);
   if (ctx->n_live[device] != P.bufs.size() || !P.L.n_chunks) return;
   Plan& Q = ds.plan;
@@ -1599,7 +1800,7 @@ void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, uint8
            q.flags == b.flags;
   }
   if (same) {
-    for (auto& b : Q.bufs) b.ptr = b.size ? abase + b.off : nullptr;
+    for (size_t i = 0; i < Q.bufs.size(); ++i) Q.bufs[i].ptr = A.buf(Q.bufs, i);
     Q.recs.resize(Q.bufs.size());
     build_records(Q.bufs, [&](size_t b) { return Q.bufs[b].ptr; }, Q.recs.data());
     std::swap(Q.d_desc.p, ds.desc_scratch.p);
@@ -1610,7 +1811,7 @@ void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, uint8
     return;
   }
   Q.bufs = P.bufs;
-  for (auto& b : Q.bufs) b.ptr = b.size ? abase + b.off : nullptr;
+  for (size_t i = 0; i < Q.bufs.size(); ++i) Q.bufs[i].ptr = A.buf(Q.bufs, i);
   Q.n_chunks = P.L.n_chunks;
   Q.payload_bytes = P.full_payload;
   Q.crc_off = P.L.crc_off;
@@ -1632,7 +1833,6 @@ void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, uint8
   std::swap(Q.d_desc.cap, ds.desc_scratch.cap);
   std::swap(Q.d_round.p, ds.round_scratch.p);
   std::swap(Q.d_round.cap, ds.round_scratch.cap);
-  (void)rounds;
   Q.version = ctx->version[device];
   Q.slot_bytes = ctx->slot_bytes;
 }
@@ -1666,20 +1866,20 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   if (rep) set_report(rep, P, 0, 0);
   tr("parse");
 
-  // r2: re-create the buffers: one allocation laid out like the payload
+  // r2: re-create the buffers: a few allocations (segments) laid out like the payload
   const double ta = now_ms();
-  auto arena = new_arena(ctx, device, stream, P.L.payload_bytes);
-  if (!arena)  // (an invalid image still reports BAD_IMAGE first)
+  stream = stream_on(stream, device);
+  RestoreAlloc A;
+  if (!new_alloc(ctx, device, stream, P.bufs, P.L.payload_bytes, &A))  // (an invalid image still reports BAD_IMAGE first)
     return get_u32(img->host + 124) == meta_crc(img->host, P.L.payload_off) ? CHECL_ERR_OUT_OF_DEVICE_MEMORY
                                                                            : CHECL_ERR_BAD_IMAGE;
+  order_after(ds, stream);  // nothing below touches the new memory before the caller's queued work
   tm.alloc_ms = now_ms() - ta;
   tr("alloc");
   const uint64_t nch = P.L.n_chunks;
   ds.h_recs.ensure(std::max<size_t>(P.bufs.size(), 1));
-  uint8_t* abase = static_cast<uint8_t*>(arena->base);
   // (zero-size buffers get a null pointer, as in adopt_plan's records)
-  const uint64_t rounds = build_records(
-      P.bufs, [&](size_t b) { return P.bufs[b].size ? abase + P.bufs[b].off : nullptr; }, ds.h_recs.p);
+  const uint64_t rounds = build_records(P.bufs, [&](size_t b) { return A.buf(P.bufs, b); }, ds.h_recs.p);
   ds.desc_scratch.ensure(std::max<uint64_t>(nch, 1));
   ds.round_scratch.ensure(nch + 1);
   ds.recs_scratch.ensure(std::max<size_t>(P.bufs.size(), 1));
@@ -1833,15 +2033,15 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   if (n_bad) {
     tm.total_ms = now_ms() - t0;
     defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_RESTORE);
-    return CHECL_ERR_CRC_MISMATCH;  // arena freed by its destructor; nothing rebound
+    return CHECL_ERR_CRC_MISMATCH;  // segments freed by their destructors; nothing rebound
   }
   // r5: rebind every handle (all-or-nothing)
   (void)in_migrate;
   const double tc = now_ms();
   tr("events");
-  commit(ctx, P, device, arena);
+  commit(ctx, P, device, A);
   tr("commit");
-  adopt_plan(ctx, ds, device, P, abase, rounds);
+  adopt_plan(ctx, ds, device, P, A);
   tr("adopt");
   tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
@@ -2036,12 +2236,13 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   tm.sync_ms = now_ms() - ts;
   if (rep) set_report(rep, Z, 0, 0);
 
-  // r2: one allocation laid out like the full payload
+  // r2: segments laid out like the full payload
   const double ta = now_ms();
-  auto arena = new_arena(ctx, device, stream, F.full_payload);
-  if (!arena) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
+  stream = stream_on(stream, device);
+  RestoreAlloc A;
+  if (!new_alloc(ctx, device, stream, F.bufs, F.full_payload, &A)) return CHECL_ERR_OUT_OF_DEVICE_MEMORY;
+  order_after(ds, stream);
   tm.alloc_ms = now_ms() - ta;
-  uint8_t* abase = static_cast<uint8_t*>(arena->base);
   const uint64_t nch = F.L.n_chunks;
 
   // descriptors of every delta's present chunks: ptr = destination in the arena,
@@ -2073,7 +2274,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
           cur = DStage{i, hdesc.size(), hdesc.size(), pos, pos};
           open = true;
         }
-        hdesc.push_back(ChunkDesc{reinterpret_cast<uint64_t>(abase + a), (uint32_t)(pos / kBufferAlign),
+        hdesc.push_back(ChunkDesc{reinterpret_cast<uint64_t>(A.at(a)), (uint32_t)(pos / kBufferAlign),
                                   make_len_pad(len, (uint32_t)(z - a - len))});
         pos += z - a;
         cur.c1 = hdesc.size();
@@ -2089,15 +2290,17 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
   ds.crc_scratch.ensure(std::max<uint64_t>(nch, 1));
   ds.h_recs.ensure(std::max<size_t>(F.bufs.size(), 1));
   ds.recs_scratch.ensure(std::max<size_t>(F.bufs.size(), 1));
-  const uint64_t rounds = build_records(F.bufs, [&](size_t b) { return abase + F.bufs[b].off; }, ds.h_recs.p);
+  const uint64_t rounds = build_records(F.bufs, [&](size_t b) { return A.buf(F.bufs, b); }, ds.h_recs.p);
   ds.round_scratch.ensure(nch + 1);
   tm.plan_ms = now_ms() - tp;
 
   cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get(), base_in = ds.events.get();
   ck(cudaEventRecord(c_begin, ds.copy));
-  // r3: F's payload straight into the arena; the last CRC table; the delta chunk list
-  if (F.full_payload)
-    ck(cudaMemcpyAsync(abase, chain[0]->host + F.L.payload_off, F.full_payload, cudaMemcpyHostToDevice, ds.copy));
+  // r3: F's payload straight into the segments; the last CRC table; the delta chunk list
+  for (size_t k = 0; k < A.segs.size(); ++k)
+    if (A.segs[k].hi > A.segs[k].lo)
+      ck(cudaMemcpyAsync(A.arenas[k]->base, chain[0]->host + F.L.payload_off + A.segs[k].lo, A.segs[k].hi - A.segs[k].lo,
+                         cudaMemcpyHostToDevice, ds.copy));
   ck(cudaEventRecord(base_in, ds.copy));
   if (nch)
     ck(cudaMemcpyAsync(ds.crc_scratch.p, chain[n_img - 1]->host + Z.L.crc_off, 4 * nch, cudaMemcpyHostToDevice, ds.copy));
@@ -2168,7 +2371,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
     return CHECL_ERR_CRC_MISMATCH;
   }
   const double tc = now_ms();
-  commit(ctx, Z, device, arena);
+  commit(ctx, Z, device, A);
   tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
   defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_CHAIN);
@@ -2211,21 +2414,14 @@ checl_status checl_destroy(checl_ctx* ctx) {
       ctx->entries.clear();
       ctx->arenas.clear();
       for (auto& n : ctx->n_live) n = 0;
-      for (auto& sp : ctx->spare) sp.reset();
+      for (auto& sp : ctx->spares) sp.clear();
+      ctx->deferred.clear();
     }
     for (auto*& d : ctx->devs) {
       if (d) {
         d->destroy();
         delete d;
         d = nullptr;
-      }
-    }
-    for (auto*& m : ctx->mig_img) {
-      if (m) {
-        m->free_device();
-        m->free_host();
-        delete m;
-        m = nullptr;
       }
     }
     for (auto& c : g_signal_ctx) {
@@ -2293,21 +2489,23 @@ checl_status checl_release(checl_ctx* ctx, checl_handle h) {
       Entry& e = it->second;
       dev = e.device;
       if (!e.arena && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
-      if (e.arena && --e.arena->n_handles == 0) {  // the arena's last handle
+      if (e.arena && --e.arena->n_handles == 0) {  // the segment's last handle
         auto f = ctx->arenas.find(e.arena);
         drop = std::move(f->second);
         ctx->arenas.erase(f);
         if (drop->base) ctx->by_addr[drop->device].erase(reinterpret_cast<uintptr_t>(drop->base));
+        // a checkpoint / restore / migrate running on another thread may have planned
+        // reads of it: that call frees it when it ends (BusyGuard)
+        if (ctx->busy.load()) ctx->deferred.push_back(std::move(drop));
       }
       ctx->version[e.device]++;
       ctx->n_live[e.device]--;
       ctx->entries.erase(it);
     }
-    if (drop && drop.use_count() == 1) {
-      DeviceGuard g(dev);
-      ck(cudaDeviceSynchronize());
-    }
-    drop.reset();
+    (void)dev;
+    std::vector<std::shared_ptr<Arena>> v;
+    if (drop) v.push_back(std::move(drop));
+    free_arenas(v);  // (after the device is idle)
     return CHECL_SUCCESS;
   });
 }
@@ -2460,11 +2658,23 @@ checl_status checl_migrate(checl_ctx* ctx, int src_device, int dst_device, void*
   if (!b.ok) return CHECL_ERR_BUSY;
   return guarded([&]() -> checl_status {
     const double t0 = now_ms();
-    if (!ctx->mig_img[src_device]) ctx->mig_img[src_device] = new checl_image();
-    checl_image& img = *ctx->mig_img[src_device];
+    // m1: the image of src's buffers in src's HBM, allocated through the context's
+    // allocator and freed as soon as K2 on dst has read it (a move: the source GPU
+    // keeps nothing, L41 §IV-C), so it returns to the caller's memory pool
+    checl_image img;
+    img.dalloc = ctx->alloc;
+    img.dstream = stream_on(cuda_stream, src_device);
+    struct Drop {
+      checl_image& i;
+      ~Drop() {
+        i.free_device();
+        i.free_host();
+      }
+    } drop{img};
     checl_status st = do_checkpoint(ctx, src_device, cuda_stream, 0, &img, true);
     settle(ctx);
     checl_timing ck_t = ctx->last;
+    // m2-m3: verify + scatter on dst reading src's HBM over NVLink, rebind to dst
     if (st == CHECL_SUCCESS) st = do_restore(ctx, &img, dst_device, cuda_stream, rep, true);
     settle(ctx);
     std::lock_guard<std::mutex> lk(ctx->tmu);
@@ -2666,18 +2876,21 @@ static bool parallel_io(uint64_t n, F fn) {
 checl_status checl_image_write(const checl_image* img, const char* path, uint32_t flags) {
   if (!img || !path || flags & ~3u) return CHECL_ERR_INVALID_VALUE;
   return guarded([&]() -> checl_status {
-    const int bfd = ::open(path, O_WRONLY | O_CREAT | O_TRUNC, 0644);
+    // (read-write: a MAP_SHARED PROT_WRITE mapping needs a descriptor opened for reading too)
+    const int bfd = ::open(path, O_RDWR | O_CREAT | O_TRUNC, 0644);
     if (bfd < 0) return CHECL_ERR_INVALID_VALUE;
     int dfd = (flags & CHECL_IO_DIRECT) ? ::open(path, O_WRONLY | O_DIRECT) : -1;
     bool ok = true;
     if (img->location == CHECL_IMAGE_HOST && img->image_bytes) {
       const bool direct = dfd >= 0 && (reinterpret_cast<uintptr_t>(img->host) & 4095u) == 0;
-      // O_DIRECT: blocks allocated up front so the parallel pieces overwrite in place;
-      // mapping: only the size (pages are then allocated by the parallel copies)
-      if (!direct || posix_fallocate(bfd, 0, (off_t)img->image_bytes) != 0)
-        ok = ::ftruncate(bfd, (off_t)img->image_bytes) == 0;
+      // blocks allocated up front: the parallel pieces overwrite in place, and a page
+      // fault of the shared mapping below cannot run out of space (ENOSPC inside a
+      // mapping is SIGBUS, not an error return). Without the reservation the file is
+      // written with pwrite, whose errors come back as INVALID_VALUE.
+      const bool reserved = posix_fallocate(bfd, 0, (off_t)img->image_bytes) == 0;
+      if (!reserved) ok = ::ftruncate(bfd, (off_t)img->image_bytes) == 0;
       void* map = MAP_FAILED;
-      if (ok && !direct) map = ::mmap(nullptr, img->image_bytes, PROT_WRITE, MAP_SHARED, bfd, 0);
+      if (ok && !direct && reserved) map = ::mmap(nullptr, img->image_bytes, PROT_WRITE, MAP_SHARED, bfd, 0);
       if (!ok) {
       } else if (map != MAP_FAILED) {
         // page-cache / tmpfs target: parallel copies into the shared mapping (write(2)
@@ -2772,12 +2985,15 @@ checl_status checl_image_read(const char* path, uint32_t flags, checl_image** ou
 checl_status checl_trim(checl_ctx* ctx) {
   if (!ctx) return CHECL_ERR_INVALID_VALUE;
   return guarded([&]() -> checl_status {
-    std::shared_ptr<Arena> drop[kMaxDevices];
+    std::vector<std::shared_ptr<Arena>> drop;
     {
       std::lock_guard<std::mutex> lk(ctx->mu);
-      for (int d = 0; d < kMaxDevices; ++d) drop[d] = std::move(ctx->spare[d]);
+      for (int d = 0; d < kMaxDevices; ++d) {
+        for (auto& a : ctx->spares[d]) drop.push_back(std::move(a));
+        ctx->spares[d].clear();
+      }
     }
-    for (auto& a : drop) a.reset();
+    free_arenas(drop);
     pinned_pool().trim();
     return CHECL_SUCCESS;
   });

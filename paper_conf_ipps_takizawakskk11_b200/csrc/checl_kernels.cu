@@ -305,16 +305,22 @@ __device__ __forceinline__ void publish_status(const LaunchParams& p) {
   }
 }
 
+// diagnostics (experiments build only, CHECL_WARP_TRACE): lane 0 of every warp
+// records {start, tables ready, end}; the product build compiles both to nothing
+#ifdef CHECL_EXPERIMENTS
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
-// diagnostics: lane 0 of every warp records {start, tables ready, end}
 __device__ __forceinline__ void warp_trace(const LaunchParams& p, int k, unsigned long long t) {
   if (p.warp_trace && (threadIdx.x & 31) == 0)
     p.warp_trace[((uint64_t)blockIdx.x * kWarpsPerCta + (threadIdx.x >> 5)) * 4 + k] = t;
 }
+#else
+__device__ __forceinline__ unsigned long long gtimer() { return 0; }
+__device__ __forceinline__ void warp_trace(const LaunchParams&, int, unsigned long long) {}
+#endif
 
 template <int kOp>
 __device__ __forceinline__ void chunk_ptrs(const LaunchParams& p, const ChunkDesc& d, const uint8_t*& src,
@@ -1343,14 +1349,18 @@ static cudaError_t configure_op() {
   if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck)
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(tma_kernel<kOp, false>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmemBytes);
+#ifdef CHECL_EXPERIMENTS
   if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck)
     if (e == cudaSuccess)
       e = cudaFuncSetAttribute(tma_kernel<kOp, true>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kTmaSmemBytes);
+#endif
   return e;
 }
 
-// Kernel 4 as 2-CTA clusters with the multicast table prologue: CHECL_TABLE_MC=1
-// asks for it; used only if every SM can hold a CTA of a co-resident cluster.
+// Kernel 4 as 2-CTA clusters with the multicast table prologue (experiments build
+// only: measured no gain, profiles/r01o/table_mc_ab.txt): CHECL_TABLE_MC=1 asks for
+// it; used only if every SM can hold a CTA of a co-resident cluster.
+#ifdef CHECL_EXPERIMENTS
 static bool g_table_mc = false;
 
 static bool table_mc_possible() {
@@ -1375,6 +1385,9 @@ static bool table_mc_possible() {
   }
   return 2 * n >= (n_sms & ~1);
 }
+#else
+constexpr bool g_table_mc = false;
+#endif
 
 cudaError_t snapshot_configure() {
   cudaError_t e = configure_op<kOpPack>();
@@ -1383,10 +1396,12 @@ cudaError_t snapshot_configure() {
   if (e == cudaSuccess) e = configure_op<kOpCheck>();
   if (e == cudaSuccess) e = configure_op<kOpCopy>();
   if (e == cudaSuccess) e = configure_op<kOpScatter>();
+#ifdef CHECL_EXPERIMENTS
   if (e == cudaSuccess) {
     const char* m = std::getenv("CHECL_TABLE_MC");
     g_table_mc = m && std::atoi(m) != 0 && table_mc_possible();
   }
+#endif
   return e;
 }
 
@@ -1403,6 +1418,7 @@ static void launch_op(const LaunchParams& p, unsigned ctas, cudaStream_t s, int 
         tma_kernel<kOp, false><<<ctas, kThreadsPerCta, kTmaSmemBytes, s>>>(p);
         return;
       }
+#ifdef CHECL_EXPERIMENTS
       cudaLaunchConfig_t cfg = {};
       cfg.gridDim = dim3(ctas);
       cfg.blockDim = dim3(kThreadsPerCta);
@@ -1417,6 +1433,7 @@ static void launch_op(const LaunchParams& p, unsigned ctas, cudaStream_t s, int 
       cfg.numAttrs = 1;
       cudaLaunchKernelEx(&cfg, tma_kernel<kOp, true>, p);
       return;
+#endif
     }
   }
   if (kernel == 3 || kernel == 4)
@@ -1432,8 +1449,10 @@ static const void* op_fn(int kernel, size_t* smem) {
   if constexpr (kOp == kOpPack || kOp == kOpVerify || kOp == kOpCrc || kOp == kOpCheck) {
     if (kernel == 4) {
       *smem = kTmaSmemBytes;
-      return g_table_mc ? reinterpret_cast<const void*>(tma_kernel<kOp, true>)
-                        : reinterpret_cast<const void*>(tma_kernel<kOp, false>);
+#ifdef CHECL_EXPERIMENTS
+      if (g_table_mc) return reinterpret_cast<const void*>(tma_kernel<kOp, true>);
+#endif
+      return reinterpret_cast<const void*>(tma_kernel<kOp, false>);
     }
   }
   if (kernel == 3 || kernel == 4) {

@@ -12,6 +12,6 @@ def pytest_configure(config):
     # libchecl.so is an in-tree build artefact (git-ignored): make sure it exists so the
     # ABI tests exercise the real library. nvcc cross-compiles sm_100a without a GPU.
     import __graft_entry__
-    __graft_entry__._build_module().build()
+    __graft_entry__._build_module().build(experiments=True)
     config.addinivalue_line("markers", "gpu: needs a CUDA device (B200); run with -m gpu")
     config.addinivalue_line("markers", "slow: long-running")

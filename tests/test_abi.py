@@ -46,6 +46,20 @@ def test_library_is_sm100a(built):
     assert "sm_100a" in out
 
 
+def test_product_library_has_no_experiment_hooks(built):
+    """The A/B and tracing switches live only in the experiments build
+    (libchecl_exp.so, -DCHECL_EXPERIMENTS): the product library does not even contain
+    their names, so no environment variable can turn a checkpoint into an invalid
+    image or add tracing to the hot path."""
+    data = open(built, "rb").read()
+    for name in (b"CHECL_EXP_PACK_OP", b"CHECL_WARP_TRACE", b"CHECL_STAGE_TRACE", b"CHECL_TABLE_MC",
+                 b"CHECL_STATIC_PERMILLE", b"CHECL_DYN_BLOCK", b"CHECL_D2H_SPLIT"):
+        assert name not in data, name
+    from paper_conf_ipps_takizawakskk11_b200 import build
+    build.build(experiments=True)
+    assert b"CHECL_EXP_PACK_OP" in open(build.LIB_EXP, "rb").read()
+
+
 def test_python_binding_declares_every_export(built):
     from paper_conf_ipps_takizawakskk11_b200 import checl
     assert sorted(checl.EXPORTS) == declared_symbols()

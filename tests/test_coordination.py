@@ -95,3 +95,65 @@ def test_abort_keeps_caller_owned_reused_image():
     not freed, not returned, committed = False."""
     for rank, ok, f, nb, tb, same, freed, none in _run(2, "fail_keep"):
         assert not ok and f == 1 and none and not freed
+
+
+class FakeCtx:
+    """Stands in for checl.Context in coordinated_checkpoint: count() and
+    checkpoint(device, stream, epoch, into=None) (a new image or the reused one,
+    stamped with the epoch). Rank `fail_rank` fails its local checkpoint at the epochs
+    listed in `fail_at`."""
+
+    def __init__(self, rank, fail_rank, fail_at):
+        self.rank, self.fail_rank, self.fail_at = rank, fail_rank, fail_at
+        self.made = []
+
+    def count(self, device):
+        return 2, 64
+
+    def checkpoint(self, device, stream=None, epoch=0, into=None):
+        if self.rank == self.fail_rank and epoch in self.fail_at:
+            raise RuntimeError("local checkpoint failed")
+        img = into if into is not None else FakeImage()
+        if into is None:
+            self.made.append(img)
+        img.epoch = epoch
+        return img
+
+
+def _pair_worker(rank, world, port, q):
+    import torch.distributed as dist
+    from paper_conf_ipps_takizawakskk11_b200.coordination import ImagePair, coordinated_checkpoint
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    ctx = FakeCtx(rank, world - 1, {2, 3, 5})
+    pair = ImagePair()
+    log = []
+    for epoch in range(1, 7):
+        snap = coordinated_checkpoint(ctx, 0, epoch, into=pair)
+        c = pair.committed
+        log.append((epoch, snap.committed, c.epoch if c is not None else None, c.freed if c is not None else None))
+    q.put((rank, log, len(ctx.made)))
+    dist.destroy_process_group()
+
+
+def test_image_pair_keeps_last_committed_snapshot_on_abort():
+    """Double-buffered global snapshots (reading 16): every new
+    local snapshot goes into the image that does not hold the last committed one, so
+    after an aborted vote the committed image still holds the previous global
+    snapshot (epochs 2, 3 and 5 abort here: rank 1 fails), and only two images are
+    ever pinned per rank."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_pair_worker, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    out = sorted(q.get(timeout=120) for _ in range(2))
+    for p in ps:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    want = [(1, True, 1, False), (2, False, 1, False), (3, False, 1, False), (4, True, 4, False),
+            (5, False, 4, False), (6, True, 6, False)]
+    for rank, log, made in out:
+        assert log == want, (rank, log)
+        assert made <= 2 + (2 if rank == 0 else 0), made  # rank 0's aborted first-slot image is freed and re-made

@@ -100,6 +100,21 @@ def test_forced_kernel_shapes_bit_exact(kernel):
         dyn = dyn[:-1]
     if dyn:
         env.update(CHECL_STATIC_PERMILLE=dyn[0], CHECL_DYN_BLOCK=dyn[1], CHECL_DYN_MIN_ROUNDS="0")
+    if dyn or "CHECL_TABLE_MC" in env:  # those overrides exist only in the experiments build
+        env.update(CHECL_LIB=os.path.join(ROOT, "paper_conf_ipps_takizawakskk11_b200", "libchecl_exp.so"))
     r = subprocess.run([sys.executable, "-c", SCRIPT % ROOT], capture_output=True, text=True, env=env, cwd=ROOT,
                        timeout=600)
     assert r.returncode == 0 and "kernel ok" in r.stdout, r.stdout + r.stderr
+
+
+def test_product_build_ignores_experiment_hooks():
+    """The product library does not read the experiments build's A/B switches: with
+    CHECL_EXP_PACK_OP=2 (CRC-only pack, no valid image, in libchecl_exp.so) and the
+    dynamic-tail overrides set, libchecl.so still writes the oracle's image."""
+    env = dict(os.environ, CHECL_EXP_PACK_OP="2", CHECL_STATIC_PERMILLE="0", CHECL_DYN_BLOCK="1",
+               CHECL_DYN_MIN_ROUNDS="0", CHECL_TABLE_MC="1", CHECL_WARP_TRACE="1")
+    env.pop("CHECL_LIB", None)
+    r = subprocess.run([sys.executable, "-c", SCRIPT % ROOT], capture_output=True, text=True, env=env, cwd=ROOT,
+                       timeout=600)
+    assert r.returncode == 0 and "kernel ok" in r.stdout, r.stdout + r.stderr
+    assert "[checl] op" not in r.stderr  # no warp trace from the product library
