@@ -268,9 +268,11 @@ int oracle_validate(const uint8_t* img, size_t len, oracle_report* rep) {
       get_u32(img + 20) != O_ALIGN || get_u64(img + 40) != O_HEADER || flags > 1)
     return ORACLE_BAD_IMAGE;
   for (int i = 96; i < 124; ++i) {
-    int used = flags == 1 && ((i >= 96 && i < 108) || (i >= 112 && i < 120)); /* base_epoch, base_table_crc, n_present */
+    /* base_epoch, base_table_crc, dirty_rule, n_present */
+    int used = flags == 1 && ((i >= 96 && i < 108) || (i >= 108 && i < 112) || (i >= 112 && i < 120));
     if (!used && img[i] != 0) return ORACLE_BAD_IMAGE;
   }
+  if (flags == 1 && get_u32(img + 108) > 1) return ORACLE_BAD_IMAGE; /* dirty_rule 0 or 1 */
   uint64_t n = get_u64(img + 24), nch = get_u64(img + 32);
   uint64_t crc_off = get_u64(img + 48), payload_off = get_u64(img + 56);
   uint64_t payload_bytes = get_u64(img + 64), image_bytes = get_u64(img + 72);
@@ -400,12 +402,48 @@ static uint32_t table_crc_of(const uint8_t* img) {
 int oracle_checkpoint_incremental(const oracle_buffer* bufs, size_t n, int32_t device, uint64_t epoch,
                                   const uint8_t* base, size_t base_len, uint8_t* out, size_t out_cap,
                                   uint64_t* out_len) {
-  oracle_report brep;
+  return oracle_checkpoint_incremental_rule(bufs, n, device, epoch, base, base_len, NULL, 0, 0, out, out_cap,
+                                            out_len);
+}
+
+/* Is chunk j of manifest record b "updated" (FORMAT.md "Present set")?
+ * rule 0: its CRC32C in the table of `full` (now) differs from base's entry
+ *         (reading 21);
+ * rule 1: its bytes in `full` differ from its bytes in `base_full`, the full image of
+ *         the base's state (reading 25) — the plain definition of L45's
+ *         "updated since the last checkpoint". */
+static int chunk_updated(const uint8_t* full, const uint8_t* base, const uint8_t* base_full, uint32_t rule,
+                         uint64_t b, uint64_t j) {
+  uint64_t crc_off = get_u64(full + 48);
+  const uint8_t* r = full + O_HEADER + O_RECORD * b;
+  uint64_t k = get_u64(r + 24) + j;
+  if (rule == 0) return get_u32(full + crc_off + 4u * k) != get_u32(base + crc_off + 4u * k);
+  uint64_t size = get_u64(r + 8), off = get_u64(r + 16);
+  uint64_t lo = j * O_CHUNK;
+  uint64_t len = size - lo < O_CHUNK ? size - lo : O_CHUNK;
+  return memcmp(full + get_u64(full + 56) + off + lo, base_full + get_u64(base_full + 56) + off + lo, len) != 0;
+}
+
+int oracle_checkpoint_incremental_rule(const oracle_buffer* bufs, size_t n, int32_t device, uint64_t epoch,
+                                       const uint8_t* base, size_t base_len, const uint8_t* base_full,
+                                       size_t base_full_len, uint32_t dirty_rule, uint8_t* out, size_t out_cap,
+                                       uint64_t* out_len) {
+  oracle_report brep, frep;
   int st;
-  if (!out_len) return ORACLE_INVALID_VALUE;
+  if (!out_len || dirty_rule > 1) return ORACLE_INVALID_VALUE;
   /* the base must be a valid image (full or incremental) */
   st = oracle_validate(base, base_len, &brep);
   if (st) return st;
+  if (dirty_rule == 1) {
+    /* base_full: a valid full image of the base's state: same epoch, manifest and
+     * CRC table as the base */
+    if (!base_full || oracle_validate(base_full, base_full_len, &frep) || get_u32(base_full + 84) != 0)
+      return ORACLE_INVALID_VALUE;
+    uint64_t bco = get_u64(base + 48), bnch = get_u64(base + 32);
+    if (get_u64(base_full + 88) != get_u64(base + 88) || get_u64(base_full + 32) != bnch ||
+        get_u64(base_full + 48) != bco || memcmp(base_full + O_HEADER, base + O_HEADER, bco + 4u * bnch - O_HEADER) != 0)
+      return ORACLE_INVALID_VALUE;
+  }
 
   /* Step 1: the full image of the registry now (the definition of its content). */
   oracle_layout L;
@@ -434,16 +472,14 @@ int oracle_checkpoint_incremental(const oracle_buffer* bufs, size_t n, int32_t d
     return ORACLE_SUCCESS;
   }
 
-  /* Step 3: chunk k is present iff its CRC differs from the base's entry. */
+  /* Step 3: chunk k is present iff it was updated (chunk_updated, by the rule). */
   uint64_t nch = L.n_chunks, crc_off = L.crc_off;
   uint64_t map_bytes = nch / 8 + (nch % 8 ? 1 : 0);
   uint64_t n_present = 0, payload = 0;
   for (uint64_t b = 0; b < L.n_buffers; ++b) {
     uint64_t nb = chunks_of(get_u64(full + O_HEADER + O_RECORD * b + 8));
-    uint64_t first = get_u64(full + O_HEADER + O_RECORD * b + 24);
     for (uint64_t j = 0; j < nb; ++j) {
-      uint64_t k = first + j;
-      if (get_u32(full + crc_off + 4u * k) == get_u32(base + crc_off + 4u * k)) continue;
+      if (!chunk_updated(full, base, base_full, dirty_rule, b, j)) continue;
       uint64_t start, stop;
       chunk_span(full, L.n_buffers, b, j, L.payload_bytes, &start, &stop);
       n_present++;
@@ -474,6 +510,7 @@ int oracle_checkpoint_incremental(const oracle_buffer* bufs, size_t n, int32_t d
   put_u32(out + 84, 1);
   put_u64(out + 96, get_u64(base + 88));
   put_u32(out + 104, table_crc_of(base));
+  put_u32(out + 108, dirty_rule);
   put_u64(out + 112, n_present);
   memcpy(out + O_HEADER, full + O_HEADER, crc_off - O_HEADER);
   memcpy(out + crc_off, full + crc_off, 4u * nch);
@@ -484,7 +521,7 @@ int oracle_checkpoint_incremental(const oracle_buffer* bufs, size_t n, int32_t d
     uint64_t first = get_u64(full + O_HEADER + O_RECORD * b + 24);
     for (uint64_t j = 0; j < nb; ++j) {
       uint64_t k = first + j;
-      if (get_u32(full + crc_off + 4u * k) == get_u32(base + crc_off + 4u * k)) continue;
+      if (!chunk_updated(full, base, base_full, dirty_rule, b, j)) continue;
       uint64_t start, stop;
       chunk_span(full, L.n_buffers, b, j, L.payload_bytes, &start, &stop);
       map[k / 8] |= (uint8_t)(1u << (k % 8));

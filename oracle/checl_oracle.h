@@ -89,7 +89,8 @@ int oracle_restore(const uint8_t* img, size_t len, uint8_t* out_bytes,
 /* ---- Incremental images (FORMAT.md "Incremental images") ----
  * PAPER.md L45 §IV-D (future work): "only the OpenCL objects updated since the
  * last checkpoint need to be written". Unit = 64 KiB chunk; updated = its CRC32C
- * differs from the base image's entry (reading 21). */
+ * differs from the base image's entry (reading 21), or, with dirty rule 1,
+ * its bytes differ from the base state's (reading 25). */
 
 /* Writes into out[0, *out_len) the incremental image of the registry at `epoch`
  * relative to `base` (a full or incremental image). When base's manifest, chunk
@@ -99,6 +100,20 @@ int oracle_restore(const uint8_t* img, size_t len, uint8_t* out_bytes,
 int oracle_checkpoint_incremental(const oracle_buffer* bufs, size_t n, int32_t device, uint64_t epoch,
                                   const uint8_t* base, size_t base_len, uint8_t* out, size_t out_cap,
                                   uint64_t* out_len);
+
+/* Same, with the rule that decides which chunks were updated (FORMAT.md "Present
+ * set", written to the delta's dirty_rule field):
+ *   0: the chunk's CRC32C differs from base's CRC-table entry (reading 21;
+ *      base_full unused, may be NULL) — oracle_checkpoint_incremental;
+ *   1: the chunk's bytes differ from its bytes in the base's state (DESIGN.md reading
+ *      25). base_full = the full image of that state: base itself when base is full,
+ *      else merge(...merge(F, D1)..., base). It must validate, be full, and carry
+ *      base's epoch, manifest and CRC table (ORACLE_INVALID_VALUE otherwise).
+ * ORACLE_INVALID_VALUE also for a rule > 1. */
+int oracle_checkpoint_incremental_rule(const oracle_buffer* bufs, size_t n, int32_t device, uint64_t epoch,
+                                       const uint8_t* base, size_t base_len, const uint8_t* base_full,
+                                       size_t base_full_len, uint32_t dirty_rule, uint8_t* out, size_t out_cap,
+                                       uint64_t* out_len);
 
 /* merge(F, D): the full image of D's epoch from full image F and delta D whose
  * link names F. ORACLE_BAD_IMAGE if either does not validate, F is not full, D is

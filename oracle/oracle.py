@@ -164,26 +164,36 @@ def _sigs_incremental(L):
         return L
     L.oracle_checkpoint_incremental.argtypes = [C.POINTER(_Buf), C.c_size_t, C.c_int32, C.c_uint64, C.c_void_p,
                                                 C.c_size_t, C.c_void_p, C.c_size_t, C.POINTER(C.c_uint64)]
+    L.oracle_checkpoint_incremental_rule.argtypes = [C.POINTER(_Buf), C.c_size_t, C.c_int32, C.c_uint64, C.c_void_p,
+                                                     C.c_size_t, C.c_void_p, C.c_size_t, C.c_uint32, C.c_void_p,
+                                                     C.c_size_t, C.POINTER(C.c_uint64)]
     L.oracle_merge.argtypes = [C.c_void_p, C.c_size_t, C.c_void_p, C.c_size_t, C.c_void_p, C.c_size_t,
                                C.POINTER(C.c_uint64)]
     L._incr = True
     return L
 
 
-def checkpoint_incremental(entries: Sequence[Entry], base, device: int = 0, epoch: int = 0) -> np.ndarray:
+RULE_CRC, RULE_BYTES = 0, 1  # FORMAT.md "Present set" (readings 21 and 25)
+
+
+def checkpoint_incremental(entries: Sequence[Entry], base, device: int = 0, epoch: int = 0, rule: int = RULE_CRC,
+                           base_full=None) -> np.ndarray:
     """Incremental image of the registry relative to `base` (FORMAT.md "Incremental
-    images"); the full image when the layout differs from the base's."""
+    images"); the full image when the layout differs from the base's. rule=RULE_BYTES
+    needs base_full, the full image of the base's state (base itself when full)."""
     L = _sigs_incremental(lib())
     arr, keep = _bufs(entries, device)
     b = _u8(base)
+    f = _u8(base_full) if base_full is not None else None
+    fp, fn = (f.ctypes.data if f is not None and f.size else None), (f.size if f is not None else 0)
     need = C.c_uint64(0)
-    st = L.oracle_checkpoint_incremental(arr, len(entries), device, epoch, b.ctypes.data if b.size else None, b.size,
-                                         None, 0, C.byref(need))
+    st = L.oracle_checkpoint_incremental_rule(arr, len(entries), device, epoch, b.ctypes.data if b.size else None,
+                                              b.size, fp, fn, rule, None, 0, C.byref(need))
     if st != INVALID_VALUE or need.value == 0:  # cap 0: reports the size it needs
         raise ValueError(f"oracle_checkpoint_incremental status {st}")
     out = np.empty(max(1, need.value), dtype=np.uint8)
-    st = L.oracle_checkpoint_incremental(arr, len(entries), device, epoch, b.ctypes.data if b.size else None, b.size,
-                                         out.ctypes.data, out.size, C.byref(need))
+    st = L.oracle_checkpoint_incremental_rule(arr, len(entries), device, epoch, b.ctypes.data if b.size else None,
+                                              b.size, fp, fn, rule, out.ctypes.data, out.size, C.byref(need))
     if st:
         raise ValueError(f"oracle_checkpoint_incremental status {st}")
     return out[: need.value]

@@ -1,5 +1,9 @@
 """Pins for the incremental-checkpoint oracle (PAPER.md L45
 §IV-D "only the OpenCL objects updated since the last checkpoint"), -m "not gpu".
+Two rules decide "updated" (FORMAT.md "Present set"): the CRC rule (DESIGN.md
+reading 21) and the bytes rule (reading 25, the plain definition; pinned at the end
+by byte differences computed here with numpy and by merge == full image even for a
+change the CRC cannot see).
 
 Checked against things other than the oracle's own incremental code: an
 independent reading of FORMAT.md "Incremental images" (header fields, bitmap,
@@ -50,7 +54,8 @@ def _spans(ents):
     return out
 
 
-def _check_delta_by_definition(delta: np.ndarray, base: np.ndarray, new_full: np.ndarray, ents_now, present):
+def _check_delta_by_definition(delta: np.ndarray, base: np.ndarray, new_full: np.ndarray, ents_now, present,
+                               rule: int = 0):
     """Independent reading of FORMAT.md "Incremental images"."""
     d, f, b = delta.tobytes(), new_full.tobytes(), base.tobytes()
     nch, crc_off = struct.unpack_from("<QQ", f, 32)[0], struct.unpack_from("<Q", f, 48)[0]
@@ -60,7 +65,7 @@ def _check_delta_by_definition(delta: np.ndarray, base: np.ndarray, new_full: np
     assert d[80:84] == f[80:84] and d[88:96] == f[88:96]  # device, epoch
     flags, = struct.unpack_from("<I", d, 84)
     base_epoch, base_tab, res1, n_present, res2 = struct.unpack_from("<QIIQI", d, 96)
-    assert (flags, res1, res2) == (1, 0, 0)
+    assert (flags, res1, res2) == (1, rule, 0)  # res1 = dirty_rule
     assert base_epoch == struct.unpack_from("<Q", b, 88)[0]
     assert base_tab == _crc(b[crc_off: crc_off + 4 * nch])
     map_bytes = (nch + 7) // 8
@@ -233,3 +238,137 @@ def test_crc_blind_change_is_not_in_the_delta():
     F = O.checkpoint([O.Entry(1, data)], epoch=0)
     D = O.checkpoint_incremental([O.Entry(1, data ^ delta_bytes)], F, epoch=1)
     assert struct.unpack_from("<Q", D.tobytes(), 112)[0] == 0  # not present
+
+
+# ---- dirty rule 1: a chunk is updated iff its bytes differ (reading 25) ----
+
+def _crc_blind_delta(n=64):
+    """A non-zero change vector whose CRC32C difference is zero (GF(2) elimination
+    over the CRC's linear map restricted to the first 40 bits)."""
+    base = np.zeros(n, np.uint8)
+    c0 = O.crc32c(base)
+    pivots, combo = {}, None
+    for i in range(40):
+        e = base.copy()
+        e[i // 8] ^= 1 << (i % 8)
+        v, mask = O.crc32c(e) ^ c0, 1 << i
+        while v:
+            hb = v.bit_length() - 1
+            if hb not in pivots:
+                pivots[hb] = (v, mask)
+                break
+            pv, pm = pivots[hb]
+            v ^= pv
+            mask ^= pm
+        if v == 0:
+            combo = mask
+            break
+    d = np.zeros(n, np.uint8)
+    for i in range(40):
+        if combo >> i & 1:
+            d[i // 8] ^= 1 << (i % 8)
+    return d
+
+
+def _byte_present(old_ents, new_ents):
+    """Chunks whose bytes differ, by FORMAT.md's chunking, computed here with numpy."""
+    out, k = [], 0
+    for a, b in zip(sorted(old_ents, key=lambda e: e.handle), sorted(new_ents, key=lambda e: e.handle)):
+        for j in range((a.data.size + 65535) // 65536):
+            if not np.array_equal(a.data[65536 * j:65536 * (j + 1)], b.data[65536 * j:65536 * (j + 1)]):
+                out.append(k)
+            k += 1
+    return out
+
+
+def test_bytes_rule_writes_the_crc_blind_change():
+    """The change the CRC rule misses (test_crc_blind_change_is_not_in_the_delta) is
+    present under the bytes rule, and merge(F, D) is the full image of the new state,
+    byte for byte; under the CRC rule the merge keeps the stale bytes."""
+    d = _crc_blind_delta()
+    rng = np.random.default_rng(31)
+    data = rng.integers(0, 256, 70000, dtype=np.uint8)
+    now = data.copy()
+    now[65536:65536 + d.size] ^= d  # inside chunk 1
+    assert O.crc32c(now[65536:]) == O.crc32c(data[65536:])
+    F = O.checkpoint([O.Entry(1, data)], epoch=0)
+    F2 = O.checkpoint([O.Entry(1, now)], epoch=1)
+    D = O.checkpoint_incremental([O.Entry(1, now)], F, epoch=1, rule=O.RULE_BYTES, base_full=F)
+    _check_delta_by_definition(D, F, F2, [O.Entry(1, now)], [1], rule=1)
+    st, M = O.merge(F, D)
+    assert st == 0 and np.array_equal(M, F2)
+    Dc = O.checkpoint_incremental([O.Entry(1, now)], F, epoch=1, rule=O.RULE_CRC)
+    st, Mc = O.merge(F, Dc)
+    assert st == 0 and not np.array_equal(Mc, F2)  # the CRC rule's documented miss
+
+
+def test_bytes_rule_present_set_is_the_byte_difference():
+    rng = np.random.default_rng(32)
+    for trial in range(40):
+        sizes = [int(x) for x in rng.choice(SIZES + [200003, 1], size=int(rng.integers(1, 4)))]
+        handles = sorted(rng.choice(np.arange(1, 100), size=len(sizes), replace=False).tolist())
+        ents = [O.Entry(int(h), rng.integers(0, 256, s, dtype=np.uint8), trial) for h, s in zip(handles, sizes)]
+        changes = []
+        for i, s in enumerate(sizes):
+            for _ in range(int(rng.integers(0, 4)) if s else 0):
+                changes.append((i, int(rng.integers(0, s)), int(rng.integers(1, 256))))
+        if changes and trial % 3 == 0:  # a change undone by a second one: bytes equal again
+            i, pos, x = changes[0]
+            changes.append((i, pos, x))
+        now = _mutate(ents, changes)
+        F = O.checkpoint(ents, device=3, epoch=trial)
+        F2 = O.checkpoint(now, device=3, epoch=trial + 1)
+        D = O.checkpoint_incremental(now, F, device=3, epoch=trial + 1, rule=O.RULE_BYTES, base_full=F)
+        _check_delta_by_definition(D, F, F2, now, _byte_present(ents, now), rule=1)
+        st, M = O.merge(F, D)
+        assert st == 0 and np.array_equal(M, F2)
+
+
+def test_bytes_rule_chain_with_delta_base():
+    """A delta as the base: base_full is the merge of its chain."""
+    rng = np.random.default_rng(33)
+    s0 = [O.Entry(h, rng.integers(0, 256, n, dtype=np.uint8)) for h, n in [(1, 300000), (2, 5), (3, 131072)]]
+    d = _crc_blind_delta()
+    s1 = _mutate(s0, [(0, 70000, 1), (2, 3, 9)])
+    s2 = [O.Entry(e.handle, e.data.copy(), e.flags) for e in s1]
+    s2[0].data[131072:131072 + d.size] ^= d  # CRC-blind, in chunk 2 of buffer 1
+    F0 = O.checkpoint(s0, epoch=0)
+    D1 = O.checkpoint_incremental(s1, F0, epoch=1, rule=O.RULE_BYTES, base_full=F0)
+    st, M1 = O.merge(F0, D1)
+    assert st == 0
+    D2 = O.checkpoint_incremental(s2, D1, epoch=2, rule=O.RULE_BYTES, base_full=M1)
+    assert struct.unpack_from("<Q", D2.tobytes(), 112)[0] == 1
+    st, rep, back = O.restore_chain([F0, D1, D2])
+    assert st == 0 and all(np.array_equal(a.data, b.data) for a, b in zip(back, s2))
+    st, M2 = O.merge(M1, D2)
+    assert st == 0 and np.array_equal(M2, O.checkpoint(s2, epoch=2))
+
+
+def test_bytes_rule_needs_the_base_state():
+    rng = np.random.default_rng(34)
+    s0 = [O.Entry(1, rng.integers(0, 256, 1000, dtype=np.uint8))]
+    s1 = _mutate(s0, [(0, 5, 1)])
+    F0 = O.checkpoint(s0, epoch=0)
+    F1 = O.checkpoint(s1, epoch=1)
+    with pytest.raises(ValueError):  # no base state
+        O.checkpoint_incremental(s1, F0, epoch=2, rule=O.RULE_BYTES)
+    with pytest.raises(ValueError):  # the state of another epoch
+        O.checkpoint_incremental(s1, F0, epoch=2, rule=O.RULE_BYTES, base_full=F1)
+    with pytest.raises(ValueError):  # no such rule
+        O.checkpoint_incremental(s1, F0, epoch=2, rule=2, base_full=F0)
+
+
+def test_dirty_rule_field_validation():
+    """FORMAT.md: a delta's dirty_rule (offset 108) is 0 or 1; anything else is
+    BAD_IMAGE even with a correct meta CRC (recomputed here with the hardware crc32)."""
+    rng = np.random.default_rng(35)
+    s0 = [O.Entry(1, rng.integers(0, 256, 100000, dtype=np.uint8))]
+    F = O.checkpoint(s0, epoch=0)
+    D = O.checkpoint_incremental(_mutate(s0, [(0, 1, 1)]), F, epoch=1, rule=O.RULE_BYTES, base_full=F)
+    assert O.validate(D)[0] == 0 and struct.unpack_from("<I", D.tobytes(), 108)[0] == 1
+    poff = struct.unpack_from("<Q", D.tobytes(), 56)[0]
+    for v, want in ((0, 0), (2, O.BAD_IMAGE), (0xFFFFFFFF, O.BAD_IMAGE)):
+        bad = bytearray(D.tobytes())
+        struct.pack_into("<I", bad, 108, v)
+        struct.pack_into("<I", bad, 124, _crc(bytes(bad[:124]) + bytes(bad[128:poff])))
+        assert O.validate(np.frombuffer(bytes(bad), np.uint8))[0] == want, v
