@@ -56,6 +56,8 @@ def parse():
     ap.add_argument("--mode", default="snapshot", choices=["snapshot", "incremental"],
                     help="incremental: checl_checkpoint_incremental with --dirty of the chunks rewritten per step")
     ap.add_argument("--dirty", type=float, default=0.1)
+    ap.add_argument("--rule", default="bytes", choices=["bytes", "crc"],
+                    help="incremental dirty rule: bytes (exact, default) or crc (fast option)")
     return ap.parse_args()
 
 
@@ -392,6 +394,7 @@ def run_incremental(a):
         torch.cuda.synchronize()
 
     cur = torch.cuda.current_stream(dev)
+    rule = checl.DIRTY_BYTES if a.rule == "bytes" else checl.DIRTY_CRC
 
     def timed(fn):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -419,12 +422,12 @@ def run_incremental(a):
 
     for i in range(a.warmup):
         mutate()
-        advance(ctx.checkpoint_incremental(dev, base, epoch=i + 1))
+        advance(ctx.checkpoint_incremental(dev, base, epoch=i + 1, rule=rule))
     ms_steps, drained, present, tms = [], [], [], []
     with ClockSampler(dev) as clk:
         for i in range(a.steps):
             mutate()
-            ms, d = timed(lambda: ctx.checkpoint_incremental(dev, base, epoch=a.warmup + i + 1))
+            ms, d = timed(lambda: ctx.checkpoint_incremental(dev, base, epoch=a.warmup + i + 1, rule=rule))
             h = d.header()
             ms_steps.append(ms)
             drained.append(h["payload_bytes"])
@@ -435,7 +438,7 @@ def run_incremental(a):
     # restore [merge(full@now), ...] instead: take a fresh full and one delta
     f2 = ctx.checkpoint(dev, epoch=100)
     mutate()
-    d2 = ctx.checkpoint_incremental(dev, f2, epoch=101)
+    d2 = ctx.checkpoint_incremental(dev, f2, epoch=101, rule=rule)
     rs_ms, rep = timed(lambda: ctx.restore_chain([f2, d2], dev))
     n_diff = 0
     for h, t in zip(range(1, len(tensors) + 1), tensors):
@@ -451,11 +454,13 @@ def run_incremental(a):
         "value": S / (t_inc * 1e-3) / 1e9, "unit": "GB/s", "n_gpus": 1, "steps": a.steps, "warmup": a.warmup,
         "ms_per_step": t_inc, "ms_per_step_all": ms_steps, "higher_is_better": True, "dtype": "u8", "data": "synthetic",
         "config": {"workload": w.name, "payload_bytes_per_gpu": S, "n_chunks": len(starts),
-                   "dirty_fraction": a.dirty, "chunks_rewritten_per_step": k},
+                   "dirty_fraction": a.dirty, "chunks_rewritten_per_step": k, "dirty_rule": a.rule},
         "full_checkpoint_ms": t_full, "speedup_vs_full": t_full / t_inc,
         "drained_bytes_per_step": statistics.mean(drained), "present_chunks_per_step": statistics.mean(present),
         "kernel_ms_per_step": crc_ms,
-        "crc_pass": {"bytes_read": S, "note": "kOpCrc reads S; gather reads + writes only the present spans"},
+        "dirty_pass": ({"bytes_read": 2 * S, "note": "diff_kernel reads S (buffers) + S (shadow), writes the "
+                        "changed rounds; gather + CRC of the present spans only"} if a.rule == "bytes" else
+                       {"bytes_read": S, "note": "kOpCrc reads S; gather reads + writes only the present spans"}),
         "last_timing": tms[-1], "chain_restore_ms": rs_ms, "chain_restore_GBs": S / (rs_ms * 1e-3) / 1e9,
         "verified": n_diff == 0 and rep.n_bad_chunks == 0, "clocks": clk.summary(), "hbm_peak": hbm}))
     ctx.close()

@@ -37,6 +37,7 @@ ERR_BUSY = -10
 IMAGE_HOST, IMAGE_DEVICE = 0, 1
 IO_DIRECT, IO_SYNC = 1, 2
 FILL_RANDOM, FILL_FLOAT, FILL_ZEROS = 0, 1, 2
+DIRTY_CRC, DIRTY_BYTES = 0, 1  # incremental checkpoint dirty rules (checl.h, FORMAT.md "Present set")
 
 EXPORTS = (
     "checl_create", "checl_destroy", "checl_set_staging", "checl_register_buffer", "checl_release",
@@ -44,7 +45,7 @@ EXPORTS = (
     "checl_image_view", "checl_image_info", "checl_image_wrap", "checl_image_to_host", "checl_image_free",
     "checl_restore", "checl_migrate", "checl_last_timing", "checl_status_string", "checl_last_cuda_error",
     "checl_version", "checl_debug_fill", "checl_debug_compare", "checl_debug_corrupt",
-    "checl_checkpoint_incremental", "checl_restore_chain", "checl_image_merge",
+    "checl_checkpoint_incremental", "checl_checkpoint_incremental_ex", "checl_restore_chain", "checl_image_merge",
     "checl_request_checkpoint", "checl_checkpoint_pending", "checl_install_signal", "checl_sync_point",
     "checl_image_write", "checl_image_read", "checl_trim", "checl_stats_get", "checl_stats_reset",
 )
@@ -107,6 +108,7 @@ def _load() -> C.CDLL:
         "checl_debug_compare": [C.c_int, V, V, SZ, C.POINTER(U64)],
         "checl_debug_corrupt": [P, U64, C.c_uint8],
         "checl_checkpoint_incremental": [P, C.c_int, V, U64, P, PP],
+        "checl_checkpoint_incremental_ex": [P, C.c_int, V, U64, P, U32, PP],
         "checl_restore_chain": [P, C.POINTER(C.c_void_p), U32, C.c_int, V, C.POINTER(_Report)],
         "checl_image_merge": [P, P, PP],
         "checl_request_checkpoint": [P],
@@ -223,7 +225,7 @@ class Image:
         h = {"n_buffers": u64(24), "n_chunks": u64(32), "crc_off": u64(48), "payload_off": u64(56),
              "payload_bytes": u64(64), "image_bytes": u64(72), "device": u32(80), "flags": u32(84), "epoch": u64(88)}
         if h["flags"] == 1:
-            h.update(base_epoch=u64(96), base_table_crc=u32(104), n_present=u64(112))
+            h.update(base_epoch=u64(96), base_table_crc=u32(104), dirty_rule=u32(108), n_present=u64(112))
         return h
 
     def write(self, path: str, direct: bool = True, sync: bool = False):
@@ -385,12 +387,15 @@ class Context:
                "checl_checkpoint_device")
         return Image(out.value)
 
-    def checkpoint_incremental(self, device: int, base: Image, stream=None, epoch: int = 0) -> Image:
+    def checkpoint_incremental(self, device: int, base: Image, stream=None, epoch: int = 0,
+                               rule: int = DIRTY_BYTES) -> Image:
         """Incremental checkpoint (L45 future work; FORMAT.md "Incremental images"):
-        only chunks whose CRC32C differs from `base`'s table are drained."""
+        only the updated chunks are drained — rule DIRTY_BYTES (default, exact): the
+        chunks whose bytes differ from `base`'s state; DIRTY_CRC (fast option): the
+        chunks whose CRC32C differs from `base`'s table."""
         out = C.c_void_p()
-        _check(lib.checl_checkpoint_incremental(self._p, device, _stream_ptr(stream), epoch, base.handle, C.byref(out)),
-               "checl_checkpoint_incremental")
+        _check(lib.checl_checkpoint_incremental_ex(self._p, device, _stream_ptr(stream), epoch, base.handle, rule,
+                                                   C.byref(out)), "checl_checkpoint_incremental_ex")
         return Image(out.value)
 
     def restore_chain(self, chain, device: int, stream=None) -> Report:

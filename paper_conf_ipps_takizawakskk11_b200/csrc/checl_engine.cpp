@@ -41,8 +41,12 @@ cudaError_t launch_build_tables(const TableParams& tp, uint32_t* out, cudaStream
 cudaError_t launch_fill(uint8_t* ptr, uint64_t bytes, uint64_t key, int kind, int n_sms, cudaStream_t s);
 cudaError_t launch_compare(const uint8_t* a, const uint8_t* b, uint64_t bytes, unsigned long long* n_diff, int n_sms,
                            cudaStream_t s);
-cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, const uint32_t* crc_base, uint64_t n,
-                              uint32_t* map_words, ChunkDesc* cdesc, unsigned long long* totals, cudaStream_t s);
+cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, const uint32_t* crc_base,
+                              const uint32_t* dirty, uint64_t n, uint32_t* map_words, ChunkDesc* cdesc, uint32_t* cidx,
+                              unsigned long long* totals, cudaStream_t s);
+cudaError_t launch_diff(const ChunkDesc* desc, uint64_t n, uint8_t* shadow, uint32_t* dirty, int n_sms, cudaStream_t s);
+cudaError_t launch_crc_scatter(const uint32_t* ccrc, const uint32_t* cidx, const unsigned long long* totals,
+                               uint64_t n_max, uint32_t* table, int n_sms, cudaStream_t s);
 cudaError_t launch_delta_stages(const ChunkDesc* cdesc, const unsigned long long* totals, uint64_t W, uint64_t n_stages,
                                 unsigned long long* first, unsigned long long* lo, cudaStream_t s);
 cudaError_t launch_expand(const BufferRecord* recs, uint32_t n, uint64_t payload_bytes, uint64_t n_chunks,
@@ -389,6 +393,15 @@ struct DevState {
   DevBuf<ChunkDesc> cdesc;
   DevBuf<unsigned long long> dtotals, stage_first, stage_lo;
   PinnedBuf<unsigned long long> h_dtab;
+  // exact incremental checkpoint (dirty rule 1, reading 25): the shadow holds
+  // the payload of the state a checkpoint last described (payload layout), identified by
+  // that image's epoch, CRC-table CRC and manifest CRC; dirty bits, the compacted
+  // chunks' CRCs and global indices
+  DevBuf<uint8_t> shadow;
+  bool shadow_ok = false;
+  uint64_t shadow_epoch = 0, shadow_payload = 0;
+  uint32_t shadow_table_crc = 0, shadow_meta_crc = 0;
+  DevBuf<uint32_t> dirty, ccrc, cidx;
   // 1 = warp per chunk (throughput), 2 = 4 KiB units swept by the grid (latency of
   // small launches), 3 = balanced stretches of rounds, 4 = balanced stretches with
   // bulk (TMA) copies and the column CRC; 0 = by plan; env
@@ -460,6 +473,10 @@ struct DevState {
     map_words.release();
     cdesc.release();
     dtotals.release();
+    shadow.release();
+    dirty.release();
+    ccrc.release();
+    cidx.release();
     stage_first.release();
     stage_lo.release();
     h_dtab.release();
@@ -890,7 +907,7 @@ checl_status parse_image(const uint8_t* img, size_t len, bool meta_only, Parsed*
   if (flags == 0) {
     for (int i = 96; i < 124; ++i)
       if (img[i]) return CHECL_ERR_BAD_IMAGE;
-  } else if (get_u32(img + 108) != 0 || get_u32(img + 120) != 0) {
+  } else if (get_u32(img + 108) > 1 || get_u32(img + 120) != 0) {  // dirty_rule 0 (CRC) or 1 (bytes)
     return CHECL_ERR_BAD_IMAGE;
   }
   const uint64_t n = get_u64(img + 24), nch = get_u64(img + 32);
@@ -2058,8 +2075,29 @@ bool same_layout(const uint8_t* base, const Parsed& B, const Plan& P, int device
          std::memcmp(base + kHeaderBytes, P.meta.data() + kHeaderBytes, P.crc_off - kHeaderBytes) == 0;
 }
 
+// The shadow of `device` now holds the payload of the full state `host_payload` (a full
+// host image's payload) / `dev_payload` (a device image's); identified like the image.
+void seed_shadow(DevState& ds, const Plan& P, const uint8_t* host_payload, const checl_image* dimg, uint64_t epoch,
+                 uint32_t table_crc, uint32_t meta_crc_v) {
+  ds.shadow_ok = false;
+  ds.shadow.ensure(std::max<uint64_t>(P.payload_bytes, 1));
+  if (P.payload_bytes) {
+    if (host_payload)
+      ck(cudaMemcpyAsync(ds.shadow.p, host_payload, P.payload_bytes, cudaMemcpyHostToDevice, ds.compute));
+    else if (dimg->device == ds.dev)
+      ck(cudaMemcpyAsync(ds.shadow.p, dimg->d_payload, P.payload_bytes, cudaMemcpyDeviceToDevice, ds.compute));
+    else
+      ck(cudaMemcpyPeerAsync(ds.shadow.p, ds.dev, dimg->d_payload, dimg->device, P.payload_bytes, ds.compute));
+  }
+  ds.shadow_epoch = epoch;
+  ds.shadow_table_crc = table_crc;
+  ds.shadow_meta_crc = meta_crc_v;
+  ds.shadow_payload = P.payload_bytes;
+  ds.shadow_ok = true;
+}
+
 checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream, uint64_t epoch,
-                                       const checl_image* base, checl_image* img) {
+                                       const checl_image* base, checl_image* img, uint32_t rule) {
   // r1-style validation of the base's metadata (header, manifest, CRC table, bitmap)
   Parsed B;
   checl_status st = parse_image(base->host, base->location == CHECL_IMAGE_DEVICE ? base->payload_off : base->image_bytes,
@@ -2069,10 +2107,36 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   DeviceGuard g(device);
   DevState& ds = ctx->dev(device);
   const uint64_t aux0 = ds.aux_launches;
+  const bool exact = rule == CHECL_DIRTY_BYTES;
+  uint32_t mcrc = 0, tcrc = 0;
   {
     // the plan (and so the layout test) needs the registry as of this call
     Plan& P0 = get_plan(ctx, ds, device);
-    if (!same_layout(base->host, B, P0, device)) return do_checkpoint(ctx, device, stream, epoch, img, false);
+    const bool same = same_layout(base->host, B, P0, device);
+    if (exact) {
+      mcrc = host_crc32c(P0.meta.data() + kHeaderBytes, P0.crc_off - kHeaderBytes);
+      tcrc = host_crc32c(base->host + B.L.crc_off, 4 * B.L.n_chunks);
+    }
+    const bool have_state = ds.shadow_ok && ds.shadow_epoch == B.epoch && ds.shadow_table_crc == tcrc &&
+                            ds.shadow_meta_crc == mcrc && ds.shadow_payload == P0.payload_bytes;
+    if (!same || (exact && !have_state && B.flags != 0)) {
+      // a layout change, or (bytes rule) a delta base whose state the device does not
+      // hold: the full image, which is a valid result of any incremental checkpoint
+      st = do_checkpoint(ctx, device, stream, epoch, img, false);
+      if (st == CHECL_SUCCESS && exact) {  // its state becomes the shadow (next delta: exact)
+        Plan& P1 = get_plan(ctx, ds, device);
+        seed_shadow(ds, P1, img->host + P1.payload_off, nullptr, epoch, host_crc32c(img->host + P1.crc_off, 4 * P1.n_chunks),
+                    host_crc32c(P1.meta.data() + kHeaderBytes, P1.crc_off - kHeaderBytes));
+        ck(cudaStreamSynchronize(ds.compute));
+      }
+      return st;
+    }
+    if (exact && !have_state) {  // a full base: its payload becomes the shadow
+      if (base->location == CHECL_IMAGE_DEVICE)
+        seed_shadow(ds, P0, nullptr, base, B.epoch, tcrc, mcrc);
+      else
+        seed_shadow(ds, P0, base->host + B.L.payload_off, nullptr, B.epoch, tcrc, mcrc);
+    }
   }
   begin_events(ctx, ds);
   KernelTimer kt;
@@ -2096,23 +2160,43 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   ds.stage_first.ensure(max_stages + 1);
   ds.stage_lo.ensure(max_stages + 1);
   ds.h_dtab.ensure(2 + 2 * (max_stages + 1));
+  if (exact) {
+    ds.dirty.ensure(std::max<uint64_t>((n + 31) / 32, 1));
+    ds.ccrc.ensure(std::max<uint64_t>(n, 1));
+    ds.cidx.ensure(std::max<uint64_t>(n, 1));
+  }
   tm.plan_ms = now_ms() - tp;
 
-  // CRC of every chunk as it is now (kOpCrc: read-only pass), then the present set,
-  // the compacted chunk list and the stage table (delta_scan / delta_stages)
+  // The present set:
+  //  CRC rule: CRC of every chunk as it is now (kOpCrc: read-only pass) vs base's table;
+  //  bytes rule: every chunk compared with the shadow (diff_kernel, which also brings
+  //  the shadow up to date); then the compacted chunk list and the stage table
+  //  (delta_scan / delta_stages)
   LaunchParams lp = base_params(ds);
   lp.desc = P.d_desc.p;
   lp.round_base = P.d_round.p;
   lp.crc = ds.crc_scratch.p;
   lp.c0 = 0;
   lp.c1 = n;
-  if (n) ck(cudaMemcpyAsync(ds.base_crc.p, base->host + B.L.crc_off, 4 * n, cudaMemcpyHostToDevice, ds.compute));
-  if (n) timed_launch(ds, kt, kOpCrc, lp, ds.compute);
-  cudaEvent_t sa = ds.events.get(), sb = ds.events.get();
-  ck(cudaEventRecord(sa, ds.compute));
-  ds.aux_launches += 2;
-  ck(launch_delta_scan(P.d_desc.p, ds.crc_scratch.p, ds.base_crc.p, n, ds.map_words.p, ds.cdesc.p, ds.dtotals.p,
+  if (n)
+    ck(cudaMemcpyAsync(exact ? ds.crc_scratch.p : ds.base_crc.p, base->host + B.L.crc_off, 4 * n, cudaMemcpyHostToDevice,
                        ds.compute));
+  cudaEvent_t sa = ds.events.get(), sb = ds.events.get();
+  if (exact) {
+    ds.shadow_ok = false;  // (advanced in place below; valid again once the delta is written)
+    ck(cudaEventRecord(sa, ds.compute));
+    ck(cudaMemsetAsync(ds.dirty.p, 0, 4 * ((n + 31) / 32), ds.compute));
+    ds.aux_launches += 3;
+    ck(launch_diff(P.d_desc.p, n, ds.shadow.p, ds.dirty.p, ds.n_sms, ds.compute));
+    ck(launch_delta_scan(P.d_desc.p, nullptr, nullptr, ds.dirty.p, n, ds.map_words.p, ds.cdesc.p, ds.cidx.p, ds.dtotals.p,
+                         ds.compute));
+  } else {
+    if (n) timed_launch(ds, kt, kOpCrc, lp, ds.compute);
+    ck(cudaEventRecord(sa, ds.compute));
+    ds.aux_launches += 2;
+    ck(launch_delta_scan(P.d_desc.p, ds.crc_scratch.p, ds.base_crc.p, nullptr, n, ds.map_words.p, ds.cdesc.p, nullptr,
+                         ds.dtotals.p, ds.compute));
+  }
   ck(launch_delta_stages(ds.cdesc.p, ds.dtotals.p, W, max_stages, ds.stage_first.p, ds.stage_lo.p, ds.compute));
   ck(cudaEventRecord(sb, ds.compute));
   kt.spans.push_back({sa, sb});
@@ -2136,8 +2220,9 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   }
   img->ensure_host(image_bytes, true);
 
-  // a3 + a4 over the present chunks only: gather (kOpCopy, the CRCs are known)
-  // into slot s % n_slots while the copy engine drains the previous slot
+  // a3 + a4 over the present chunks only: gather into slot s % n_slots while the copy
+  // engine drains the previous slot (CRC rule: kOpCopy, the CRCs are known; bytes rule:
+  // kOpPack, the CRC of each present chunk into ccrc, scattered into the table after)
   ds.ensure_slots(ctx->slot_bytes, ctx->n_slots);
   std::vector<cudaEvent_t> packed(ds.n_slots), drained(ds.n_slots);
   for (uint32_t i = 0; i < ds.n_slots; ++i) {
@@ -2148,6 +2233,7 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   ck(cudaEventRecord(c_begin, ds.copy));
   lp.desc = ds.cdesc.p;
   lp.round_base = nullptr;  // compacted list: grid-stride kernels
+  if (exact) lp.crc = ds.ccrc.p;
   size_t used = 0;
   for (uint64_t s = 0; s < max_stages; ++s) {
     if (first[s] == first[s + 1]) continue;
@@ -2157,7 +2243,7 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
     lp.c1 = first[s + 1];
     lp.image = ds.slot(k);
     lp.image_base = lo[s];
-    timed_launch(ds, kt, kOpCopy, lp, ds.compute);
+    timed_launch(ds, kt, exact ? kOpPack : kOpCopy, lp, ds.compute);
     ck(cudaEventRecord(packed[k], ds.compute));
     ck(cudaStreamWaitEvent(ds.copy, packed[k], 0));
     d2h_page_aligned(img->host_mut + payload_off + lo[s], ds.slot(k), lo[s + 1] - lo[s], ds.copy);
@@ -2165,6 +2251,13 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
     ++used;
   }
   if (n) {
+    if (exact) {  // the base's table with the present chunks' new CRCs
+      ++ds.aux_launches;
+      ck(launch_crc_scatter(ds.ccrc.p, ds.cidx.p, ds.dtotals.p, n_present, ds.crc_scratch.p, ds.n_sms, ds.compute));
+      cudaEvent_t tab = ds.events.get();
+      ck(cudaEventRecord(tab, ds.compute));
+      ck(cudaStreamWaitEvent(ds.copy, tab, 0));
+    }
     ck(cudaMemcpyAsync(img->host_mut + P.crc_off, ds.crc_scratch.p, 4 * n, cudaMemcpyDeviceToHost, ds.copy));
     ck(cudaMemcpyAsync(img->host_mut + P.crc_off + 4 * n, ds.map_words.p, map_bytes, cudaMemcpyDeviceToHost, ds.copy));
   }
@@ -2182,12 +2275,17 @@ checl_status do_checkpoint_incremental(checl_ctx* ctx, int device, void* stream,
   put_u32(o + 84, 1);
   put_u64(o + 88, epoch);
   put_u64(o + 96, B.epoch);
-  put_u32(o + 104, host_crc32c(base->host + B.L.crc_off, 4 * n));
-  put_u32(o + 108, 0);
+  put_u32(o + 104, exact ? tcrc : host_crc32c(base->host + B.L.crc_off, 4 * n));
+  put_u32(o + 108, rule);
   put_u64(o + 112, n_present);
   put_u32(o + 120, 0);
   std::memset(o + P.crc_off + 4 * n + map_bytes, 0, payload_off - P.crc_off - 4 * n - map_bytes);
   put_u32(o + 124, meta_crc(o, payload_off));
+  if (exact) {  // the shadow now holds this image's state
+    ds.shadow_epoch = epoch;
+    ds.shadow_table_crc = host_crc32c(o + P.crc_off, 4 * n);
+    ds.shadow_ok = true;
+  }
   tm.commit_ms = now_ms() - tf;
   img->image_bytes = image_bytes;
   img->payload_off = payload_off;
@@ -2692,12 +2790,19 @@ checl_status checl_migrate(checl_ctx* ctx, int src_device, int dst_device, void*
 
 checl_status checl_checkpoint_incremental(checl_ctx* ctx, int device, void* cuda_stream, uint64_t epoch,
                                           const checl_image* base, checl_image** out) {
-  if (!ctx || !out || !base || !base->host) return CHECL_ERR_INVALID_VALUE;
+  return checl_checkpoint_incremental_ex(ctx, device, cuda_stream, epoch, base, CHECL_DIRTY_BYTES, out);
+}
+
+checl_status checl_checkpoint_incremental_ex(checl_ctx* ctx, int device, void* cuda_stream, uint64_t epoch,
+                                             const checl_image* base, uint32_t dirty_rule, checl_image** out) {
+  if (!ctx || !out || !base || !base->host || dirty_rule > CHECL_DIRTY_BYTES) return CHECL_ERR_INVALID_VALUE;
   if (!valid_device(device)) return CHECL_ERR_INVALID_DEVICE;
   checl_image* img = new (std::nothrow) checl_image();
   if (!img) return CHECL_ERR_OUT_OF_HOST_MEMORY;
   BusyGuard b(ctx);
-  checl_status st = b.ok ? guarded([&]() { return do_checkpoint_incremental(ctx, device, cuda_stream, epoch, base, img); })
+  checl_status st = b.ok ? guarded([&]() {
+    return do_checkpoint_incremental(ctx, device, cuda_stream, epoch, base, img, dirty_rule);
+  })
                          : CHECL_ERR_BUSY;
   if (st) {
     checl_image_free(img);

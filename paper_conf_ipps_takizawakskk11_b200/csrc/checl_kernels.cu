@@ -1246,11 +1246,89 @@ __global__ void expand_plan_kernel(const BufferRecord* __restrict__ recs, uint32
 // ballot writes 32 bitmap bits per warp, a block scan of (span, present) gives
 // each present chunk its compacted offset and index, and the chunk's descriptor is
 // re-emitted with the compacted offset (same ptr / len / pad).
+// Exact dirty test (FORMAT.md dirty rule 1, reading 25). `shadow` holds the
+// base state's payload in payload layout (chunk c at img_off_256 * 256). Unit u =
+// (chunk u / 16, 4 KiB round u % 16), one warp per unit, grid-stride: the round's
+// bytes in the registered buffer are compared with the shadow's; when they differ the
+// round is copied into the shadow (which so becomes the current state) and the
+// chunk's bit is set in dirty[c / 32] (zero before the launch). A pure stream: read S
+// from the buffers + S from the shadow, write the changed rounds.
+__global__ void __launch_bounds__(256) diff_kernel(const ChunkDesc* __restrict__ desc, uint64_t n,
+                                                   uint8_t* __restrict__ shadow, uint32_t* __restrict__ dirty) {
+  const int lane = threadIdx.x & 31;
+  const unsigned full = 0xFFFFFFFFu;
+  const uint64_t nwarps = (uint64_t)gridDim.x * (blockDim.x >> 5);
+  for (uint64_t u = (uint64_t)blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5); u < n * 16; u += nwarps) {
+    const uint64_t c = u >> 4;
+    const uint32_t r = (uint32_t)(u & 15u) * (uint32_t)kRoundBytes;
+    const ChunkDesc d = desc[c];
+    const uint32_t len = desc_len(d);
+    if (r >= len) continue;
+    const uint32_t nb = len - r < (uint32_t)kRoundBytes ? len - r : (uint32_t)kRoundBytes;
+    const uint8_t* src = reinterpret_cast<const uint8_t*>(d.ptr) + r;
+    uint8_t* sh = shadow + (uint64_t)d.img_off_256 * kBufferAlign + r;
+    bool diff = false;
+    if ((reinterpret_cast<uintptr_t>(src) & 15u) == 0) {
+      // 16-byte granules (each warp instruction = 512 contiguous bytes), then the tail
+      const uint32_t ng = nb >> 4;
+      uint4 a[8], b[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const uint32_t g = (uint32_t)lane + 32u * k;
+        if (g < ng) {
+          a[k] = __ldg(reinterpret_cast<const uint4*>(src) + g);
+          b[k] = *(reinterpret_cast<const uint4*>(sh) + g);
+        }
+      }
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const uint32_t g = (uint32_t)lane + 32u * k;
+        if (g < ng) diff |= a[k].x != b[k].x || a[k].y != b[k].y || a[k].z != b[k].z || a[k].w != b[k].w;
+      }
+      const uint32_t t = (ng << 4) + (uint32_t)lane;
+      uint8_t tb = 0;
+      if (t < nb) {
+        tb = src[t];
+        diff |= tb != sh[t];
+      }
+      if (__any_sync(full, diff)) {
+#pragma unroll
+        for (int k = 0; k < 8; ++k) {
+          const uint32_t g = (uint32_t)lane + 32u * k;
+          if (g < ng) *(reinterpret_cast<uint4*>(sh) + g) = a[k];
+        }
+        if (t < nb) sh[t] = tb;
+        if (lane == 0) atomicOr(&dirty[c >> 5], 1u << (c & 31));
+      }
+    } else {  // a misaligned registration (a tensor view with a storage offset): bytes
+      for (uint32_t i = (uint32_t)lane; i < nb; i += 32) diff |= src[i] != sh[i];
+      if (__any_sync(full, diff)) {
+        for (uint32_t i = (uint32_t)lane; i < nb; i += 32) sh[i] = src[i];
+        if (lane == 0) atomicOr(&dirty[c >> 5], 1u << (c & 31));
+      }
+    }
+  }
+}
+
+// CRC table of an exact delta: entry cidx[k] of `table` (the base's table) takes the
+// CRC computed for present chunk k (ccrc[k], from the gather launches), k < totals[0].
+__global__ void crc_scatter_kernel(const uint32_t* __restrict__ ccrc, const uint32_t* __restrict__ cidx,
+                                   const unsigned long long* __restrict__ totals, uint32_t* __restrict__ table) {
+  const uint64_t np = totals[0];
+  for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < np; k += (uint64_t)gridDim.x * blockDim.x)
+    table[cidx[k]] = ccrc[k];
+}
+
+// Present set -> bitmap words, compacted chunk list (img_off = offset in the compacted
+// payload), [n_present, compacted bytes], and optionally the global index of each
+// present chunk (cidx). Present: dirty[c/32] bit set when `dirty` is given (bytes
+// rule), else crc_now[c] != crc_base[c] (CRC rule). One CTA, chunks in order.
 __global__ void __launch_bounds__(1024, 1) delta_scan_kernel(const ChunkDesc* __restrict__ desc,
                                                              const uint32_t* __restrict__ crc_now,
-                                                             const uint32_t* __restrict__ crc_base, uint64_t n,
+                                                             const uint32_t* __restrict__ crc_base,
+                                                             const uint32_t* __restrict__ dirty, uint64_t n,
                                                              uint32_t* __restrict__ map_words,
-                                                             ChunkDesc* __restrict__ cdesc,
+                                                             ChunkDesc* __restrict__ cdesc, uint32_t* __restrict__ cidx,
                                                              unsigned long long* __restrict__ totals) {
   __shared__ unsigned long long w_bytes[32];
   __shared__ uint32_t w_cnt[32];
@@ -1260,7 +1338,7 @@ __global__ void __launch_bounds__(1024, 1) delta_scan_kernel(const ChunkDesc* __
   __syncthreads();
   for (uint64_t base = 0; base < n; base += 1024) {
     const uint64_t i = base + threadIdx.x;
-    const bool present = i < n && crc_now[i] != crc_base[i];
+    const bool present = i < n && (dirty ? ((dirty[i >> 5] >> (i & 31)) & 1u) != 0 : crc_now[i] != crc_base[i]);
     ChunkDesc d{};
     if (present) d = desc[i];
     const unsigned long long span = present ? (unsigned long long)(desc_len(d) + desc_pad(d)) : 0ull;
@@ -1297,6 +1375,7 @@ __global__ void __launch_bounds__(1024, 1) delta_scan_kernel(const ChunkDesc* __
       o.img_off_256 = (uint32_t)(off / kBufferAlign);
       o.len_pad = d.len_pad;
       cdesc[idx] = o;
+      if (cidx) cidx[idx] = (uint32_t)i;
     }
     __syncthreads();
     if (threadIdx.x == 1023) carry_bytes = off + span, carry_cnt = idx + (present ? 1u : 0u);
@@ -1512,9 +1591,28 @@ cudaError_t launch_snapshot(int op, const LaunchParams& p, int n_sms, cudaStream
   return cudaGetLastError();
 }
 
-cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, const uint32_t* crc_base, uint64_t n,
-                              uint32_t* map_words, ChunkDesc* cdesc, unsigned long long* totals, cudaStream_t s) {
-  delta_scan_kernel<<<1, 1024, 0, s>>>(desc, crc_now, crc_base, n, map_words, cdesc, totals);
+cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, const uint32_t* crc_base,
+                              const uint32_t* dirty, uint64_t n, uint32_t* map_words, ChunkDesc* cdesc, uint32_t* cidx,
+                              unsigned long long* totals, cudaStream_t s) {
+  delta_scan_kernel<<<1, 1024, 0, s>>>(desc, crc_now, crc_base, dirty, n, map_words, cdesc, cidx, totals);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_diff(const ChunkDesc* desc, uint64_t n, uint8_t* shadow, uint32_t* dirty, int n_sms,
+                        cudaStream_t s) {
+  if (n == 0) return cudaSuccess;
+  uint64_t blocks = (n * 16 + 7) / 8;  // 8 warps per CTA, one unit each per pass
+  if (blocks > (uint64_t)n_sms * 8) blocks = (uint64_t)n_sms * 8;
+  diff_kernel<<<(unsigned)blocks, 256, 0, s>>>(desc, n, shadow, dirty);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_crc_scatter(const uint32_t* ccrc, const uint32_t* cidx, const unsigned long long* totals,
+                               uint64_t n_max, uint32_t* table, int n_sms, cudaStream_t s) {
+  if (n_max == 0) return cudaSuccess;
+  uint64_t blocks = (n_max + 255) / 256;
+  if (blocks > (uint64_t)n_sms * 4) blocks = (uint64_t)n_sms * 4;
+  crc_scatter_kernel<<<(unsigned)blocks, 256, 0, s>>>(ccrc, cidx, totals, table);
   return cudaGetLastError();
 }
 
