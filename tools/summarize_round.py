@@ -1,6 +1,6 @@
 """Write the judged summaries of one GPU session into profiles/<round>/ and
 profiles/traffic.json (per-launch DRAM bytes of K1/K2 from the ncu --set full capture).
-usage: python tools/summarize_round.py <gpurun_out/tag> <profiles/rNN>"""
+usage: python tools/summarize_round.py <gpurun_out/tag> <profiles/rNN> [config of prof.ncu-rep, default C3]"""
 import csv
 import io
 import json
@@ -14,6 +14,7 @@ sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 from ncu_summary import summary  # noqa: E402
 
 src, dst = sys.argv[1], sys.argv[2]
+CFG = sys.argv[3] if len(sys.argv) > 3 else "C3"
 os.makedirs(dst, exist_ok=True)
 import glob  # noqa: E402
 for f in sorted(glob.glob(os.path.join(src, "bench*.json"))) + [
@@ -40,7 +41,7 @@ if os.path.exists(lc):
 rep = os.path.join(src, "prof.ncu-rep")
 traffic = {}
 if os.path.exists(rep):
-    lines += ["## ncu --set full (C2, device-resident image; tools/profile_step.py)", ""]
+    lines += [f"## ncu --set full ({CFG}, device-resident image; tools/profile_step.py)", ""]
     for d in summary(rep):
         name = d.pop("kernel")
         st = d.pop("stalls_per_issue")
@@ -60,14 +61,14 @@ if os.path.exists(rep):
 if os.path.exists(os.path.join(src, "bench.json")):
     try:
         b = json.loads(open(os.path.join(src, "bench.json")).read().strip().splitlines()[-1])
-        lines = ["## bench.py (C2, N=1)", "", "```", json.dumps({k: b[k] for k in ("value", "unit", "ms_per_step", "roofline", "e2e", "clocks", "cpu_baseline") if k in b}, indent=1), "```", ""] + lines
+        lines = [f"## bench.py ({b['config']['workload']}, N=1)", "", "```", json.dumps({k: b[k] for k in ("value", "unit", "ms_per_step", "roofline", "e2e", "clocks", "cpu_baseline", "extras") if k in b}, indent=1), "```", ""] + lines
     except Exception as e:
         lines.insert(0, f"(bench.json unreadable: {e})")
 open(os.path.join(dst, "SUMMARY.md"), "w").write("# GPU session summary\n\n" + "\n".join(lines) + "\n")
 if traffic:
     tp = os.path.join(os.path.dirname(dst.rstrip("/")), "traffic.json")
     cur = json.load(open(tp)) if os.path.exists(tp) else {}
-    cur["C2"] = {"dram_bytes_per_launch": max(traffic.values()), "K1": traffic.get("K1"), "K2": traffic.get("K2"),
+    cur[CFG] = {"dram_bytes_per_launch": max(traffic.values()), "K1": traffic.get("K1"), "K2": traffic.get("K2"),
                  "source": f"{dst}/SUMMARY.md (ncu --set full dram__bytes_read.sum + dram__bytes_write.sum)"}
     json.dump(cur, open(tp, "w"), indent=1)
 print(open(os.path.join(dst, "SUMMARY.md")).read()[:3000])
