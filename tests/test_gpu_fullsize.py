@@ -1,12 +1,16 @@
 """-m gpu: configs[3] (C4, SHOC-MD-shaped rank, 64 GiB) at full size on one B200.
 
 Checkpoint to a pinned host image, then restore into re-created buffers; the image
-header/manifest/CRC table are checked against the oracle's layout and meta CRC, and
-sampled chunks (random ones plus every buffer's short tail chunk) against the
-oracle's CRC32C and the synth generator's bytes; restored buffers are compared on
-the same samples (full sizes are checked on samples
-the oracle computes one by one).
+header/manifest/CRC table are checked against the oracle's layout and meta CRC;
+EVERY one of the 1,048,578 CRC-table entries against the x86 SSE4.2 crc32
+instruction's CRC32C of its chunk (tests/helpers: independent of the oracle and of
+the product, fast enough for 64 GiB), the whole payload against the buffers' bytes
+read back with plain copies, and sampled chunks (random ones plus every buffer's
+short tail chunk) against the oracle's CRC32C and the synth generator's bytes;
+restored buffers are compared on the same samples.
 """
+from concurrent.futures import ThreadPoolExecutor
+
 import struct
 
 import numpy as np
@@ -21,9 +25,37 @@ if not torch.cuda.is_available():
     pytest.skip("needs a CUDA device", allow_module_level=True)
 
 from paper_conf_ipps_takizawakskk11_b200 import checl  # noqa: E402
+from tests.helpers import hwcrc  # noqa: E402
+
+PIECE = 1 << 30  # bytes per host piece (a multiple of the 64 KiB chunk)
 
 
-def test_c4_md_rank_full_size_sampled():
+def _chunk_crcs(host: np.ndarray, n: int) -> np.ndarray:
+    """CRC32C (SSE4.2) of the 64 KiB chunks of host[:n], 8 threads."""
+    offs = np.arange(0, n, 65536, dtype=np.uint64)
+    lens = np.minimum(65536, n - offs).astype(np.uint64)
+    parts = np.array_split(np.arange(offs.size), 8)
+    with ThreadPoolExecutor(8) as ex:
+        res = list(ex.map(lambda ix: hwcrc.hw_crc32c_many(host, offs[ix], lens[ix]), parts))
+    return np.concatenate(res) if res else np.zeros(0, np.uint32)
+
+
+def _full_table_and_payload_check(recs, crcs, dev_bytes_of, img_payload_of):
+    """Every CRC entry = hw CRC32C of its chunk of the buffer's bytes (read back with a
+    plain copy, dev_bytes_of(bi, lo, n)); with img_payload_of, the image's payload of
+    every buffer equals those bytes."""
+    for bi, (h, size, off, first, fl, dv, _) in enumerate(recs):
+        for lo in range(0, size, PIECE):
+            n = min(PIECE, size - lo)
+            data = dev_bytes_of(bi, lo, n)
+            hw = _chunk_crcs(data, n)
+            k0 = first + lo // 65536
+            assert np.array_equal(hw, crcs[k0:k0 + hw.size]), (bi, lo, int(np.count_nonzero(hw != crcs[k0:k0 + hw.size])))
+            if img_payload_of is not None:
+                assert np.array_equal(img_payload_of(off + lo, n), data), (bi, lo)
+
+
+def test_c4_md_rank_full_size():
     w = synth.c4_md_rank(0)
     S = w.total_bytes
     free, _ = torch.cuda.mem_get_info(0)
@@ -45,6 +77,10 @@ def test_c4_md_rank_full_size_sampled():
     assert st == 0 and rep["n_chunks"] == 1048578
     recs = [struct.unpack_from("<QQQQIiQ", got, 128 + 48 * i) for i in range(3)]
     crcs = np.frombuffer(got, dtype="<u4", count=L["n_chunks"], offset=L["crc_off"])
+    if hwcrc.available():
+        _full_table_and_payload_check(
+            recs, crcs, lambda bi, lo, n: tensors[bi][lo:lo + n].cpu().numpy(),
+            lambda o, n: got[L["payload_off"] + o:L["payload_off"] + o + n])
     rng = np.random.default_rng(44)
     samples = []
     for bi, (h, size, off, first, fl, dv, _) in enumerate(recs):
@@ -80,7 +116,7 @@ def _device_bytes(ptr: int, n: int) -> np.ndarray:
     return torch.as_tensor(_Iface(), device="cuda:0").cpu().numpy()
 
 
-def test_c4_full_size_device_image_restart_sampled():
+def test_c4_full_size_device_image_restart():
     """configs[3] at full size in bench.py's launch configuration: HBM-resident image,
     restart mode (every handle released, restore re-creates the buffers). The image
     metadata mirror, sampled CRC table entries and payload chunks are checked against
@@ -108,6 +144,17 @@ def test_c4_full_size_device_image_restart_sampled():
     recs = [struct.unpack_from("<QQQQIiQ", meta, 128 + 48 * i) for i in range(3)]
     crcs = np.frombuffer(meta, dtype="<u4", count=L["n_chunks"], offset=L["crc_off"])
     pay = img.info()["device_payload"]
+    if hwcrc.available():
+        # the whole CRC table against the buffers; the HBM payload against them on the
+        # device (torch.equal: a plain comparison, not the library's)
+        _full_table_and_payload_check(recs, crcs, lambda bi, lo, n: tensors[bi][lo:lo + n].cpu().numpy(), None)
+        for bi, (h, size, off, first, fl, dv, _) in enumerate(recs):
+            for lo in range(0, size, PIECE):
+                n = min(PIECE, size - lo)
+                class _I:
+                    __cuda_array_interface__ = {"shape": (n,), "typestr": "|u1", "data": (pay + off + lo, False),
+                                                "version": 2, "strides": None}
+                assert torch.equal(torch.as_tensor(_I(), device="cuda:0"), tensors[bi][lo:lo + n]), (bi, lo)
     rng = np.random.default_rng(45)
     samples = []
     for bi, (h, size, off, first, fl, dv, _) in enumerate(recs):
