@@ -7,7 +7,7 @@ that split buffers across stages), then checks: the host image equals the oracle
 byte for byte, the HBM image's metadata mirror equals it too, restore from both
 reproduces every buffer, a random single-bit payload flip is reported at the
 oracle's chunk, and an incremental image after random rewrites equals the
-oracle's delta."""
+oracle's delta (exact rule on even cases, CRC rule on odd ones)."""
 import os
 
 import numpy as np
@@ -90,7 +90,13 @@ def test_random_registry(case):
             live[i][p:p + 1].bitwise_xor_(0x21)
             ds.host[i][p] ^= 0x21
     torch.cuda.synchronize()
-    d = ctx.checkpoint_incremental(DEV, img, epoch=epoch + 1)
-    assert np.array_equal(d.view(), O.checkpoint_incremental(oracle_entries(ds), want, device=DEV, epoch=epoch + 1))
+    if case % 2:  # the CRC rule (reading 21)
+        d = ctx.checkpoint_incremental(DEV, img, epoch=epoch + 1, rule=checl.DIRTY_CRC)
+        want_d = O.checkpoint_incremental(oracle_entries(ds), want, device=DEV, epoch=epoch + 1)
+    else:  # the exact rule (default; reading 25): the base's state is the full image `want`
+        d = ctx.checkpoint_incremental(DEV, img, epoch=epoch + 1)
+        want_d = O.checkpoint_incremental(oracle_entries(ds), want, device=DEV, epoch=epoch + 1, rule=O.RULE_BYTES,
+                                          base_full=want)
+    assert np.array_equal(d.view(), want_d)
     release_all(ctx, ds)
     ctx.close()
