@@ -360,6 +360,16 @@ struct Plan {
   std::vector<BufferRecord> recs;
   std::vector<Stage> stages;
   std::vector<uint8_t> meta;  // header (meta_crc = 0, epoch = 0) + manifest
+  // the CRC32C register after meta's header bytes [0, 124) and manifest [128, crc_off)
+  // (epoch 0), and x^(8 (crc_off - 100)): the shift of the epoch bytes to the end of
+  // the manifest (finalize adds the epoch by linearity instead of re-reading the
+  // manifest); meta_gen changes whenever meta is rebuilt
+  uint32_t meta_state0 = 0, epoch_shift = 0;
+  uint64_t meta_gen = 0;
+  // the restore layout (LayoutCache::gen) the plan's buffers were re-created with, and
+  // the segments its chunk list addresses (0 / empty: built from the registry)
+  uint64_t layout_gen = 0;
+  std::vector<void*> list_bases;
   DevBuf<ChunkDesc> d_desc;
   DevBuf<uint32_t> d_round;  // round_base of the balanced kernel (n_chunks + 1)
   DevBuf<BufferRecord> d_recs;
@@ -375,10 +385,11 @@ struct DevState {
   DevBuf<ChunkDesc> desc_scratch;
   DevBuf<uint32_t> round_scratch;
   DevBuf<BufferRecord> recs_scratch;
-  // what desc_scratch / round_scratch hold: the expansion of these records (valid
-  // iff scratch_payload != ~0); a restore whose records match skips its expansion
-  std::vector<BufferRecord> scratch_recs;
-  uint64_t scratch_payload = ~0ull;
+  // what desc_scratch / round_scratch hold: the chunk list of layout scratch_gen over
+  // the segments at scratch_bases (0: nothing known); a restore with the same key
+  // skips its expansion
+  uint64_t scratch_gen = 0;
+  std::vector<void*> scratch_bases;
   // verify status {first bad, n bad, CTAs done}; between restores it rests at
   // {~0, 0, 0} (reset by the publishing launch) unless status_clean is false
   DevBuf<unsigned long long> status;
@@ -522,6 +533,8 @@ struct Arena {
   }
 };
 
+struct LayoutCache;
+
 struct Entry {
   int device;
   uint8_t* ptr;
@@ -561,6 +574,9 @@ struct checl_image {
   // device address of host_mut (mapped pinned memory), cached: nullptr = not known yet
   const uint8_t* mapped_for = nullptr;
   uint8_t* mapped_dev = nullptr;
+  // host_mut[128, crc_off) holds the manifest of plan generation meta_gen
+  bool meta_valid = false;
+  uint64_t meta_gen = 0;
 
   void* dev_alloc(size_t n) {  // on the current device (= `device`); nullptr on failure
     if (dalloc.alloc) return dalloc.alloc(n, device, dstream, dalloc.user);
@@ -601,6 +617,7 @@ struct checl_image {
     }
     host = host_mut = nullptr;
     host_cap = 0;
+    meta_valid = false;
   }
   void ensure_host(size_t n, bool want_pinned) {
     if (owned && host_mut && host_cap >= n && pinned == want_pinned) return;
@@ -619,6 +636,7 @@ struct checl_image {
     host = host_mut = static_cast<uint8_t*>(p);
     host_cap = cap;
     pinned = want_pinned;
+    meta_valid = false;
   }
 };
 
@@ -671,6 +689,17 @@ struct checl_ctx {
   // arenas whose last handle was released while a checkpoint / restore / migrate ran
   // (its plan may still read them): freed when that call ends (BusyGuard)
   std::vector<std::shared_ptr<Arena>> deferred;
+  // per device: the layout of its last full-image restore (restore fast path)
+  std::unique_ptr<LayoutCache> layout[kMaxDevices];
+  // the bindings of the last commit: its entries in manifest order (map nodes are
+  // stable) and the segments they point into; a commit of the same layout onto the
+  // same device with the registry unchanged since (version) rebinds them in place
+  struct BindCache {
+    int device = -1;
+    uint64_t gen = 0, version = 0;
+    std::vector<Entry*> entries;
+    std::vector<Arena*> arenas;
+  } bind;
 
   DevState& dev(int d) {
     if (!devs[d]) {
@@ -983,6 +1012,15 @@ checl_status parse_image(const uint8_t* img, size_t len, bool meta_only, Parsed*
 
 // -- checkpoint -------------------------------------------------------------------
 
+std::atomic<uint64_t> g_meta_gen{0};  // process-wide: a generation names one manifest
+
+void plan_meta_state(Plan& P) {
+  P.meta_state0 = host_crc32c_update(0xFFFFFFFFu, P.meta.data(), 124);
+  P.meta_state0 = host_crc32c_update(P.meta_state0, P.meta.data() + kHeaderBytes, P.crc_off - kHeaderBytes);
+  P.epoch_shift = gf_x8n(P.crc_off - 100);  // bytes after the epoch's last one: header 96..123 + manifest
+  P.meta_gen = ++g_meta_gen;
+}
+
 // Builds (or reuses) the plan of `device` under the context lock.
 Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
   std::lock_guard<std::mutex> lk(ctx->mu);
@@ -1006,6 +1044,7 @@ Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
   P.meta.assign(L.crc_off, 0);
   write_header(P.meta.data(), L, P.bufs.size(), device, 0);
   write_manifest(P.meta.data() + kHeaderBytes, P.bufs, device);
+  plan_meta_state(P);
   P.d_desc.ensure(std::max<uint64_t>(L.n_chunks, 1));
   P.d_round.ensure(L.n_chunks + 1);
   P.d_recs.ensure(std::max<size_t>(P.recs.size(), 1));
@@ -1019,6 +1058,8 @@ Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
   }
   P.version = ctx->version[device];
   P.slot_bytes = ctx->slot_bytes;
+  P.layout_gen = 0;
+  P.list_bases.clear();
   return P;
 }
 
@@ -1262,13 +1303,29 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
 #endif
 }
 
-// Writes header + manifest + meta_crc into the image's host bytes [0, payload_off);
-// the CRC table must already be there.
-void finalize_meta(uint8_t* host, const Plan& P, uint64_t epoch) {
-  std::memcpy(host, P.meta.data(), P.crc_off);
+// a5, first half (while K1 runs): header and manifest into the image's host bytes (the
+// manifest only when the image does not hold this plan's already), the zero pad after
+// the CRC table, and the meta CRC register after header + manifest: the plan's
+// epoch-0 register plus the epoch bytes' term, R(e, 0) * x^(8 (crc_off - 100)) (CRC
+// linearity; DESIGN.md §5 "Finalize"). Nothing DMAs into [0, crc_off) or the pad.
+uint32_t prefinalize(checl_image* img, const Plan& P, uint64_t epoch) {
+  uint8_t* host = img->host_mut;
+  if (!img->meta_valid || img->meta_gen != P.meta_gen) {
+    std::memcpy(host + kHeaderBytes, P.meta.data() + kHeaderBytes, P.crc_off - kHeaderBytes);
+    img->meta_valid = true;
+    img->meta_gen = P.meta_gen;
+  }
+  std::memcpy(host, P.meta.data(), kHeaderBytes);
   put_u64(host + 88, epoch);
   std::memset(host + P.crc_off + 4 * P.n_chunks, 0, P.payload_off - P.crc_off - 4 * P.n_chunks);
-  put_u32(host + 124, meta_crc(host, P.payload_off));
+  uint8_t e[8];
+  put_u64(e, epoch);
+  return P.meta_state0 ^ gf_mul(host_crc32c_update(0u, e, 8), P.epoch_shift);
+}
+
+// a5, second half (the CRC table has landed): the meta CRC over the table and the pad.
+void finalize_meta(uint8_t* host, const Plan& P, uint32_t state) {
+  put_u32(host + 124, ~host_crc32c_update(state, host + P.crc_off, P.payload_off - P.crc_off));
 }
 
 // -- deferred timing (checl_ctx::PendingTiming) -----------------------------------
@@ -1380,6 +1437,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
   tm.plan_ms = now_ms() - tp;
 
   cudaEvent_t c_begin = ds.events.get(), c_end = ds.events.get();
+  uint32_t meta_state = 0;
   if (to_device) {
     // device-resident image: payload and CRC table in HBM, meta mirrored on host
     if (img->location != CHECL_IMAGE_DEVICE || img->device != device) {
@@ -1427,6 +1485,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
     tr("mirror");
     if (P.n_chunks) timed_launch(ds, kt, kOpPack, lp, ds.compute);
     tr("launch");
+    meta_state = prefinalize(img, P, epoch);  // (while K1 runs)
     if (P.n_chunks && !mirror) {
       ck(cudaEventRecord(c_begin, ds.compute));
       ck(cudaMemcpyAsync(img->host_mut + P.crc_off, img->d_crc, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.compute));
@@ -1478,6 +1537,7 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       timed_launch(ds, kt, kOpPack, lp, ds.compute);
       ck(cudaEventRecord(c_end, ds.compute));
       tm.n_stages = 1;
+      meta_state = prefinalize(img, P, epoch);
       settle(ctx);  // the previous call's spans, read while K1 runs
       ck(cudaStreamSynchronize(ds.compute));
     } else {
@@ -1543,13 +1603,15 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
       ck(cudaMemcpyAsync(img->host_mut + P.crc_off, ds.crc_scratch.p, 4 * P.n_chunks, cudaMemcpyDeviceToHost, ds.copy));
     ck(cudaEventRecord(c_end, ds.copy));
     tm.n_stages = P.stages.size();
+    meta_state = prefinalize(img, P, epoch);
     settle(ctx);  // the previous call's spans, read while the pipeline runs
     ck(cudaStreamSynchronize(ds.copy));
     }
   }
-  // a5: header, manifest and meta CRC (the CRC table has landed)
+  // a5: the meta CRC over the CRC table, which has landed (header and manifest were
+  // written while K1 ran)
   const double tf = now_ms();
-  finalize_meta(img->host_mut, P, epoch);
+  finalize_meta(img->host_mut, P, meta_state);
   tm.commit_ms = now_ms() - tf;
   tr("finalize");
   img->image_bytes = P.image_bytes;
@@ -1627,6 +1689,26 @@ struct Segment {
   uint64_t lo, hi;
 };
 
+// The layout of the last full-image restore on a device: its header and manifest bytes
+// (epoch and meta CRC zeroed), parse, segment plan and round count. A restore whose
+// image header matches reuses it without parsing the manifest again; the manifest
+// bytes are compared while K2 runs (a mismatch redoes the restore the long way).
+// `gen` names the layout process-wide in chunk-list keys.
+struct LayoutCache {
+  uint64_t gen = 0;
+  std::vector<uint8_t> meta;
+  Parsed P;
+  std::vector<Segment> segs;
+  uint64_t rounds = 0;
+};
+std::atomic<uint64_t> g_layout_gen{0};
+
+// The header fields a layout is made of: everything but the epoch (88) and meta CRC (124).
+bool header_same(const uint8_t* h, const std::vector<uint8_t>& meta) {
+  return meta.size() >= kHeaderBytes && std::memcmp(h, meta.data(), 88) == 0 &&
+         std::memcmp(h + 96, meta.data() + 96, 28) == 0;
+}
+
 // Consecutive records in manifest order; a segment is closed before a record that
 // would take it past segment_bytes(), so a buffer at least that large is alone.
 std::vector<Segment> plan_segments(const std::vector<BufRec>& bufs, uint64_t payload_bytes) {
@@ -1688,8 +1770,8 @@ std::shared_ptr<Arena> alloc_arena(checl_ctx* ctx, int device, void* stream, uin
 // this device released (best fit, at most 1/8 larger) or through the context's
 // allocator. false when the allocator fails (whatever was taken is freed).
 bool new_alloc(checl_ctx* ctx, int device, void* stream, const std::vector<BufRec>& bufs, uint64_t payload_bytes,
-               RestoreAlloc* out) {
-  out->segs = plan_segments(bufs, payload_bytes);
+               RestoreAlloc* out, const std::vector<Segment>* segs = nullptr) {
+  out->segs = segs ? *segs : plan_segments(bufs, payload_bytes);
   out->arenas.assign(out->segs.size(), nullptr);
   out->seg_of.assign(bufs.size(), ~0u);
   std::vector<size_t> need;  // segments the spares did not cover
@@ -1722,49 +1804,88 @@ bool new_alloc(checl_ctx* ctx, int device, void* stream, const std::vector<BufRe
   return true;
 }
 
+std::vector<void*> bases_of(const RestoreAlloc& A) {
+  std::vector<void*> v(A.arenas.size());
+  for (size_t k = 0; k < v.size(); ++k) v[k] = A.arenas[k]->base;
+  return v;
+}
+
 // Swaps every handle of the image to its new buffer (L15); frees library-owned
-// buffers previously bound to those handles (after their devices are idle).
-void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A) {
+// buffers previously bound to those handles (after their devices are idle). `gen` is
+// the image's layout (LayoutCache::gen, 0 = none).
+void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64_t gen) {
   std::vector<std::shared_ptr<Arena>> dropped;  // distinct arenas that lost their last handle
+  auto& bc = ctx->bind;
   {
     std::lock_guard<std::mutex> lk(ctx->mu);
     for (auto& a : A.arenas)
       if (a->base) ctx->by_addr[device][reinterpret_cast<uintptr_t>(a->base)] = {a->bytes, 0};
-    uint64_t max_h = 0;
-    // P.bufs ascend by handle, like the map: walk both in order (O(n), sequential)
-    // instead of one O(log n) search per handle (C3: 10 000 handles)
-    auto it = P.bufs.empty() ? ctx->entries.end() : ctx->entries.lower_bound(P.bufs.front().handle);
-    for (size_t bi = 0; bi < P.bufs.size(); ++bi) {
-      const BufRec& b = P.bufs[bi];
-      while (it != ctx->entries.end() && it->first < b.handle) ++it;
-      const bool fresh = it == ctx->entries.end() || it->first != b.handle;
-      if (fresh) it = ctx->entries.emplace_hint(it, b.handle, Entry{});
-      Entry& e = it->second;
-      if (!fresh) {  // rebind an existing handle in place
-        if (!e.arena && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
-        ctx->version[e.device]++;
-        ctx->n_live[e.device]--;
-        if (e.arena && --e.arena->n_handles == 0) {  // its last handle moved away
-          auto f = ctx->arenas.find(e.arena);
-          dropped.push_back(std::move(f->second));
-          ctx->arenas.erase(f);
-        }
+    const size_t n = P.bufs.size();
+    for (auto& a : A.arenas) a->n_handles = 0;  // (a reused spare may carry its old count)
+    if (gen && bc.gen == gen && bc.device == device && bc.version == ctx->version[device] && bc.entries.size() == n) {
+      // The same layout onto the same device, registry untouched since the last commit:
+      // these handles are exactly that commit's entries, bound to its segments and to
+      // nothing else. Rebind them in place; its segments lose all their handles.
+      for (Arena* old : bc.arenas) {
+        auto f = ctx->arenas.find(old);
+        if (f == ctx->arenas.end()) continue;
+        dropped.push_back(std::move(f->second));
+        ctx->arenas.erase(f);
       }
-      ctx->n_live[device]++;
-      e.device = device;
-      e.ptr = A.buf(P.bufs, bi);
-      e.bytes = b.size;
-      e.flags = b.flags;
-      e.owned = true;
-      Arena* na = b.size ? A.arenas[A.seg_of[bi]].get() : nullptr;
-      e.arena = na;
-      if (na) na->n_handles++;
-      max_h = std::max(max_h, b.handle);
+      for (size_t bi = 0; bi < n; ++bi) {
+        Entry* e = bc.entries[bi];
+        const uint64_t size = P.bufs[bi].size;
+        e->ptr = A.buf(P.bufs, bi);
+        Arena* na = size ? A.arenas[A.seg_of[bi]].get() : nullptr;
+        e->arena = na;
+        if (na) na->n_handles++;
+      }
+    } else {
+      bc.entries.resize(n);
+      uint64_t max_h = 0;
+      // P.bufs ascend by handle, like the map: walk both in order (O(n), sequential)
+      // instead of one O(log n) search per handle (C3: 10 000 handles)
+      auto it = P.bufs.empty() ? ctx->entries.end() : ctx->entries.lower_bound(P.bufs.front().handle);
+      for (size_t bi = 0; bi < n; ++bi) {
+        const BufRec& b = P.bufs[bi];
+        while (it != ctx->entries.end() && it->first < b.handle) ++it;
+        const bool fresh = it == ctx->entries.end() || it->first != b.handle;
+        if (fresh) it = ctx->entries.emplace_hint(it, b.handle, Entry{});
+        Entry& e = it->second;
+        if (!fresh) {  // rebind an existing handle in place
+          if (!e.arena && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
+          ctx->version[e.device]++;
+          ctx->n_live[e.device]--;
+          if (e.arena && --e.arena->n_handles == 0) {  // its last handle moved away
+            auto f = ctx->arenas.find(e.arena);
+            dropped.push_back(std::move(f->second));
+            ctx->arenas.erase(f);
+          }
+        }
+        ctx->n_live[device]++;
+        e.device = device;
+        e.ptr = A.buf(P.bufs, bi);
+        e.bytes = b.size;
+        e.flags = b.flags;
+        e.owned = true;
+        Arena* na = b.size ? A.arenas[A.seg_of[bi]].get() : nullptr;
+        e.arena = na;
+        if (na) na->n_handles++;
+        max_h = std::max(max_h, b.handle);
+        bc.entries[bi] = &e;
+      }
+      ctx->next_id = std::max(ctx->next_id, max_h + 1);
     }
+    bc.arenas.clear();
     for (auto& a : A.arenas)
-      if (a->n_handles) ctx->arenas.emplace(a.get(), a);
+      if (a->n_handles) {
+        ctx->arenas.emplace(a.get(), a);
+        bc.arenas.push_back(a.get());
+      }
     ctx->version[device]++;
-    ctx->next_id = std::max(ctx->next_id, max_h + 1);
+    bc.device = device;
+    bc.gen = gen;
+    bc.version = ctx->version[device];
     for (auto& a : dropped)
       if (a->base) ctx->by_addr[a->device].erase(reinterpret_cast<uintptr_t>(a->base));
   }
@@ -1774,12 +1895,8 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A) {
   // (the previous spares are freed)
   std::vector<std::shared_ptr<Arena>> keep, old;
   uint64_t kept = 0;
-  bool other = false;
   for (auto& a : dropped) {
-    if (a->device != device) {
-      other = true;
-      continue;
-    }
+    if (a->device != device) continue;
     if (a.use_count() == 1 && a->base && kept + a->bytes <= spare_limit()) {
       kept += a->bytes;
       keep.push_back(std::move(a));
@@ -1791,7 +1908,7 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A) {
     ctx->spares[device] = std::move(keep);
   }
   free_arenas(old);
-  if (other || !dropped.empty()) free_arenas(dropped);
+  free_arenas(dropped);
 }
 
 // After a successful restore onto `device`, the chunk list it expanded for the new
@@ -1799,31 +1916,37 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A) {
 // checkpoint of `device` needs when the device's live buffers are the image's: it
 // becomes that plan (buffers swapped, no re-expansion), so a checkpoint right
 // after a restore or migration skips the plan rebuild.
-void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, const RestoreAlloc& A) {
+void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, const RestoreAlloc& A, uint64_t gen) {
   std::lock_guard<std::mutex> lk(ctx->mu);
   if (ctx->n_live[device] != P.bufs.size() || !P.L.n_chunks) return;
   Plan& Q = ds.plan;
-  // the plan's current chunk list moves to the scratch buffers: so does its description
-  const bool q_valid = Q.version != ~0ull && Q.n_chunks && Q.recs.size() == Q.bufs.size();
-  ds.scratch_recs.swap(Q.recs);
-  ds.scratch_payload = q_valid ? Q.payload_bytes : ~0ull;
-  // the same layout as the current plan (every restore of a checkpoint/restore loop):
-  // only the buffer addresses change; stages, header and manifest stay
-  bool same = Q.version != ~0ull && Q.bufs.size() == P.bufs.size() && Q.n_chunks == P.L.n_chunks &&
-              Q.payload_bytes == P.full_payload && Q.crc_off == P.L.crc_off && Q.slot_bytes == ctx->slot_bytes;
-  for (size_t i = 0; same && i < Q.bufs.size(); ++i) {
-    const BufRec &q = Q.bufs[i], &b = P.bufs[i];
-    same = q.handle == b.handle && q.size == b.size && q.off == b.off && q.first_chunk == b.first_chunk &&
-           q.flags == b.flags;
-  }
-  if (same) {
-    for (size_t i = 0; i < Q.bufs.size(); ++i) Q.bufs[i].ptr = A.buf(Q.bufs, i);
-    Q.recs.resize(Q.bufs.size());
-    build_records(Q.bufs, [&](size_t b) { return Q.bufs[b].ptr; }, Q.recs.data());
+  // the plan's current chunk list moves to the scratch buffers, its key with it; the
+  // restore's list (key: gen over A's segments) becomes the plan's
+  auto swap_lists = [&] {
     std::swap(Q.d_desc.p, ds.desc_scratch.p);
     std::swap(Q.d_desc.cap, ds.desc_scratch.cap);
     std::swap(Q.d_round.p, ds.round_scratch.p);
     std::swap(Q.d_round.cap, ds.round_scratch.cap);
+    ds.scratch_gen = Q.layout_gen;
+    ds.scratch_bases.swap(Q.list_bases);
+    Q.layout_gen = gen;
+    Q.list_bases = bases_of(A);
+  };
+  // the same layout as the current plan (every restore of a checkpoint/restore loop):
+  // only the buffer addresses change; stages, header and manifest stay. (The plan's
+  // BufRec pointers are not used after the plan is built: its chunk list is.)
+  bool same = Q.version != ~0ull && gen && Q.layout_gen == gen && Q.slot_bytes == ctx->slot_bytes;
+  if (!same) {
+    same = Q.version != ~0ull && Q.bufs.size() == P.bufs.size() && Q.n_chunks == P.L.n_chunks &&
+           Q.payload_bytes == P.full_payload && Q.crc_off == P.L.crc_off && Q.slot_bytes == ctx->slot_bytes;
+    for (size_t i = 0; same && i < Q.bufs.size(); ++i) {
+      const BufRec &q = Q.bufs[i], &b = P.bufs[i];
+      same = q.handle == b.handle && q.size == b.size && q.off == b.off && q.first_chunk == b.first_chunk &&
+             q.flags == b.flags;
+    }
+  }
+  if (same) {
+    swap_lists();
     Q.version = ctx->version[device];
     return;
   }
@@ -1846,16 +1969,14 @@ void adopt_plan(checl_ctx* ctx, DevState& ds, int device, const Parsed& P, const
   Q.meta.assign(Q.crc_off, 0);
   write_header(Q.meta.data(), L, Q.bufs.size(), device, 0);
   write_manifest(Q.meta.data() + kHeaderBytes, Q.bufs, device);
-  std::swap(Q.d_desc.p, ds.desc_scratch.p);
-  std::swap(Q.d_desc.cap, ds.desc_scratch.cap);
-  std::swap(Q.d_round.p, ds.round_scratch.p);
-  std::swap(Q.d_round.cap, ds.round_scratch.cap);
+  plan_meta_state(Q);
+  swap_lists();
   Q.version = ctx->version[device];
   Q.slot_bytes = ctx->slot_bytes;
 }
 
 checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void* stream, checl_report* rep,
-                        bool in_migrate) {
+                        bool in_migrate, bool long_way = false) {
   const double t0 = now_ms();
   Trace tr("restore");
   DeviceGuard g(device);
@@ -1875,11 +1996,23 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   // structural check has passed, so K2 only reads inside the image and writes inside
   // the new allocation, which an invalid image leaves unbound and frees
   const double tp = now_ms();
-  Parsed P;
   const bool dev_img = img->location == CHECL_IMAGE_DEVICE;
-  checl_status st = parse_image(img->host, dev_img ? img->payload_off : img->image_bytes, dev_img, &P, false);
-  if (st) return st;
-  if (P.flags != 0) return CHECL_ERR_BAD_IMAGE;  // a delta restores only as part of a chain
+  const size_t len = dev_img ? img->payload_off : img->image_bytes;
+  // Fast path: the image's header names the layout of this device's last full-image
+  // restore (every restore of a checkpoint/restore loop): its parse, segments and
+  // chunk list are reused, and the manifest bytes are compared with it while K2 runs.
+  // K2 with that layout stays inside the image (the header fixes its sizes) and inside
+  // the new segments, so a mismatching manifest only costs a second, long-way restore.
+  LayoutCache* lc = ctx->layout[device].get();
+  const bool fast = !long_way && lc && lc->gen && img->host && len >= kHeaderBytes && header_same(img->host, lc->meta) &&
+                    len >= (dev_img ? lc->P.L.payload_off : lc->P.L.image_bytes);
+  Parsed parsed;
+  if (!fast) {
+    checl_status st = parse_image(img->host, len, dev_img, &parsed, false);
+    if (st) return st;
+    if (parsed.flags != 0) return CHECL_ERR_BAD_IMAGE;  // a delta restores only as part of a chain
+  }
+  const Parsed& P = fast ? lc->P : parsed;
   if (rep) set_report(rep, P, 0, 0);
   tr("parse");
 
@@ -1887,16 +2020,15 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   const double ta = now_ms();
   stream = stream_on(stream, device);
   RestoreAlloc A;
-  if (!new_alloc(ctx, device, stream, P.bufs, P.L.payload_bytes, &A))  // (an invalid image still reports BAD_IMAGE first)
+  if (!new_alloc(ctx, device, stream, P.bufs, P.L.payload_bytes, &A, fast ? &lc->segs : nullptr))
+    // (an invalid image still reports BAD_IMAGE first)
     return get_u32(img->host + 124) == meta_crc(img->host, P.L.payload_off) ? CHECL_ERR_OUT_OF_DEVICE_MEMORY
                                                                            : CHECL_ERR_BAD_IMAGE;
   order_after(ds, stream);  // nothing below touches the new memory before the caller's queued work
   tm.alloc_ms = now_ms() - ta;
   tr("alloc");
   const uint64_t nch = P.L.n_chunks;
-  ds.h_recs.ensure(std::max<size_t>(P.bufs.size(), 1));
-  // (zero-size buffers get a null pointer, as in adopt_plan's records)
-  const uint64_t rounds = build_records(P.bufs, [&](size_t b) { return A.buf(P.bufs, b); }, ds.h_recs.p);
+  std::vector<void*> bases = bases_of(A);
   ds.desc_scratch.ensure(std::max<uint64_t>(nch, 1));
   ds.round_scratch.ensure(nch + 1);
   ds.recs_scratch.ensure(std::max<size_t>(P.bufs.size(), 1));
@@ -1910,23 +2042,26 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   // publishing launch below leaves it at rest again (status_clean set after the sync)
   const bool was_clean = ds.status_clean, status_clean = was_clean && ds.status_host_dev;
   ds.status_clean = false;
-  // the chunk list of the new allocation: already in the scratch buffers when the
-  // allocation and layout are those of an earlier restore (arenas alternate between
-  // the two allocations of consecutive restores: see adopt_plan), else expanded on
-  // the GPU (compute stream, ahead of the verify launches); the expansion also
-  // initialises the verify status
-  const bool have_list = status_clean && ds.scratch_payload == P.L.payload_bytes &&
-                         ds.scratch_recs.size() == P.bufs.size() &&
-                         std::memcmp(ds.scratch_recs.data(), ds.h_recs.p, P.bufs.size() * sizeof(BufferRecord)) == 0;
+  // the chunk list of the new segments: already in the scratch buffers when its key
+  // (layout, segment addresses) is that of an earlier restore (segments alternate
+  // between the two sets of consecutive restores: see adopt_plan), else expanded on
+  // the GPU from one record per buffer (compute stream, ahead of the verify launches);
+  // the expansion also initialises the verify status
+  const bool have_list = status_clean && fast && ds.scratch_gen == lc->gen && ds.scratch_bases == bases;
   if (nch && !have_list) {
-    ds.scratch_payload = ~0ull;
+    ds.scratch_gen = 0;
+    ds.h_recs.ensure(std::max<size_t>(P.bufs.size(), 1));
+    // (zero-size buffers get a null pointer)
+    const uint64_t rounds = build_records(P.bufs, [&](size_t b) { return A.buf(P.bufs, b); }, ds.h_recs.p);
     ck(cudaMemcpyAsync(ds.recs_scratch.p, ds.h_recs.p, P.bufs.size() * sizeof(BufferRecord), cudaMemcpyHostToDevice,
                        ds.compute));
     ++ds.aux_launches;
     ck(launch_expand(ds.recs_scratch.p, (uint32_t)P.bufs.size(), P.L.payload_bytes, nch, ds.desc_scratch.p,
                      ds.round_scratch.p, rounds, ds.status.p, ds.n_sms, ds.compute));
-    ds.scratch_recs.assign(ds.h_recs.p, ds.h_recs.p + P.bufs.size());
-    ds.scratch_payload = P.L.payload_bytes;
+    if (fast) {  // the key of the list just expanded (a long-way restore sets it on success)
+      ds.scratch_gen = lc->gen;
+      ds.scratch_bases = bases;
+    }
   }
   lp.status_host = ds.status_host_dev;  // the last verify launch publishes (below)
   tr("expand");
@@ -2031,10 +2166,20 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
     ds.h_status.p[0] = ~0ull;
     ds.h_status.p[1] = 0;
   }
-  const bool meta_ok = get_u32(img->host + 124) == meta_crc(img->host, P.L.payload_off);  // r1, under K2
+  // r1, under K2: the meta CRC; on the fast path also the manifest the parse was skipped for
+  const bool layout_ok =
+      !fast || std::memcmp(img->host + kHeaderBytes, lc->meta.data() + kHeaderBytes, P.L.crc_off - kHeaderBytes) == 0;
+  const bool meta_ok = layout_ok && get_u32(img->host + 124) == meta_crc(img->host, P.L.payload_off);
   settle(ctx);  // the previous call's spans, read while K2 runs
   ck(cudaDeviceSynchronize());  // K2, the copies, and every queue of the target (quiesce, L16)
   tr("wait");
+  if (!layout_ok) {  // another manifest behind the same header: the long way
+    ds.status_clean = nch ? lp.status_host != nullptr : was_clean;
+    tmp_payload.release();
+    tmp_crc.release();
+    A = RestoreAlloc{};
+    return do_restore(ctx, img, device, stream, rep, in_migrate, true);
+  }
   ds.status_clean = nch ? lp.status_host != nullptr : was_clean;
   const uint64_t first_bad = ds.h_status.p[0], n_bad = ds.h_status.p[1];
   tm.n_kernels = kt.spans.size() + (ds.aux_launches - aux0);
@@ -2056,9 +2201,24 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
   (void)in_migrate;
   const double tc = now_ms();
   tr("events");
-  commit(ctx, P, device, A);
+  if (!fast) {  // this layout becomes the device's cached one
+    auto nl = std::make_unique<LayoutCache>();
+    nl->gen = ++g_layout_gen;
+    nl->meta.assign(img->host, img->host + P.L.crc_off);
+    std::memset(nl->meta.data() + 88, 0, 8);
+    std::memset(nl->meta.data() + 124, 0, 4);
+    nl->P = std::move(parsed);
+    nl->segs = A.segs;
+    ctx->layout[device] = std::move(nl);
+    lc = ctx->layout[device].get();
+    if (nch) {  // the list just expanded is this layout's over these segments
+      ds.scratch_gen = lc->gen;
+      ds.scratch_bases = bases;
+    }
+  }
+  commit(ctx, lc->P, device, A, lc->gen);
   tr("commit");
-  adopt_plan(ctx, ds, device, P, A);
+  adopt_plan(ctx, ds, device, lc->P, A, lc->gen);
   tr("adopt");
   tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
@@ -2381,7 +2541,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
     }
     if (open) dst.push_back(cur);
   }
-  ds.scratch_payload = ~0ull;  // the scratch list is overwritten (no longer described)
+  ds.scratch_gen = 0;  // the scratch list is overwritten (no longer described)
   ds.status_clean = false;
   ds.desc_scratch.ensure(std::max<uint64_t>(std::max<uint64_t>(nch, hdesc.size()), 1));
   ds.cdesc.ensure(std::max<size_t>(hdesc.size(), 1));
@@ -2469,7 +2629,7 @@ checl_status do_restore_chain(checl_ctx* ctx, const checl_image* const* chain, u
     return CHECL_ERR_CRC_MISMATCH;
   }
   const double tc = now_ms();
-  commit(ctx, Z, device, A);
+  commit(ctx, Z, device, A, 0);
   tm.commit_ms = now_ms() - tc;
   tm.total_ms = now_ms() - t0;
   defer_timing(ctx, ds, tm, kt, c_begin, c_end, CHECL_STATS_CHAIN);
@@ -3204,6 +3364,7 @@ checl_status checl_debug_corrupt(checl_image* img, uint64_t image_offset, uint8_
     }
     if (!img->owned) return CHECL_ERR_INVALID_VALUE;  // wrapped bytes are the caller's
     img->host_mut[image_offset] ^= mask;
+    img->meta_valid = false;  // (the next checkpoint into it rewrites its manifest)
     return CHECL_SUCCESS;
   });
 }

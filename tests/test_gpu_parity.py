@@ -458,3 +458,53 @@ def test_repeated_device_restores_reuse_chunk_list_and_status(ctx):
         ctx.restore(himg if i % 2 else dimg, DEV)
         for h, b in zip(ds.handles, ds.host):
             assert np.array_equal(bound_bytes(ctx, h), b), (i, h)
+
+
+def test_same_header_other_manifest_takes_the_long_way(ctx):
+    """Restore reuses the parse, segments and chunk list of the device's last restore
+    when the image header matches (DESIGN.md §5 "Restore fast path"), comparing the
+    manifest while K2 runs. Two oracle images with identical headers but different
+    manifests (other handles, other flags): each restore must bind exactly its own
+    image's handles, flags and bytes."""
+    rng = np.random.default_rng(71)
+    sizes = [70001, 3, 65536 * 2 + 9]
+    data = [rng.integers(0, 256, s, dtype=np.uint8) for s in sizes]
+    A = O.checkpoint([O.Entry(h, d, 5) for h, d in zip((11, 12, 13), data)], device=DEV, epoch=1)
+    B = O.checkpoint([O.Entry(h, d ^ 0x5A, 5) for h, d in zip((21, 22, 23), data)], device=DEV, epoch=2)
+    C = O.checkpoint([O.Entry(h, d, 6) for h, d in zip((11, 12, 13), data)], device=DEV, epoch=3)  # flags only
+    assert A[:88].tobytes() == B[:88].tobytes() == C[:88].tobytes()
+    for rnd in range(2):
+        for img, hs, want, fl in ((A, (11, 12, 13), data, 5), (B, (21, 22, 23), [d ^ 0x5A for d in data], 5),
+                                  (A, (11, 12, 13), data, 5), (C, (11, 12, 13), data, 6)):
+            rep = ctx.restore(checl.Image.wrap(img), DEV)
+            assert rep.n_bad_chunks == 0 and rep.n_buffers == 3
+            for h, d in zip(hs, want):
+                assert np.array_equal(bound_bytes(ctx, h), d), (rnd, h)
+        # the image checkpointed now holds every live handle with its flags
+        got = ctx.checkpoint(DEV, epoch=9).view()
+        st, _, ents = O.restore(got)
+        assert st == 0 and {e.handle: e.flags for e in ents} == {11: 6, 12: 6, 13: 6, 21: 5, 22: 5, 23: 5}
+
+
+def test_restore_fast_paths_follow_registry_changes(ctx):
+    """A checkpoint/restore loop takes the fast paths (cached layout, chunk-list key,
+    in-place rebinding); a registration or release in between must send the next
+    commit the long way, and every handle must stay exact."""
+    sizes = [1 << 20, 70001, 0, 3 * 65536 + 5, 4097]
+    ds = make_set(ctx, sizes, seed=72, offsets=[0, 4, 0, 1, 0])
+    dimg = ctx.checkpoint_device(DEV, epoch=1)
+    extra = []
+    for i in range(8):
+        ctx.checkpoint(DEV, epoch=i + 2, into=dimg)
+        ctx.restore(dimg, DEV)
+        for h, b in zip(ds.handles, ds.host):
+            assert np.array_equal(bound_bytes(ctx, h), b), (i, h)
+        if i == 3:  # a new registration: the next image has another layout
+            t = torch.full((777,), 9, dtype=torch.uint8, device=DEV)
+            extra.append((ctx.register(t), t))
+        if i == 5:  # and its release: back to the first layout
+            h, t = extra.pop()
+            ctx.release(h)
+    n, total = ctx.count(DEV)
+    assert n == len(sizes) and total == sum(sizes)
+    release_all(ctx, ds)
