@@ -13,6 +13,7 @@ stream.
 * A handle released on another thread while a checkpoint runs: the checkpoint still
   writes the bytes it planned (the release is deferred to the end of the call).
 """
+import gc
 import threading
 import time
 
@@ -35,7 +36,10 @@ MiB = 1 << 20
 
 def _held() -> int:
     """Bytes the caching allocator has handed out (the library's re-created buffers and
-    migration images come from it): independent of how it caches segments."""
+    migration images come from it): independent of how it caches segments. (Contexts
+    of earlier tests left to the garbage collector are collected first: one collected
+    mid-test would free its buffers inside the measured window.)"""
+    gc.collect()
     torch.cuda.synchronize()
     return torch.cuda.memory_allocated(0)
 

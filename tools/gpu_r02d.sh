@@ -27,3 +27,11 @@ timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --c
 CHECL_TRACE=1 timeout 300 python tools/trace_step.py C3 6 > $O/trace_c3.log 2>&1
 CHECL_TRACE=1 timeout 120 python tools/trace_step.py C2 6 > $O/trace_c2.log 2>&1
 du -sh $O
+for rep in 1 2; do
+  timeout 600 python bench.py --no-cpu-baseline --no-extras > $O/c3_$rep.json 2>/dev/null
+  timeout 300 python bench.py --config C2 --no-cpu-baseline --no-extras > $O/c2_$rep.json 2>/dev/null
+done
+for f in $O/c3_*.json $O/c2_*.json; do python -c "
+import json
+d=json.load(open('$f'));r=d['roofline'];e=d.get('e2e') or {}
+print('$f'.split('/')[-1], 'value %.1f step %.4f ms pack %.1f us verify %.1f us frac %.3f e2e %.2f' % (d['value'], d['ms_per_step'], r['pack_ms']*1e3, r['verify_ms']*1e3, r['frac'], e.get('value', 0)))" 2>&1 | tail -1; done | tee $O/quick.txt
