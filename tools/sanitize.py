@@ -31,8 +31,16 @@ for h, b in zip(hs, host):
 t = ctx.tensor(hs[0])
 t[12345:12346].add_(1)
 torch.cuda.synchronize()
-delta = ctx.checkpoint_incremental(dev, img, epoch=3)
+delta = ctx.checkpoint_incremental(dev, img, epoch=3)  # exact rule: seeds the shadow, diff_kernel
 ctx.restore_chain([img, delta], dev)
+t = ctx.tensor(hs[3])
+t[100:101].add_(1)  # (a misaligned buffer in the original registry: byte path of diff_kernel before the restore)
+torch.cuda.synchronize()
+delta2 = ctx.checkpoint_incremental(dev, delta, epoch=5)  # shadow follows the chain
+delta3 = ctx.checkpoint_incremental(dev, img, epoch=6, rule=checl.DIRTY_CRC)
+for _ in range(3):  # restore fast path (cached layout, chunk-list key, in-place rebinding)
+    ctx.checkpoint(dev, epoch=7, into=d)
+    ctx.restore(d, dev)
 ctx.set_staging(196608, 2)
 img2 = ctx.checkpoint(dev, epoch=4)
 ctx.restore(img2, dev)
