@@ -72,10 +72,11 @@ constexpr int kMaxSignal = 65;
 std::atomic<checl_ctx*> g_signal_ctx[kMaxSignal];
 
 // Pinned host buffers of freed library-owned images, kept for the next image
-// (cudaHostAlloc of a large buffer costs ~1 ms per few MB: an incremental
-// checkpoint loop would otherwise pin a new image every step). Bounded by
-// CHECL_PINNED_POOL_BYTES (default 4 GiB); the least recently returned buffers are
-// released first. Pinned sizes are rounded up to size classes (<= 12.5% slack) so
+// (cudaHostAlloc pins ~2.4 GB/s on the B200 boxes: an incremental checkpoint loop, or
+// a file restore loop, would otherwise pin a new image every step). Bounded by
+// CHECL_PINNED_POOL_BYTES (default min(16 GiB, 1/8 of the host's RAM): a 4 GiB cap
+// re-pinned every C3-sized image, 1.8 s per 4 GiB, profiles/r02/cost_model_*); the
+// least recently returned buffers are released first; checl_trim empties it. Pinned sizes are rounded up to size classes (<= 12.5% slack) so
 // that images of similar size reuse each other's buffers.
 size_t pinned_class(size_t n) {
   if (n <= (2u << 20)) return (n + 4095) & ~(size_t)4095;
@@ -91,7 +92,9 @@ struct PinnedPool {
   size_t bytes = 0, limit = 0;
   PinnedPool() {
     const char* e = std::getenv("CHECL_PINNED_POOL_BYTES");
-    limit = e ? (size_t)std::strtoull(e, nullptr, 10) : (4ull << 30);
+    const long pages = sysconf(_SC_PHYS_PAGES), psz = sysconf(_SC_PAGESIZE);
+    const size_t ram = pages > 0 && psz > 0 ? (size_t)pages * (size_t)psz : (32ull << 30);
+    limit = e ? (size_t)std::strtoull(e, nullptr, 10) : std::min<size_t>(16ull << 30, ram / 8);
   }
   // the smallest pooled buffer with n <= capacity <= 2n + 64 MiB, or nullptr
   void* take(size_t n, size_t* cap) {
@@ -1778,11 +1781,20 @@ bool new_alloc(checl_ctx* ctx, int device, void* stream, const std::vector<BufRe
   {
     std::lock_guard<std::mutex> lk(ctx->mu);
     auto& sp = ctx->spares[device];
-    for (size_t k = 0; k < out->segs.size(); ++k) {
+    // the spares of the previous restore of the same layout are in segment order:
+    // taken in place when every size matches exactly (a checkpoint/restore loop)
+    bool in_order = sp.size() == out->segs.size();
+    for (size_t k = 0; in_order && k < sp.size(); ++k) in_order = sp[k]->bytes == out->segs[k].hi - out->segs[k].lo;
+    if (in_order) {
+      for (size_t k = 0; k < sp.size(); ++k) out->arenas[k] = std::move(sp[k]);
+      sp.clear();
+    }
+    for (size_t k = 0; !in_order && k < out->segs.size(); ++k) {
       const uint64_t n = out->segs[k].hi - out->segs[k].lo;
       size_t best = sp.size();
       for (size_t i = 0; n && i < sp.size(); ++i)
-        if (sp[i]->bytes >= n && sp[i]->bytes - n <= n / 8 && (best == sp.size() || sp[i]->bytes < sp[best]->bytes))
+        if (sp[i] && sp[i]->bytes >= n && sp[i]->bytes - n <= n / 8 &&
+            (best == sp.size() || sp[i]->bytes < sp[best]->bytes))
           best = i;
       if (best != sp.size()) {
         out->arenas[k] = std::move(sp[best]);
@@ -1832,13 +1844,25 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
         dropped.push_back(std::move(f->second));
         ctx->arenas.erase(f);
       }
+      // per segment: its arena and the address of payload offset 0 in it
+      std::vector<Arena*> ak(A.arenas.size());
+      std::vector<uint8_t*> at0(A.arenas.size());
+      for (size_t k = 0; k < ak.size(); ++k) {
+        ak[k] = A.arenas[k].get();
+        at0[k] = static_cast<uint8_t*>(ak[k]->base) - A.segs[k].lo;
+      }
       for (size_t bi = 0; bi < n; ++bi) {
         Entry* e = bc.entries[bi];
-        const uint64_t size = P.bufs[bi].size;
-        e->ptr = A.buf(P.bufs, bi);
-        Arena* na = size ? A.arenas[A.seg_of[bi]].get() : nullptr;
-        e->arena = na;
-        if (na) na->n_handles++;
+        const BufRec& b = P.bufs[bi];
+        const uint32_t k = A.seg_of[bi];
+        if (b.size) {
+          e->ptr = at0[k] + b.off;
+          e->arena = ak[k];
+          ak[k]->n_handles++;
+        } else {
+          e->ptr = nullptr;
+          e->arena = nullptr;
+        }
       }
     } else {
       bc.entries.resize(n);
