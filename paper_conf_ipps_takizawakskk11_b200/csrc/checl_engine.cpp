@@ -1828,13 +1828,17 @@ std::vector<void*> bases_of(const RestoreAlloc& A) {
 void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64_t gen) {
   std::vector<std::shared_ptr<Arena>> dropped;  // distinct arenas that lost their last handle
   auto& bc = ctx->bind;
+  Trace tr("commit");
+  bool fast_bind = false;
   {
     std::lock_guard<std::mutex> lk(ctx->mu);
     for (auto& a : A.arenas)
       if (a->base) ctx->by_addr[device][reinterpret_cast<uintptr_t>(a->base)] = {a->bytes, 0};
     const size_t n = P.bufs.size();
     for (auto& a : A.arenas) a->n_handles = 0;  // (a reused spare may carry its old count)
+    tr("lock+by_addr");
     if (gen && bc.gen == gen && bc.device == device && bc.version == ctx->version[device] && bc.entries.size() == n) {
+      fast_bind = true;
       // The same layout onto the same device, registry untouched since the last commit:
       // these handles are exactly that commit's entries, bound to its segments and to
       // nothing else. Rebind them in place; its segments lose all their handles.
@@ -1900,6 +1904,7 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
       }
       ctx->next_id = std::max(ctx->next_id, max_h + 1);
     }
+    tr(fast_bind ? "rebind_in_place" : "rebind_walk");
     bc.arenas.clear();
     for (auto& a : A.arenas)
       if (a->n_handles) {
@@ -1912,6 +1917,7 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
     bc.version = ctx->version[device];
     for (auto& a : dropped)
       if (a->base) ctx->by_addr[a->device].erase(reinterpret_cast<uintptr_t>(a->base));
+    tr("arenas");
   }
   // arenas whose last handle moved away are freed here, outside the lock, once their
   // device is idle (the restore synchronised `device` after K2; another device is
@@ -1931,8 +1937,10 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
     old.swap(ctx->spares[device]);
     ctx->spares[device] = std::move(keep);
   }
+  tr("spares");
   free_arenas(old);
   free_arenas(dropped);
+  tr("free");
 }
 
 // After a successful restore onto `device`, the chunk list it expanded for the new
