@@ -57,3 +57,20 @@ def test_reference_arm_two_ranks_rank0_prints_once():
     lines = _json_lines(r.stdout)
     assert len(lines) == 1
     _check_line(lines[0], 2)
+
+
+def test_host_ram_check_and_meminfo(monkeypatch):
+    """The e2e leg pins one image per local rank: bench.host_ram_check compares that
+    with MemAvailable (70 % of it), which bench.meminfo_available reads from
+    /proc/meminfo (C4 at 8 ranks needs ~512 GiB: scaled down)."""
+    sys.path.insert(0, ROOT)
+    import bench
+    avail = bench.meminfo_available()
+    assert avail > 0
+    monkeypatch.setattr(bench, "meminfo_available", lambda: 196 << 30)
+    fits, need, av = bench.host_ram_check(68_719_476_448, 8)
+    assert not fits and need == 8 * 68_719_476_448 and av == 196 << 30
+    fits, need, _ = bench.host_ram_check(5_350_180_722, 8)
+    assert fits and need == 8 * 5_350_180_722
+    monkeypatch.setattr(bench, "meminfo_available", lambda: 0)  # unknown: assume it fits
+    assert bench.host_ram_check(1 << 40, 8)[0]
