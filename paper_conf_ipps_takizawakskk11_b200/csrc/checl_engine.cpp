@@ -15,6 +15,7 @@
 
 #include <algorithm>
 #include <unordered_map>
+#include <unordered_set>
 #include <atomic>
 #include <chrono>
 #include <cstdio>
@@ -538,14 +539,28 @@ struct Arena {
 
 struct LayoutCache;
 
+// The bindings of one commit (restore / migrate): record i's current buffer address
+// and segment. The entries it bound point at their slot (Entry::bind, idx) instead of
+// holding the address, so a commit that rebinds the same handles to the same layout in
+// new segments rewrites these two contiguous arrays, not 10 000 map nodes.
+struct Binding {
+  std::vector<uint8_t*> ptr;
+  std::vector<Arena*> arena;  // nullptr for a zero-size buffer
+  uint64_t refs = 0;          // entries bound through it
+};
+
 struct Entry {
   int device;
-  uint8_t* ptr;
+  uint8_t* ptr;  // user-registered buffers (bind == nullptr)
   uint64_t bytes;
   uint32_t flags;
   bool owned;
-  Arena* arena;  // owned buffers: the arena holding them (kept alive by checl_ctx::arenas)
+  Binding* bind;  // owned (re-created) buffers: their slot, bind->ptr[idx] / bind->arena[idx]
+  uint32_t idx;
 };
+
+uint8_t* entry_ptr(const Entry& e) { return e.bind ? e.bind->ptr[e.idx] : e.ptr; }
+Arena* entry_arena(const Entry& e) { return e.bind ? e.bind->arena[e.idx] : nullptr; }
 
 // Phase-time events for checl_timing.
 struct KernelTimer {  // the event pair around every timed launch of a call
@@ -700,9 +715,10 @@ struct checl_ctx {
   struct BindCache {
     int device = -1;
     uint64_t gen = 0, version = 0;
-    std::vector<Entry*> entries;
-    std::vector<Arena*> arenas;
+    Binding* binding = nullptr;  // bound exactly the entries of that commit (nullptr: none)
+    std::vector<Arena*> arenas;  // the segments it bound into
   } bind;
+  std::unordered_set<Binding*> bindings;  // with refs > 0
 
   DevState& dev(int d) {
     if (!devs[d]) {
@@ -1032,7 +1048,7 @@ Plan& get_plan(checl_ctx* ctx, DevState& ds, int device) {
   P.bufs.clear();
   for (auto& kv : ctx->entries)
     if (kv.second.device == device)
-      P.bufs.push_back(BufRec{kv.first, kv.second.bytes, 0, 0, kv.second.flags, kv.second.ptr});
+      P.bufs.push_back(BufRec{kv.first, kv.second.bytes, 0, 0, kv.second.flags, entry_ptr(kv.second)});
   Layout L = layout_records(P.bufs);
   if (L.payload_bytes > (1ull << 40)) throw std::bad_alloc();
   P.n_chunks = L.n_chunks;
@@ -1825,6 +1841,19 @@ std::vector<void*> bases_of(const RestoreAlloc& A) {
 // Swaps every handle of the image to its new buffer (L15); frees library-owned
 // buffers previously bound to those handles (after their devices are idle). `gen` is
 // the image's layout (LayoutCache::gen, 0 = none).
+// An entry leaves its binding (released or rebound); the binding goes with its last
+// entry. Under the context lock.
+void unbind(checl_ctx* ctx, Entry& e) {
+  Binding* b = e.bind;
+  if (!b) return;
+  e.bind = nullptr;
+  if (--b->refs == 0) {
+    if (ctx->bind.binding == b) ctx->bind.binding = nullptr;
+    ctx->bindings.erase(b);
+    delete b;
+  }
+}
+
 void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64_t gen) {
   std::vector<std::shared_ptr<Arena>> dropped;  // distinct arenas that lost their last handle
   auto& bc = ctx->bind;
@@ -1836,40 +1865,42 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
       if (a->base) ctx->by_addr[device][reinterpret_cast<uintptr_t>(a->base)] = {a->bytes, 0};
     const size_t n = P.bufs.size();
     for (auto& a : A.arenas) a->n_handles = 0;  // (a reused spare may carry its old count)
+    // per segment: its arena and the address of payload offset 0 in it
+    std::vector<Arena*> ak(A.arenas.size());
+    std::vector<uint8_t*> at0(A.arenas.size());
+    for (size_t k = 0; k < ak.size(); ++k) {
+      ak[k] = A.arenas[k].get();
+      at0[k] = static_cast<uint8_t*>(ak[k]->base) - A.segs[k].lo;
+    }
     tr("lock+by_addr");
-    if (gen && bc.gen == gen && bc.device == device && bc.version == ctx->version[device] && bc.entries.size() == n) {
-      fast_bind = true;
+    Binding* B = bc.binding;
+    if (gen && B && bc.gen == gen && bc.device == device && bc.version == ctx->version[device] && B->refs == n &&
+        B->ptr.size() == n) {
       // The same layout onto the same device, registry untouched since the last commit:
-      // these handles are exactly that commit's entries, bound to its segments and to
-      // nothing else. Rebind them in place; its segments lose all their handles.
+      // these handles are exactly that commit's entries, bound through B to its
+      // segments and to nothing else. Rewrite B's slots; its segments lose all handles.
+      fast_bind = true;
       for (Arena* old : bc.arenas) {
         auto f = ctx->arenas.find(old);
         if (f == ctx->arenas.end()) continue;
         dropped.push_back(std::move(f->second));
         ctx->arenas.erase(f);
       }
-      // per segment: its arena and the address of payload offset 0 in it
-      std::vector<Arena*> ak(A.arenas.size());
-      std::vector<uint8_t*> at0(A.arenas.size());
-      for (size_t k = 0; k < ak.size(); ++k) {
-        ak[k] = A.arenas[k].get();
-        at0[k] = static_cast<uint8_t*>(ak[k]->base) - A.segs[k].lo;
-      }
       for (size_t bi = 0; bi < n; ++bi) {
-        Entry* e = bc.entries[bi];
         const BufRec& b = P.bufs[bi];
         const uint32_t k = A.seg_of[bi];
         if (b.size) {
-          e->ptr = at0[k] + b.off;
-          e->arena = ak[k];
-          ak[k]->n_handles++;
-        } else {
-          e->ptr = nullptr;
-          e->arena = nullptr;
+          B->ptr[bi] = at0[k] + b.off;
+          B->arena[bi] = ak[k];
         }
       }
+      for (size_t k = 0; k < A.segs.size(); ++k)
+        for (size_t bi = A.segs[k].b0; bi < A.segs[k].b1; ++bi) ak[k]->n_handles += P.bufs[bi].size ? 1 : 0;
     } else {
-      bc.entries.resize(n);
+      B = new Binding();
+      B->ptr.assign(n, nullptr);
+      B->arena.assign(n, nullptr);
+      ctx->bindings.insert(B);
       uint64_t max_h = 0;
       // P.bufs ascend by handle, like the map: walk both in order (O(n), sequential)
       // instead of one O(log n) search per handle (C3: 10 000 handles)
@@ -1881,26 +1912,38 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
         if (fresh) it = ctx->entries.emplace_hint(it, b.handle, Entry{});
         Entry& e = it->second;
         if (!fresh) {  // rebind an existing handle in place
-          if (!e.arena && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
+          if (!e.owned && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
           ctx->version[e.device]++;
           ctx->n_live[e.device]--;
-          if (e.arena && --e.arena->n_handles == 0) {  // its last handle moved away
-            auto f = ctx->arenas.find(e.arena);
+          Arena* old = entry_arena(e);
+          if (old && --old->n_handles == 0) {  // its last handle moved away
+            auto f = ctx->arenas.find(old);
             dropped.push_back(std::move(f->second));
             ctx->arenas.erase(f);
           }
+          unbind(ctx, e);
         }
         ctx->n_live[device]++;
         e.device = device;
-        e.ptr = A.buf(P.bufs, bi);
+        e.ptr = nullptr;
         e.bytes = b.size;
         e.flags = b.flags;
         e.owned = true;
-        Arena* na = b.size ? A.arenas[A.seg_of[bi]].get() : nullptr;
-        e.arena = na;
-        if (na) na->n_handles++;
+        e.bind = B;
+        e.idx = (uint32_t)bi;
+        if (b.size) {
+          const uint32_t k = A.seg_of[bi];
+          B->ptr[bi] = at0[k] + b.off;
+          B->arena[bi] = ak[k];
+          ak[k]->n_handles++;
+        }
         max_h = std::max(max_h, b.handle);
-        bc.entries[bi] = &e;
+      }
+      B->refs = n;
+      if (!n) {
+        ctx->bindings.erase(B);
+        delete B;
+        B = nullptr;
       }
       ctx->next_id = std::max(ctx->next_id, max_h + 1);
     }
@@ -1915,6 +1958,7 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
     bc.device = device;
     bc.gen = gen;
     bc.version = ctx->version[device];
+    bc.binding = B;
     for (auto& a : dropped)
       if (a->base) ctx->by_addr[a->device].erase(reinterpret_cast<uintptr_t>(a->base));
     tr("arenas");
@@ -2702,6 +2746,9 @@ checl_status checl_destroy(checl_ctx* ctx) {
         if (prev >= 0) cudaSetDevice(prev);
       }
       ctx->entries.clear();
+      for (Binding* b : ctx->bindings) delete b;
+      ctx->bindings.clear();
+      ctx->bind.binding = nullptr;
       ctx->arenas.clear();
       for (auto& n : ctx->n_live) n = 0;
       for (auto& sp : ctx->spares) sp.clear();
@@ -2757,7 +2804,8 @@ checl_status checl_register_buffer(checl_ctx* ctx, int device, void* dev_ptr, si
     e.bytes = bytes;
     e.flags = flags;
     e.owned = false;
-    e.arena = nullptr;
+    e.bind = nullptr;
+    e.idx = 0;
     ctx->entries.emplace(h, std::move(e));
     ctx->n_live[device]++;
     if (bytes) ctx->by_addr[device][lo] = {bytes, h};
@@ -2778,9 +2826,11 @@ checl_status checl_release(checl_ctx* ctx, checl_handle h) {
       if (it == ctx->entries.end()) return CHECL_ERR_INVALID_HANDLE;
       Entry& e = it->second;
       dev = e.device;
-      if (!e.arena && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
-      if (e.arena && --e.arena->n_handles == 0) {  // the segment's last handle
-        auto f = ctx->arenas.find(e.arena);
+      if (!e.owned && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
+      Arena* ea = entry_arena(e);
+      unbind(ctx, e);
+      if (ea && --ea->n_handles == 0) {  // the segment's last handle
+        auto f = ctx->arenas.find(ea);
         drop = std::move(f->second);
         ctx->arenas.erase(f);
         if (drop->base) ctx->by_addr[drop->device].erase(reinterpret_cast<uintptr_t>(drop->base));
@@ -2805,7 +2855,7 @@ checl_status checl_translate(const checl_ctx* ctx, checl_handle h, void** dev_pt
   std::lock_guard<std::mutex> lk(ctx->mu);
   auto it = ctx->entries.find(h);
   if (it == ctx->entries.end()) return CHECL_ERR_INVALID_HANDLE;
-  if (dev_ptr) *dev_ptr = it->second.ptr;
+  if (dev_ptr) *dev_ptr = entry_ptr(it->second);
   if (bytes) *bytes = it->second.bytes;
   if (device) *device = it->second.device;
   return CHECL_SUCCESS;
