@@ -1421,6 +1421,10 @@ void* stream_on(void* stream, int device) {
 // were still pending could otherwise be overwritten by those kernels after K2. The
 // library's streams wait for everything queued on that stream so far.
 void order_after(DevState& ds, void* stream) {
+  // nothing queued on it is still pending: nothing to order after (the common case:
+  // no cross-stream wait in front of K2's graph launch)
+  if (cudaStreamQuery(static_cast<cudaStream_t>(stream)) == cudaSuccess) return;
+  cudaGetLastError();  // (cudaErrorNotReady)
   cudaEvent_t ev = ds.events.get();
   ck(cudaEventRecord(ev, static_cast<cudaStream_t>(stream)));
   ck(cudaStreamWaitEvent(ds.compute, ev, 0));
