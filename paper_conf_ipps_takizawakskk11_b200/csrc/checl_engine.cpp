@@ -539,14 +539,18 @@ struct Arena {
 
 struct LayoutCache;
 
-// The bindings of one commit (restore / migrate): record i's current buffer address
-// and segment. The entries it bound point at their slot (Entry::bind, idx) instead of
-// holding the address, so a commit that rebinds the same handles to the same layout in
-// new segments rewrites these two contiguous arrays, not 10 000 map nodes.
+// The bindings of one commit (restore / migrate): record i lives in segment seg[i] at
+// offset rel[i] (seg = ~0: a zero-size buffer), and each segment's arena and address
+// are kept once. The entries it bound point at their record (Entry::bind, idx)
+// instead of holding an address, so a commit that rebinds the same handles to the
+// same layout in new segments rewrites one pointer per segment (80 for C3's 10 000
+// buffers), not one map node per handle.
 struct Binding {
-  std::vector<uint8_t*> ptr;
-  std::vector<Arena*> arena;  // nullptr for a zero-size buffer
-  uint64_t refs = 0;          // entries bound through it
+  std::vector<uint32_t> seg;
+  std::vector<uint64_t> rel;
+  std::vector<uint8_t*> seg_base;
+  std::vector<Arena*> seg_arena;
+  uint64_t refs = 0;  // entries bound through it
 };
 
 struct Entry {
@@ -559,8 +563,16 @@ struct Entry {
   uint32_t idx;
 };
 
-uint8_t* entry_ptr(const Entry& e) { return e.bind ? e.bind->ptr[e.idx] : e.ptr; }
-Arena* entry_arena(const Entry& e) { return e.bind ? e.bind->arena[e.idx] : nullptr; }
+uint8_t* entry_ptr(const Entry& e) {
+  if (!e.bind) return e.ptr;
+  const uint32_t k = e.bind->seg[e.idx];
+  return k == ~0u ? nullptr : e.bind->seg_base[k] + e.bind->rel[e.idx];
+}
+Arena* entry_arena(const Entry& e) {
+  if (!e.bind) return nullptr;
+  const uint32_t k = e.bind->seg[e.idx];
+  return k == ~0u ? nullptr : e.bind->seg_arena[k];
+}
 
 // Phase-time events for checl_timing.
 struct KernelTimer {  // the event pair around every timed launch of a call
@@ -1869,41 +1881,40 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
       if (a->base) ctx->by_addr[device][reinterpret_cast<uintptr_t>(a->base)] = {a->bytes, 0};
     const size_t n = P.bufs.size();
     for (auto& a : A.arenas) a->n_handles = 0;  // (a reused spare may carry its old count)
-    // per segment: its arena and the address of payload offset 0 in it
-    std::vector<Arena*> ak(A.arenas.size());
-    std::vector<uint8_t*> at0(A.arenas.size());
-    for (size_t k = 0; k < ak.size(); ++k) {
-      ak[k] = A.arenas[k].get();
-      at0[k] = static_cast<uint8_t*>(ak[k]->base) - A.segs[k].lo;
-    }
     tr("lock+by_addr");
     Binding* B = bc.binding;
+    const size_t nseg = A.arenas.size();
     if (gen && B && bc.gen == gen && bc.device == device && bc.version == ctx->version[device] && B->refs == n &&
-        B->ptr.size() == n) {
+        B->seg.size() == n && B->seg_base.size() == nseg && bc.arenas.size() <= nseg) {
       // The same layout onto the same device, registry untouched since the last commit:
       // these handles are exactly that commit's entries, bound through B to its
-      // segments and to nothing else. Rewrite B's slots; its segments lose all handles.
+      // segments and to nothing else, in the same segment plan. Point B's segments at
+      // the new arenas (each takes over its predecessor's handle count); the old ones
+      // lose all their handles.
       fast_bind = true;
+      for (size_t k = 0; k < nseg; ++k) {
+        Arena* old = B->seg_arena[k];
+        Arena* na = A.arenas[k].get();
+        na->n_handles = old ? old->n_handles : 0;
+        B->seg_arena[k] = na;
+        B->seg_base[k] = static_cast<uint8_t*>(na->base) - A.segs[k].lo;
+      }
       for (Arena* old : bc.arenas) {
         auto f = ctx->arenas.find(old);
         if (f == ctx->arenas.end()) continue;
         dropped.push_back(std::move(f->second));
         ctx->arenas.erase(f);
       }
-      for (size_t bi = 0; bi < n; ++bi) {
-        const BufRec& b = P.bufs[bi];
-        const uint32_t k = A.seg_of[bi];
-        if (b.size) {
-          B->ptr[bi] = at0[k] + b.off;
-          B->arena[bi] = ak[k];
-        }
-      }
-      for (size_t k = 0; k < A.segs.size(); ++k)
-        for (size_t bi = A.segs[k].b0; bi < A.segs[k].b1; ++bi) ak[k]->n_handles += P.bufs[bi].size ? 1 : 0;
     } else {
       B = new Binding();
-      B->ptr.assign(n, nullptr);
-      B->arena.assign(n, nullptr);
+      B->seg.assign(n, ~0u);
+      B->rel.assign(n, 0);
+      B->seg_base.resize(nseg);
+      B->seg_arena.resize(nseg);
+      for (size_t k = 0; k < nseg; ++k) {
+        B->seg_arena[k] = A.arenas[k].get();
+        B->seg_base[k] = static_cast<uint8_t*>(A.arenas[k]->base) - A.segs[k].lo;
+      }
       ctx->bindings.insert(B);
       uint64_t max_h = 0;
       // P.bufs ascend by handle, like the map: walk both in order (O(n), sequential)
@@ -1937,9 +1948,9 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
         e.idx = (uint32_t)bi;
         if (b.size) {
           const uint32_t k = A.seg_of[bi];
-          B->ptr[bi] = at0[k] + b.off;
-          B->arena[bi] = ak[k];
-          ak[k]->n_handles++;
+          B->seg[bi] = k;
+          B->rel[bi] = b.off;
+          A.arenas[k]->n_handles++;
         }
         max_h = std::max(max_h, b.handle);
       }
