@@ -1310,6 +1310,63 @@ __global__ void __launch_bounds__(256) diff_kernel(const ChunkDesc* __restrict__
   }
 }
 
+// a5 on the GPU for large device images: the meta CRC's register over the CRC table
+// and the zero pad that follows it (FORMAT.md meta_crc), continuing from `state`, the
+// host's register after header and manifest. CRC linearity: R(M, s) = s * x^(8|M|) +
+// XOR_t R(piece_t, 0) * x^(8 (|M| - end_t)); the table is cut into one piece per thread
+// (slicing-by-4 over a shared table built from the polynomial), the zero pad only
+// shifts. One CTA; *out (mapped host memory) = the final CRC (complemented).
+struct Pow8 {
+  uint32_t v[48];  // x^(8 * 2^j) mod P
+};
+__device__ __forceinline__ uint32_t x8n_dev(uint64_t n, const Pow8& pw) {
+  uint32_t r = kOne;
+  for (int j = 0; n; ++j, n >>= 1)
+    if (n & 1u) r = gf_mul(r, pw.v[j]);
+  return r;
+}
+__global__ void __launch_bounds__(1024, 1) meta_crc_kernel(const uint32_t* __restrict__ table, uint64_t table_bytes,
+                                                           uint64_t total_bytes, uint32_t state, const Pow8 pw,
+                                                           uint32_t* out) {
+  __shared__ uint32_t T[4][256];
+  __shared__ uint32_t red[32];
+  const int tid = threadIdx.x;
+  if (tid < 256) {
+    uint32_t r = (uint32_t)tid;
+    for (int b = 0; b < 8; ++b) r = gf_mulx(r);
+    T[0][tid] = r;
+  }
+  __syncthreads();
+  if (tid < 256) {
+    uint32_t r = T[0][tid];
+    for (int k = 1; k < 4; ++k) {
+      r = (r >> 8) ^ T[0][r & 0xFFu];
+      T[k][tid] = r;
+    }
+  }
+  __syncthreads();
+  const uint64_t words = table_bytes / 4, per = (words + blockDim.x - 1) / blockDim.x;
+  const uint64_t w0 = (uint64_t)tid * per, w1 = w0 + per < words ? w0 + per : words;
+  uint32_t c = 0;
+  if (w0 < w1) {
+    uint32_t r = 0;
+    for (uint64_t w = w0; w < w1; ++w) {
+      r ^= table[w];
+      r = T[3][r & 0xFFu] ^ T[2][(r >> 8) & 0xFFu] ^ T[1][(r >> 16) & 0xFFu] ^ T[0][r >> 24];
+    }
+    c = gf_mul(r, x8n_dev(total_bytes - 4 * w1, pw));
+  }
+  if (tid == 0) c ^= gf_mul(state, x8n_dev(total_bytes, pw));
+  for (int o = 16; o; o >>= 1) c ^= __shfl_xor_sync(0xFFFFFFFFu, c, o);
+  if ((tid & 31) == 0) red[tid >> 5] = c;
+  __syncthreads();
+  if (tid < 32) {
+    c = tid < (int)(blockDim.x >> 5) ? red[tid] : 0u;
+    for (int o = 16; o; o >>= 1) c ^= __shfl_xor_sync(0xFFFFFFFFu, c, o);
+    if (tid == 0) *reinterpret_cast<volatile uint32_t*>(out) = ~c;
+  }
+}
+
 // CRC table of an exact delta: entry cidx[k] of `table` (the base's table) takes the
 // CRC computed for present chunk k (ccrc[k], from the gather launches), k < totals[0].
 __global__ void crc_scatter_kernel(const uint32_t* __restrict__ ccrc, const uint32_t* __restrict__ cidx,
@@ -1595,6 +1652,17 @@ cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, co
                               const uint32_t* dirty, uint64_t n, uint32_t* map_words, ChunkDesc* cdesc, uint32_t* cidx,
                               unsigned long long* totals, cudaStream_t s) {
   delta_scan_kernel<<<1, 1024, 0, s>>>(desc, crc_now, crc_base, dirty, n, map_words, cdesc, cidx, totals);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_meta_crc(const uint32_t* table, uint64_t table_bytes, uint64_t total_bytes, uint32_t state,
+                            uint32_t* out, cudaStream_t s) {
+  static const Pow8 pw = [] {
+    Pow8 p{};
+    for (int j = 0; j < 48; ++j) p.v[j] = gf_x8n(1ull << j);
+    return p;
+  }();
+  meta_crc_kernel<<<1, 1024, 0, s>>>(table, table_bytes, total_bytes, state, pw, out);
   return cudaGetLastError();
 }
 

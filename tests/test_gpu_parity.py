@@ -508,3 +508,40 @@ def test_restore_fast_paths_follow_registry_changes(ctx):
     n, total = ctx.count(DEV)
     assert n == len(sizes) and total == sum(sizes)
     release_all(ctx, ds)
+
+
+def test_large_table_meta_crc_on_gpu(ctx):
+    """A device image whose CRC table is at least 128 KB has its meta CRC computed on
+    the GPU (meta_crc_kernel: per-thread slicing-by-4 pieces combined by CRC linearity,
+    DESIGN.md §5 "Finalize"): 40 000 one-chunk buffers (a 160 KB table, odd sizes,
+    misaligned views), host and HBM images equal the oracle's byte for byte."""
+    rng = np.random.default_rng(81)
+    n = 40000
+    sizes = [int(x) for x in rng.integers(1, 200, n)]
+    big = torch.empty(sum(sizes) + 8 * n, dtype=torch.uint8, device=DEV)
+    views, pos = [], 0
+    for i, s in enumerate(sizes):
+        off = pos + (i % 7)
+        views.append(big[off:off + s])
+        pos += s + 8
+    checl.debug_fill(big, 81, 0)
+    torch.cuda.synchronize()
+    handles = [ctx.register(v, i & 0xFF) for i, v in enumerate(views)]
+    host = big.cpu().numpy()
+    ents, pos = [], 0
+    for i, (h, s) in enumerate(zip(handles, sizes)):
+        off = pos + (i % 7)
+        ents.append(O.Entry(h, host[off:off + s], i & 0xFF))
+        pos += s + 8
+    want = O.checkpoint(ents, device=DEV, epoch=17)
+    dimg = ctx.checkpoint_device(DEV, epoch=17)
+    h = dimg.to_host()
+    assert np.array_equal(h.view(), want), "HBM image (GPU meta CRC) != oracle image"
+    for e in (18, 19):  # repeated: the manifest is not rewritten, the epoch term changes
+        ctx.checkpoint(DEV, epoch=e, into=dimg)
+        h2 = dimg.to_host()
+        assert np.array_equal(h2.view(), O.checkpoint(ents, device=DEV, epoch=e)), e
+        h2.free()
+    h.free()
+    img = ctx.checkpoint(DEV, epoch=17)
+    assert np.array_equal(img.view(), want)
