@@ -47,7 +47,7 @@ cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, co
                               unsigned long long* totals, cudaStream_t s);
 cudaError_t launch_diff(const ChunkDesc* desc, uint64_t n, uint8_t* shadow, uint32_t* dirty, int n_sms, cudaStream_t s);
 cudaError_t launch_meta_crc(const uint32_t* table, uint64_t table_bytes, uint64_t total_bytes, uint32_t state,
-                            uint32_t* out, cudaStream_t s);
+                            unsigned long long* acc, uint32_t* out, int n_sms, cudaStream_t s);
 cudaError_t launch_crc_scatter(const uint32_t* ccrc, const uint32_t* cidx, const unsigned long long* totals,
                                uint64_t n_max, uint32_t* table, int n_sms, cudaStream_t s);
 cudaError_t launch_delta_stages(const ChunkDesc* cdesc, const unsigned long long* totals, uint64_t W, uint64_t n_stages,
@@ -431,6 +431,7 @@ struct DevState {
   // the meta CRC a meta_crc_kernel computed (mapped pinned word) and its device address
   PinnedBuf<uint32_t> h_meta;
   uint32_t* meta_dev = nullptr;
+  DevBuf<unsigned long long> meta_acc;  // meta_crc_kernel's accumulator + CTA count (zero at rest)
   EventPool events;
   std::vector<LaunchGraph> graphs;
   Plan plan;
@@ -459,6 +460,8 @@ struct DevState {
       status_clean = true;
     }
     h_meta.ensure(1, cudaHostAllocMapped);
+    meta_acc.ensure(2);
+    ck(cudaMemset(meta_acc.p, 0, 2 * sizeof(unsigned long long)));
     {
       void* dp = nullptr;
       if (cudaHostGetDevicePointer(&dp, h_meta.p, 0) == cudaSuccess)
@@ -513,6 +516,7 @@ struct DevState {
     h_status.release();
     h_recs.release();
     h_meta.release();
+    meta_acc.release();
     for (auto& g : graphs) {
       cudaGraphExecDestroy(g.exec);
       cudaGraphDestroy(g.graph);
@@ -1541,7 +1545,8 @@ checl_status do_checkpoint(checl_ctx* ctx, int device, void* stream, uint64_t ep
     // L2, instead of by the host from pinned memory the GPU just wrote (~40 us for C3)
     if (ds.meta_dev && 4 * P.n_chunks >= kMetaKernelMinBytes) {
       ++ds.aux_launches;
-      ck(launch_meta_crc(img->d_crc, 4 * P.n_chunks, P.payload_off - P.crc_off, meta_state, ds.meta_dev, ds.compute));
+      ck(launch_meta_crc(img->d_crc, 4 * P.n_chunks, P.payload_off - P.crc_off, meta_state, ds.meta_acc.p, ds.meta_dev,
+                         ds.n_sms, ds.compute));
       meta_on_gpu = true;
     }
     if (P.n_chunks && !mirror) {

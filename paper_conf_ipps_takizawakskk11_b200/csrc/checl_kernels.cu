@@ -1311,33 +1311,39 @@ __global__ void __launch_bounds__(256) diff_kernel(const ChunkDesc* __restrict__
 }
 
 // a5 on the GPU for large device images: the meta CRC's register over the CRC table
-// and the zero pad that follows it (FORMAT.md meta_crc), continuing from `state`, the
-// host's register after header and manifest. CRC linearity: R(M, s) = s * x^(8|M|) +
-// XOR_t R(piece_t, 0) * x^(8 (|M| - end_t)); the table is cut into one piece per thread
-// (slicing-by-4 over a shared table built from the polynomial), the zero pad only
-// shifts. One CTA; *out (mapped host memory) = the final CRC (complemented).
-struct Pow8 {
-  uint32_t v[48];  // x^(8 * 2^j) mod P
+// and the zero pad that follows it (FORMAT.md meta_crc), continuing from the host's
+// register after header and manifest. By CRC linearity, R(T || Z, s) = s x^(8|T||Z|) +
+// R(T, 0) x^(8|Z|), and R(T, 0) is unchanged by leading zeros, so T is viewed as
+// `lead` zero words followed by the table, cut into G*256 pieces of `per` words:
+// thread t CRCs piece t from zero (slicing-by-4, per-CTA shared tables) and shifts it
+// by C^(Ttot-1-t), C = x^(32 per), one multiply by a constant per set bit (nibble
+// tables of C^(2^j) built per CTA); the pieces are XORed per CTA and across CTAs
+// (atomicXor), and the last CTA applies the pad shift and the host's state term.
+struct MetaParams {
+  const uint32_t* table;
+  uint64_t words, per, lead;
+  uint32_t cpow[16];   // C^(2^j), C = x^(8 * 4 * per)
+  uint32_t pad_pow;    // x^(8 |Z|)
+  uint32_t state_term; // host register after header + manifest, times x^(8 |T||Z|)
+  unsigned long long* acc;  // [0] XOR of the CTAs' terms, [1] CTAs done (zero at rest)
+  uint32_t* out;            // mapped host word: the final CRC (complemented)
 };
-__device__ __forceinline__ uint32_t x8n_dev(uint64_t n, const Pow8& pw) {
-  uint32_t r = kOne;
-  for (int j = 0; n; ++j, n >>= 1)
-    if (n & 1u) r = gf_mul(r, pw.v[j]);
-  return r;
-}
-__global__ void __launch_bounds__(1024, 1) meta_crc_kernel(const uint32_t* __restrict__ table, uint64_t table_bytes,
-                                                           uint64_t total_bytes, uint32_t state, const Pow8 pw,
-                                                           uint32_t* out) {
+__global__ void __launch_bounds__(256) meta_crc_kernel(const MetaParams mp) {
   __shared__ uint32_t T[4][256];
-  __shared__ uint32_t red[32];
+  __shared__ uint32_t nib[16][8][16];  // nib[j][i][v] = (v << 4i) * cpow[j]
+  __shared__ uint32_t red[8];
   const int tid = threadIdx.x;
-  if (tid < 256) {
+  {
     uint32_t r = (uint32_t)tid;
     for (int b = 0; b < 8; ++b) r = gf_mulx(r);
     T[0][tid] = r;
   }
+  for (int e = tid; e < 16 * 8 * 16; e += blockDim.x) {
+    const int j = e >> 7, i = (e >> 4) & 7, v = e & 15;
+    nib[j][i][v] = gf_mul((uint32_t)v << (4 * i), mp.cpow[j]);
+  }
   __syncthreads();
-  if (tid < 256) {
+  {
     uint32_t r = T[0][tid];
     for (int k = 1; k < 4; ++k) {
       r = (r >> 8) ^ T[0][r & 0xFFu];
@@ -1345,25 +1351,34 @@ __global__ void __launch_bounds__(1024, 1) meta_crc_kernel(const uint32_t* __res
     }
   }
   __syncthreads();
-  const uint64_t words = table_bytes / 4, per = (words + blockDim.x - 1) / blockDim.x;
-  const uint64_t w0 = (uint64_t)tid * per, w1 = w0 + per < words ? w0 + per : words;
-  uint32_t c = 0;
-  if (w0 < w1) {
-    uint32_t r = 0;
-    for (uint64_t w = w0; w < w1; ++w) {
-      r ^= table[w];
-      r = T[3][r & 0xFFu] ^ T[2][(r >> 8) & 0xFFu] ^ T[1][(r >> 16) & 0xFFu] ^ T[0][r >> 24];
-    }
-    c = gf_mul(r, x8n_dev(total_bytes - 4 * w1, pw));
+  const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + tid, ttot = (uint64_t)gridDim.x * blockDim.x;
+  uint32_t r = 0;
+  for (uint64_t v = t * mp.per; v < (t + 1) * mp.per; ++v) {
+    if (v < mp.lead) continue;  // leading zero words leave a zero register unchanged
+    r ^= mp.table[v - mp.lead];
+    r = T[3][r & 0xFFu] ^ T[2][(r >> 8) & 0xFFu] ^ T[1][(r >> 16) & 0xFFu] ^ T[0][r >> 24];
   }
-  if (tid == 0) c ^= gf_mul(state, x8n_dev(total_bytes, pw));
-  for (int o = 16; o; o >>= 1) c ^= __shfl_xor_sync(0xFFFFFFFFu, c, o);
-  if ((tid & 31) == 0) red[tid >> 5] = c;
+  uint64_t m = ttot - 1 - t;  // pieces after this one
+  for (int j = 0; m && r; ++j, m >>= 1) {
+    if (!(m & 1u)) continue;
+    uint32_t q = 0;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) q ^= nib[j][i][(r >> (4 * i)) & 15u];
+    r = q;
+  }
+  for (int o = 16; o; o >>= 1) r ^= __shfl_xor_sync(0xFFFFFFFFu, r, o);
+  if ((tid & 31) == 0) red[tid >> 5] = r;
   __syncthreads();
-  if (tid < 32) {
-    c = tid < (int)(blockDim.x >> 5) ? red[tid] : 0u;
-    for (int o = 16; o; o >>= 1) c ^= __shfl_xor_sync(0xFFFFFFFFu, c, o);
-    if (tid == 0) *reinterpret_cast<volatile uint32_t*>(out) = ~c;
+  if (tid == 0) {
+    uint32_t c = 0;
+    for (int w = 0; w < (int)(blockDim.x >> 5); ++w) c ^= red[w];
+    atomicXor(&mp.acc[0], (unsigned long long)c);
+    __threadfence();
+    if (atomicAdd(&mp.acc[1], 1ull) == gridDim.x - 1) {  // the last CTA
+      const uint32_t all = (uint32_t)atomicExch(&mp.acc[0], 0ull);
+      atomicExch(&mp.acc[1], 0ull);
+      *reinterpret_cast<volatile uint32_t*>(mp.out) = ~(mp.state_term ^ gf_mul(all, mp.pad_pow));
+    }
   }
 }
 
@@ -1656,13 +1671,22 @@ cudaError_t launch_delta_scan(const ChunkDesc* desc, const uint32_t* crc_now, co
 }
 
 cudaError_t launch_meta_crc(const uint32_t* table, uint64_t table_bytes, uint64_t total_bytes, uint32_t state,
-                            uint32_t* out, cudaStream_t s) {
-  static const Pow8 pw = [] {
-    Pow8 p{};
-    for (int j = 0; j < 48; ++j) p.v[j] = gf_x8n(1ull << j);
-    return p;
-  }();
-  meta_crc_kernel<<<1, 1024, 0, s>>>(table, table_bytes, total_bytes, state, pw, out);
+                            unsigned long long* acc, uint32_t* out, int n_sms, cudaStream_t s) {
+  MetaParams mp{};
+  mp.table = table;
+  mp.words = table_bytes / 4;
+  uint64_t grid = (mp.words + 255) / 256;  // at least one word per thread
+  grid = grid < 1 ? 1 : grid > (uint64_t)n_sms ? (uint64_t)n_sms : grid;
+  const uint64_t ttot = grid * 256;
+  mp.per = (mp.words + ttot - 1) / ttot;
+  mp.lead = mp.per * ttot - mp.words;
+  uint32_t c = gf_x8n(4 * mp.per);
+  for (int j = 0; j < 16; ++j, c = gf_mul(c, c)) mp.cpow[j] = c;
+  mp.pad_pow = gf_x8n(total_bytes - table_bytes);
+  mp.state_term = gf_mul(state, gf_x8n(total_bytes));
+  mp.acc = acc;
+  mp.out = out;
+  meta_crc_kernel<<<(unsigned)grid, 256, 0, s>>>(mp);
   return cudaGetLastError();
 }
 
