@@ -9,6 +9,8 @@ checks every live handle against a Python model: its size and device (translate)
 bytes (the image contents it was restored from, or the user's writes). The model
 follows PAPER.md L15 (handles stay valid, translation gives the current buffer) and
 FORMAT.md (an image restores exactly the bytes it was taken with)."""
+import os
+
 import numpy as np
 import pytest
 
@@ -29,7 +31,8 @@ def _bytes(ctx, h):
     return ctx.tensor(h).cpu().numpy()
 
 
-@pytest.mark.parametrize("seed", range(6))
+# CHECL_REG_FUZZ_CASES widens the sweep (default 16 sequences of 60 calls)
+@pytest.mark.parametrize("seed", range(int(os.environ.get("CHECL_REG_FUZZ_CASES", "16"))))
 def test_random_call_sequences_match_model(seed):
     rng = np.random.default_rng(900 + seed)
     ctx = checl.Context()
@@ -61,7 +64,7 @@ def test_random_call_sequences_match_model(seed):
 
     for _ in range(4):
         new_buffer()
-    for step in range(40):
+    for step in range(60):
         op = rng.choice(["reg", "rel", "write", "ckpt", "ckpt_dev", "restore", "restore_again", "migrate", "incr"],
                         p=[.1, .08, .16, .12, .1, .18, .12, .06, .08])
         if op == "reg" or not model:
