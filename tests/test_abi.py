@@ -98,7 +98,13 @@ except checl.CheclError as e:
 assert c.register_ptr(0, 0x10000, 0x1000) == 101   # released range reusable, id fresh
 img = checl.Image.wrap(bytes(4096))
 assert img.view().size == 4096 and img.info()["location"] == checl.IMAGE_HOST
+try:  # an unknown dirty rule is refused before any device work
+    c.checkpoint_incremental(0, img, epoch=1, rule=7)
+    raise SystemExit("unknown dirty rule accepted")
+except checl.CheclError as e:
+    assert e.status == checl.ERR_INVALID_VALUE
 img.free()
+c.trim()  # nothing kept yet: a no-op without a device
 c.close()
 print("ok")
 """
@@ -114,7 +120,7 @@ def test_missing_library_fails_loudly(tmp_path):
     # a copy of the package without libchecl.so must refuse to import (no CPU fallback)
     import shutil
     dst = tmp_path / "paper_conf_ipps_takizawakskk11_b200"
-    shutil.copytree(PKG, dst, ignore=shutil.ignore_patterns("*.so", "build_obj", "__pycache__"))
+    shutil.copytree(PKG, dst, ignore=shutil.ignore_patterns("*.so", "build_obj*", "__pycache__"))
     r = subprocess.run([sys.executable, "-c", "import paper_conf_ipps_takizawakskk11_b200"], cwd=tmp_path,
                        capture_output=True, text=True)
     assert r.returncode != 0 and "ImportError" in r.stderr and "no CPU fallback" in r.stderr
