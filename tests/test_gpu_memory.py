@@ -172,3 +172,31 @@ def test_release_during_checkpoint_is_deferred():
         assert np.array_equal(got, want)
         del junk
         out["img"].free()
+
+
+def test_segment_boundaries_and_partial_release():
+    """Segments (reading 18) around the 64 MiB cut: buffers just under, at and
+    just over it, zero-size buffers between and at the ends, a segment made only of
+    small buffers; every restore is bit-exact, the segment plan shows in the held bytes,
+    and releasing every handle of one segment returns that segment alone."""
+    sizes = [0, 64 * MiB - 1, 0, 64 * MiB, 3, 64 * MiB + 1, 5000, 7000, 0, 1, 32 * MiB, 33 * MiB, 0]
+    with checl.Context() as ctx:
+        ds = make_set(ctx, sizes, seed=61, offsets=[i % 4 for i in range(len(sizes))])
+        img = ctx.checkpoint_device(0, epoch=1)
+        for rep in range(3):  # a fresh allocation, then the spares of the previous commit
+            ctx.restore(img, 0)
+            for h, b in zip(ds.handles, ds.host):
+                assert np.array_equal(bound_bytes(ctx, h), b), (rep, h)
+        ctx.trim()
+        held = _held()
+        # the 33 MiB buffer: its segment starts at the 32 MiB one's offset and holds both
+        # (32 + 33 > 64 MiB would close it: so it is alone); release it and the held
+        # bytes drop by its own 2 MiB-rounded size only
+        i = sizes.index(33 * MiB)
+        ctx.release(ds.handles[i])
+        ctx.trim()
+        dropped = held - _held()
+        assert 33 * MiB <= dropped <= 36 * MiB, dropped
+        for h, b in zip(ds.handles[:i], ds.host[:i]):
+            assert np.array_equal(bound_bytes(ctx, h), b), h
+        img.free()
