@@ -189,9 +189,9 @@ def test_segment_boundaries_and_partial_release():
                 assert np.array_equal(bound_bytes(ctx, h), b), (rep, h)
         ctx.trim()
         held = _held()
-        # the 33 MiB buffer: its segment starts at the 32 MiB one's offset and holds both
-        # (32 + 33 > 64 MiB would close it: so it is alone); release it and the held
-        # bytes drop by its own 2 MiB-rounded size only
+        # the 33 MiB buffer would take the segment of the small buffers and the 32 MiB
+        # one past 64 MiB, so a new segment starts with it (only the zero-size buffer
+        # after it joins): releasing it returns that segment, ~33 MiB rounded up
         i = sizes.index(33 * MiB)
         ctx.release(ds.handles[i])
         ctx.trim()
