@@ -559,8 +559,8 @@ struct Arena {
 struct LayoutCache;
 
 // The bindings of one commit (restore / migrate): record i lives in segment seg[i] at
-// offset rel[i] (seg = ~0: a zero-size buffer), and each segment's arena and address
-// are kept once. The entries it bound point at their record (Entry::bind, idx)
+// offset rel[i] (seg = ~0: a zero-size buffer), and each segment's arena (owned here)
+// and address are kept once. The entries it bound point at their record (Entry::bind, idx)
 // instead of holding an address, so a commit that rebinds the same handles to the
 // same layout in new segments rewrites one pointer per segment (80 for C3's 10 000
 // buffers), not one map node per handle.
@@ -568,7 +568,9 @@ struct Binding {
   std::vector<uint32_t> seg;
   std::vector<uint64_t> rel;
   std::vector<uint8_t*> seg_base;
-  std::vector<Arena*> seg_arena;
+  // the segments themselves: the binding owns them (a segment whose last handle is
+  // released is moved out and freed; null from then on)
+  std::vector<std::shared_ptr<Arena>> seg_arena;
   uint64_t refs = 0;  // entries bound through it
 };
 
@@ -587,11 +589,7 @@ uint8_t* entry_ptr(const Entry& e) {
   const uint32_t k = e.bind->seg[e.idx];
   return k == ~0u ? nullptr : e.bind->seg_base[k] + e.bind->rel[e.idx];
 }
-Arena* entry_arena(const Entry& e) {
-  if (!e.bind) return nullptr;
-  const uint32_t k = e.bind->seg[e.idx];
-  return k == ~0u ? nullptr : e.bind->seg_arena[k];
-}
+
 
 // Phase-time events for checl_timing.
 struct KernelTimer {  // the event pair around every timed launch of a call
@@ -694,12 +692,8 @@ struct checl_ctx {
   checl_allocator alloc{nullptr, nullptr, nullptr};
   std::map<uint64_t, Entry> entries;                  // ascending handle = database order (L19)
   uint64_t n_live[kMaxDevices] = {};                  // entries per device
-  // arenas with at least one bound entry; an entry holds a plain pointer and the
-  // arena counts its entries (no per-handle reference-count traffic: C3 rebinds
-  // 10 000 handles per restore)
-  std::unordered_map<Arena*, std::shared_ptr<Arena>> arenas;
-  // live address ranges per device for overlap checks: user registrations (handle)
-  // and restore arenas (handle 0, one range per arena)
+  // live address ranges of user registrations per device (overlap checks; the
+  // library's own segments are checked through the bindings that own them)
   struct Range {
     uint64_t bytes, handle;
   };
@@ -747,7 +741,6 @@ struct checl_ctx {
     int device = -1;
     uint64_t gen = 0, version = 0;
     Binding* binding = nullptr;  // bound exactly the entries of that commit (nullptr: none)
-    std::vector<Arena*> arenas;  // the segments it bound into
   } bind;
   std::unordered_set<Binding*> bindings;  // with refs > 0
 
@@ -1890,6 +1883,22 @@ std::vector<void*> bases_of(const RestoreAlloc& A) {
 // the image's layout (LayoutCache::gen, 0 = none).
 // An entry leaves its binding (released or rebound); the binding goes with its last
 // entry. Under the context lock.
+void unbind(checl_ctx* ctx, Entry& e);
+
+// An owned entry gives up its buffer: its segment loses a handle, and a segment left
+// without handles moves to `dropped` (freed by the caller outside the lock). Under the
+// context lock.
+void release_slot(checl_ctx* ctx, Entry& e, std::vector<std::shared_ptr<Arena>>& dropped) {
+  if (e.bind) {
+    const uint32_t k = e.bind->seg[e.idx];
+    if (k != ~0u) {
+      std::shared_ptr<Arena>& slot = e.bind->seg_arena[k];
+      if (slot && --slot->n_handles == 0) dropped.push_back(std::move(slot));
+    }
+  }
+  unbind(ctx, e);
+}
+
 void unbind(checl_ctx* ctx, Entry& e) {
   Binding* b = e.bind;
   if (!b) return;
@@ -1902,50 +1911,39 @@ void unbind(checl_ctx* ctx, Entry& e) {
 }
 
 void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64_t gen) {
-  std::vector<std::shared_ptr<Arena>> dropped;  // distinct arenas that lost their last handle
+  std::vector<std::shared_ptr<Arena>> dropped;  // segments that lost their last handle
   auto& bc = ctx->bind;
   Trace tr("commit");
   bool fast_bind = false;
   {
     std::lock_guard<std::mutex> lk(ctx->mu);
-    for (auto& a : A.arenas)
-      if (a->base) ctx->by_addr[device][reinterpret_cast<uintptr_t>(a->base)] = {a->bytes, 0};
     const size_t n = P.bufs.size();
     for (auto& a : A.arenas) a->n_handles = 0;  // (a reused spare may carry its old count)
-    tr("lock+by_addr");
     Binding* B = bc.binding;
     const size_t nseg = A.arenas.size();
     if (gen && B && bc.gen == gen && bc.device == device && bc.version == ctx->version[device] && B->refs == n &&
-        B->seg.size() == n && B->seg_base.size() == nseg && bc.arenas.size() <= nseg) {
+        B->seg.size() == n && B->seg_base.size() == nseg) {
       // The same layout onto the same device, registry untouched since the last commit:
       // these handles are exactly that commit's entries, bound through B to its
-      // segments and to nothing else, in the same segment plan. Point B's segments at
-      // the new arenas (each takes over its predecessor's handle count); the old ones
-      // lose all their handles.
+      // segments and to nothing else, in the same segment plan. B takes the new
+      // segments (each with its predecessor's handle count); the old ones lose all
+      // their handles.
       fast_bind = true;
       for (size_t k = 0; k < nseg; ++k) {
-        Arena* old = B->seg_arena[k];
-        Arena* na = A.arenas[k].get();
-        na->n_handles = old ? old->n_handles : 0;
-        B->seg_arena[k] = na;
-        B->seg_base[k] = static_cast<uint8_t*>(na->base) - A.segs[k].lo;
-      }
-      for (Arena* old : bc.arenas) {
-        auto f = ctx->arenas.find(old);
-        if (f == ctx->arenas.end()) continue;
-        dropped.push_back(std::move(f->second));
-        ctx->arenas.erase(f);
+        std::shared_ptr<Arena>& slot = B->seg_arena[k];
+        A.arenas[k]->n_handles = slot ? slot->n_handles : 0;
+        if (slot) dropped.push_back(std::move(slot));
+        slot = A.arenas[k];
+        B->seg_base[k] = static_cast<uint8_t*>(slot->base) - A.segs[k].lo;
       }
     } else {
       B = new Binding();
       B->seg.assign(n, ~0u);
       B->rel.assign(n, 0);
       B->seg_base.resize(nseg);
-      B->seg_arena.resize(nseg);
-      for (size_t k = 0; k < nseg; ++k) {
-        B->seg_arena[k] = A.arenas[k].get();
+      B->seg_arena = A.arenas;
+      for (size_t k = 0; k < nseg; ++k)
         B->seg_base[k] = static_cast<uint8_t*>(A.arenas[k]->base) - A.segs[k].lo;
-      }
       ctx->bindings.insert(B);
       uint64_t max_h = 0;
       // P.bufs ascend by handle, like the map: walk both in order (O(n), sequential)
@@ -1961,13 +1959,7 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
           if (!e.owned && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
           ctx->version[e.device]++;
           ctx->n_live[e.device]--;
-          Arena* old = entry_arena(e);
-          if (old && --old->n_handles == 0) {  // its last handle moved away
-            auto f = ctx->arenas.find(old);
-            dropped.push_back(std::move(f->second));
-            ctx->arenas.erase(f);
-          }
-          unbind(ctx, e);
+          release_slot(ctx, e, dropped);
         }
         ctx->n_live[device]++;
         e.device = device;
@@ -1994,22 +1986,13 @@ void commit(checl_ctx* ctx, const Parsed& P, int device, RestoreAlloc& A, uint64
       ctx->next_id = std::max(ctx->next_id, max_h + 1);
     }
     tr(fast_bind ? "rebind_in_place" : "rebind_walk");
-    bc.arenas.clear();
-    for (auto& a : A.arenas)
-      if (a->n_handles) {
-        ctx->arenas.emplace(a.get(), a);
-        bc.arenas.push_back(a.get());
-      }
     ctx->version[device]++;
     bc.device = device;
     bc.gen = gen;
     bc.version = ctx->version[device];
     bc.binding = B;
-    for (auto& a : dropped)
-      if (a->base) ctx->by_addr[a->device].erase(reinterpret_cast<uintptr_t>(a->base));
-    tr("arenas");
   }
-  // arenas whose last handle moved away are freed here, outside the lock, once their
+  // segments whose last handle moved away are freed here, outside the lock, once their
   // device is idle (the restore synchronised `device` after K2; another device is
   // synchronised here); on this device they become the spares of the next restore
   // (the previous spares are freed)
@@ -2784,18 +2767,21 @@ checl_status checl_destroy(checl_ctx* ctx) {
     {
       // delete in the reverse of creation order (L19-L20)
       std::lock_guard<std::mutex> lk(ctx->mu);
-      for (auto& kv : ctx->arenas) {
-        int prev = -1;
-        cudaGetDevice(&prev);
-        cudaSetDevice(kv.first->device);
-        cudaDeviceSynchronize();
-        if (prev >= 0) cudaSetDevice(prev);
-      }
+      bool synced[kMaxDevices] = {};
+      for (Binding* b : ctx->bindings)
+        for (auto& a : b->seg_arena)
+          if (a && a->base && !synced[a->device]) {  // no kernel may still touch them
+            int prev = -1;
+            cudaGetDevice(&prev);
+            cudaSetDevice(a->device);
+            cudaDeviceSynchronize();
+            if (prev >= 0) cudaSetDevice(prev);
+            synced[a->device] = true;
+          }
       ctx->entries.clear();
-      for (Binding* b : ctx->bindings) delete b;
+      for (Binding* b : ctx->bindings) delete b;  // (frees the segments)
       ctx->bindings.clear();
       ctx->bind.binding = nullptr;
-      ctx->arenas.clear();
       for (auto& n : ctx->n_live) n = 0;
       for (auto& sp : ctx->spares) sp.clear();
       ctx->deferred.clear();
@@ -2842,6 +2828,14 @@ checl_status checl_register_buffer(checl_ctx* ctx, int device, void* dev_ptr, si
         --it;  // range starting at or before lo
         if (it->first + it->second.bytes > lo) return CHECL_ERR_INVALID_VALUE;
       }
+      // the library's own live segments (a few per restore; not in the range map, so
+      // that a commit does not update it per segment)
+      for (Binding* b : ctx->bindings)
+        for (auto& a : b->seg_arena)
+          if (a && a->base && a->device == device) {
+            const uintptr_t s0 = reinterpret_cast<uintptr_t>(a->base);
+            if (lo < s0 + a->bytes && s0 < lo + bytes) return CHECL_ERR_INVALID_VALUE;
+          }
     }
     const uint64_t h = ctx->next_id++;
     Entry e;
@@ -2873,13 +2867,10 @@ checl_status checl_release(checl_ctx* ctx, checl_handle h) {
       Entry& e = it->second;
       dev = e.device;
       if (!e.owned && e.bytes) ctx->by_addr[e.device].erase(reinterpret_cast<uintptr_t>(e.ptr));
-      Arena* ea = entry_arena(e);
-      unbind(ctx, e);
-      if (ea && --ea->n_handles == 0) {  // the segment's last handle
-        auto f = ctx->arenas.find(ea);
-        drop = std::move(f->second);
-        ctx->arenas.erase(f);
-        if (drop->base) ctx->by_addr[drop->device].erase(reinterpret_cast<uintptr_t>(drop->base));
+      std::vector<std::shared_ptr<Arena>> d;
+      release_slot(ctx, e, d);  // the segment's last handle: d holds it
+      if (!d.empty()) {
+        drop = std::move(d.front());
         // a checkpoint / restore / migrate running on another thread may have planned
         // reads of it: that call frees it when it ends (BusyGuard)
         if (ctx->busy.load()) ctx->deferred.push_back(std::move(drop));
