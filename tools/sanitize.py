@@ -45,4 +45,15 @@ ctx.set_staging(196608, 2)
 img2 = ctx.checkpoint(dev, epoch=4)
 ctx.restore(img2, dev)
 ctx.close()
+# a CRC table of >= 128 KB: the meta CRC runs on the GPU (meta_crc_kernel)
+ctx = checl.Context()
+big = torch.empty(40000 * 40, dtype=torch.uint8, device=dev)
+checl.debug_fill(big, 9, 0)
+torch.cuda.synchronize()
+for i in range(40000):
+    ctx.register(big[i * 40:i * 40 + 33])
+d = ctx.checkpoint_device(dev, epoch=8)
+ctx.restore(d, dev)
+d.free()
+ctx.close()
 print("sanitize ok")
