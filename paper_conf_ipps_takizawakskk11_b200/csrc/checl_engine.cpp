@@ -2193,6 +2193,10 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
       // so the one-GPU test box runs K2's peer-read path (register loads for every round)
       static const bool force_remote = std::getenv("CHECL_FORCE_IMAGE_REMOTE") != nullptr;
       lp.image_remote = img->device != device || force_remote;
+#ifdef CHECL_EXPERIMENTS
+      static const bool peer_bulk = std::getenv("CHECL_PEER_BULK") != nullptr;
+      lp.remote_bulk = peer_bulk;
+#endif
     }
     lp.c0 = 0;
     lp.c1 = nch;
@@ -2225,7 +2229,7 @@ checl_status do_restore(checl_ctx* ctx, const checl_image* img, int device, void
       lp.c1 = nch;
       lp.image = const_cast<uint8_t*>(mapped + P.L.payload_off);
       lp.image_base = 0;
-      lp.image_remote = 1;  // not HBM: register loads only
+      lp.image_remote = 2;  // mapped pinned host memory: register loads only
       lp.crc = reinterpret_cast<uint32_t*>(const_cast<uint8_t*>(mapped + P.L.crc_off));
       timed_launch(ds, kt, kOpVerify, lp, ds.compute);
       ck(cudaEventRecord(c_end, ds.compute));

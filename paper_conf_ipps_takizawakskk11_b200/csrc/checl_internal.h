@@ -171,8 +171,12 @@ struct LaunchParams {
   // pinned host memory) from its last CTA and resets status to {~0, 0, 0}; nullptr:
   // status is left as accumulated
   unsigned long long* status_host;
-  // the image is a peer GPU's memory (NVLink): no bulk (TMA) loads from it
+  // the image is not this GPU's HBM: 1 = a peer GPU's memory (NVLink), 2 = mapped
+  // pinned host memory (PCIe). Rounds from it take the register path (16-byte loads),
+  // except peer images when remote_bulk is set (experiments build, CHECL_PEER_BULK=1:
+  // cp.async.bulk straight from the peer's HBM, for A/B on a box with two GPUs)
   int image_remote;
+  int remote_bulk;
   // diagnostics (CHECL_WARP_TRACE): per warp {start, tables ready, end, smid}
   unsigned long long* warp_trace;
   // balanced / TMA kernels: the first static_permille/1000 of the rounds go to the

@@ -799,7 +799,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
     q.r0 = (int)(g - rb);
     q.r1 = (int)(ge - rb < (uint64_t)q.nrounds ? ge - rb : (uint64_t)q.nrounds);
     q.bulk_ok = q.mode == 0 && ((reinterpret_cast<uintptr_t>(q.src) & 15u) == 0) &&
-                (!O::kStore || (reinterpret_cast<uintptr_t>(q.dst) & 15u) == 0) && !(O::kSrcImg && p.image_remote);
+                (!O::kStore || (reinterpret_cast<uintptr_t>(q.dst) & 15u) == 0) && !(O::kSrcImg && p.image_remote && !(p.image_remote == 1 && p.remote_bulk));
     return q;
   };
   auto is_bulk = [&](const Part& q, int r) { return q.bulk_ok && (uint32_t)(r + 1) * kRoundBytes <= q.len; };

@@ -73,7 +73,8 @@ print("kernel ok")
 
 
 @pytest.mark.parametrize("kernel", ["1", "2", "3", "4", "4:0:1", "4:500:3", "4:900:16", "4:0:1:mc", "4:500:3:mc",
-                                    "0:remote", "4:remote", "4:0:1:remote", "0:nopeer", "4:nopeer", "0:nozc"])
+                                    "0:remote", "4:remote", "4:0:1:remote", "0:nopeer", "4:nopeer", "0:nozc",
+                                    "4:peerbulk"])
 def test_forced_kernel_shapes_bit_exact(kernel):
     """kernel "4:S:B" = the TMA kernel with the dynamic tail forced on at this size:
     static share S permille, dynamic blocks of B rounds (S = 0: every round dynamic;
@@ -86,6 +87,10 @@ def test_forced_kernel_shapes_bit_exact(kernel):
     the default dispatch."""
     k, *dyn = kernel.split(":")
     env = dict(os.environ, CHECL_KERNEL=k)
+    if dyn and dyn[-1] == "peerbulk":  # the peer path with bulk copies (experiments build, CHECL_PEER_BULK)
+        env.update(CHECL_FORCE_IMAGE_REMOTE="1", CHECL_PEER_BULK="1",
+                   CHECL_LIB=os.path.join(ROOT, "paper_conf_ipps_takizawakskk11_b200", "libchecl_exp.so"))
+        dyn = dyn[:-1]
     if dyn and dyn[-1] == "remote":  # K2 on an HBM image takes the peer-GPU read path (migration i -> j)
         env.update(CHECL_FORCE_IMAGE_REMOTE="1")
         dyn = dyn[:-1]
