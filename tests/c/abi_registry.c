@@ -56,6 +56,12 @@ int main(void) {
   CHECK(checl_image_view(img, &v, &vn) == CHECL_SUCCESS && v == bytes && vn == sizeof bytes);
   int loc = -1;
   CHECK(checl_image_info(img, &loc, &d, NULL, NULL) == CHECL_SUCCESS && loc == CHECL_IMAGE_HOST && d == -1);
+  /* incremental checkpoint: an unknown dirty rule and missing outputs are refused up front */
+  checl_image* delta = NULL;
+  CHECK(checl_checkpoint_incremental_ex(ctx, 0, NULL, 1, img, 2, &delta) == CHECL_ERR_INVALID_VALUE && !delta);
+  CHECK(checl_checkpoint_incremental_ex(ctx, 0, NULL, 1, img, CHECL_DIRTY_BYTES, NULL) == CHECL_ERR_INVALID_VALUE);
+  CHECK(checl_checkpoint_incremental(ctx, 0, NULL, 1, NULL, &delta) == CHECL_ERR_INVALID_VALUE);
+  CHECK(CHECL_DIRTY_CRC == 0 && CHECL_DIRTY_BYTES == 1);
   CHECK(checl_image_free(img) == CHECL_SUCCESS);
   CHECK(checl_image_free(NULL) == CHECL_SUCCESS);
   checl_timing t;
@@ -64,6 +70,7 @@ int main(void) {
   CHECK(checl_stats_get(ctx, CHECL_STATS_RESTORE, &st) == CHECL_SUCCESS && st.n_calls == 0 && st.kernel_ms == 0.0);
   CHECK(checl_stats_get(ctx, CHECL_STATS_KINDS, &st) == CHECL_ERR_INVALID_VALUE);
   CHECK(checl_stats_reset(ctx) == CHECL_SUCCESS);
+  CHECK(checl_trim(ctx) == CHECL_SUCCESS); /* nothing kept: no device work */
   CHECK(checl_destroy(ctx) == CHECL_SUCCESS);
   printf("abi_registry ok\n");
   return 0;
