@@ -3382,6 +3382,17 @@ checl_status checl_trim(checl_ctx* ctx) {
       }
     }
     free_arenas(drop);
+    // the exact incremental rule's device copy of the last delta's state: the next exact
+    // delta reseeds it from a full base, or writes a full image (reading 25)
+    BusyGuard b(ctx);
+    if (b.ok)
+      for (DevState* ds : ctx->devs)
+        if (ds && ds->shadow.p) {
+          DeviceGuard g(ds->dev);
+          ck(cudaDeviceSynchronize());
+          ds->shadow.release();
+          ds->shadow_ok = false;
+        }
     pinned_pool().trim();
     return CHECL_SUCCESS;
   });

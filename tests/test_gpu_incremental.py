@@ -293,3 +293,25 @@ def test_exact_rule_shadow_follows_the_chain_and_reseeds(ctx):
     _eq(D5.view(), _odelta(ds, Fo, Fo, 5, checl.DIRTY_BYTES), "D5 on F")
     del full2
     release_all(ctx, ds)
+
+
+def test_trim_releases_the_shadow(ctx):
+    """checl_trim frees the exact rule's device copy of the last delta's state: a delta
+    on that delta's base then has no state to compare with and is the full image; one on
+    a full host base reseeds the copy and is exact again (reading 25)."""
+    rng = np.random.default_rng(35)
+    ds = make_set(ctx, [200000, 70001, 5], seed=12)
+    F = ctx.checkpoint(DEV, epoch=0)
+    Fo = O.checkpoint(oracle_entries(ds), device=DEV, epoch=0)
+    _mutate(ds, _random_changes(ds, rng, 3))
+    D1 = ctx.checkpoint_incremental(DEV, F, epoch=1)
+    _eq(D1.view(), _odelta(ds, Fo, Fo, 1, checl.DIRTY_BYTES), "D1")
+    ctx.trim()
+    _mutate(ds, _random_changes(ds, rng, 3))
+    X = ctx.checkpoint_incremental(DEV, D1, epoch=2)
+    assert X.header()["flags"] == 0
+    _eq(X.view(), O.checkpoint(oracle_entries(ds), device=DEV, epoch=2), "full after trim")
+    ctx.trim()
+    D3 = ctx.checkpoint_incremental(DEV, F, epoch=3)  # full host base: reseeded from F
+    _eq(D3.view(), _odelta(ds, Fo, Fo, 3, checl.DIRTY_BYTES), "D3 on F")
+    release_all(ctx, ds)
