@@ -6,6 +6,16 @@
 // image layout of FORMAT.md. The data path runs in checl_kernels.cu; this file
 // plans it (flat chunk list, stages), drives the staging pipeline on two streams
 // (copy engine D2H/H2D overlapped with the pack / verify kernels), and commits.
+//
+// State kept across calls:
+//   Plan         per device: the registry's chunk list, stages, header + manifest and
+//                their meta-CRC register, cached per registry version;
+//   LayoutCache  per device: the last full-image restore's layout (restore fast path);
+//   Binding      per commit: where its records live (segment + offset) and the
+//                segments themselves (re-created buffers, reading 18);
+//   spares       per device: the segments the last commit released (next restore);
+//   shadow       per device: the exact incremental rule's copy of the last delta's
+//                state (reading 25).
 #include <cuda_runtime.h>
 #include <fcntl.h>
 #include <signal.h>
