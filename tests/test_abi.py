@@ -174,6 +174,21 @@ F = checl.Image.read(os.path.join(tmp, "full1.checl"))
 D = checl.Image.read(os.path.join(tmp, "delta1.checl"))
 st, want = O.merge(full, delta)
 assert st == 0 and np.array_equal(F.merge(D).view(), want)
+# a delta of the exact (bytes) dirty rule parses and merges in the library like the
+# oracle's (FORMAT.md dirty_rule = 1); an unknown rule value is BAD_IMAGE
+delta_b = O.checkpoint_incremental(ents, full, device=0, epoch=8, rule=O.RULE_BYTES, base_full=full)
+st, want_b = O.merge(full, delta_b)
+Db = checl.Image.wrap(delta_b)
+assert st == 0 and Db.header()["dirty_rule"] == 1 and np.array_equal(F.merge(Db).view(), want_b)
+bad_rule = bytearray(delta_b.tobytes())
+struct.pack_into("<I", bad_rule, 108, 2)
+poff = struct.unpack_from("<Q", bad_rule, 56)[0]
+struct.pack_into("<I", bad_rule, 124, O.crc32c(bytes(bad_rule[:124]) + bytes(bad_rule[128:poff])))
+try:
+    F.merge(checl.Image.wrap(np.frombuffer(bytes(bad_rule), np.uint8)))
+    raise SystemExit("dirty_rule 2 accepted")
+except checl.CheclError as e:
+    assert e.status == checl.ERR_BAD_IMAGE
 # damaged files are refused at read
 p = os.path.join(tmp, "full1.checl")
 raw = bytearray(open(p, "rb").read())
