@@ -85,6 +85,64 @@ thread_local std::string t_last_cuda_error;
 constexpr int kMaxSignal = 65;
 std::atomic<checl_ctx*> g_signal_ctx[kMaxSignal];
 
+// Pinned host memory for images. cudaHostAlloc pins at ~2.4-2.8 GB/s on the B200
+// boxes (page by page, one thread); a large buffer is instead taken 2 MiB-aligned with
+// transparent huge pages requested, faulted in by several threads at once and
+// registered with one cudaHostRegister: 26-30 GB/s for 4-8 GiB, copies at the same
+// PCIe rate (tools/microbench/pin_rate.cu, profiles/r02/pin_rate.txt). Small buffers
+// keep cudaHostAlloc. pin_free knows which is which.
+constexpr size_t kFastPinMin = 64ull << 20;
+std::mutex g_reg_mu;
+std::unordered_set<void*> g_registered;  // buffers of pin_alloc's registered path
+
+void* pin_alloc(size_t n) {
+  if (n >= kFastPinMin) {
+    void* p = nullptr;
+    if (posix_memalign(&p, 2u << 20, n) == 0) {
+      madvise(p, n, MADV_HUGEPAGE);  // (advice only: 4 KiB pages still work)
+      const unsigned hw = std::thread::hardware_concurrency();
+      const size_t T = std::max<size_t>(1, std::min<size_t>(16, hw ? hw : 4));
+      const size_t piece = (n / T + (2u << 20) - 1) & ~(size_t)((2u << 20) - 1);
+      std::vector<std::thread> th;
+      for (size_t t = 0; t < T && t * piece < n; ++t)
+        th.emplace_back([=] {
+          volatile uint8_t* q = static_cast<uint8_t*>(p) + t * piece;
+          const size_t m = std::min(piece, n - t * piece);
+          for (size_t o = 0; o < m; o += 4096) q[o] = 0;
+        });
+      for (auto& x : th) x.join();
+      if (cudaHostRegister(p, n, cudaHostRegisterPortable | cudaHostRegisterMapped) == cudaSuccess) {
+        std::lock_guard<std::mutex> lk(g_reg_mu);
+        g_registered.insert(p);
+        return p;
+      }
+      cudaGetLastError();
+      std::free(p);
+    }
+  }
+  void* p = nullptr;
+  if (cudaHostAlloc(&p, n, cudaHostAllocPortable | cudaHostAllocMapped) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return p;
+}
+
+void pin_free(void* p) {
+  if (!p) return;
+  bool reg = false;
+  {
+    std::lock_guard<std::mutex> lk(g_reg_mu);
+    reg = g_registered.erase(p) != 0;
+  }
+  if (reg) {
+    cudaHostUnregister(p);
+    std::free(p);
+  } else {
+    cudaFreeHost(p);
+  }
+}
+
 // Pinned host buffers of freed library-owned images, kept for the next image
 // (cudaHostAlloc pins ~2.4 GB/s on the B200 boxes: an incremental checkpoint loop, or
 // a file restore loop, would otherwise pin a new image every step). Bounded by
@@ -132,7 +190,7 @@ struct PinnedPool {
       all.swap(free_);
       bytes = 0;
     }
-    for (auto& e : all) cudaFreeHost(e.second);
+    for (auto& e : all) pin_free(e.second);
   }
   void give(void* p, size_t cap) {
     std::vector<void*> drop;
@@ -150,7 +208,7 @@ struct PinnedPool {
         }
       }
     }
-    for (void* d : drop) cudaFreeHost(d);
+    for (void* d : drop) pin_free(d);
   }
 };
 PinnedPool& pinned_pool() {
@@ -685,7 +743,8 @@ struct checl_image {
     if (want_pinned) {
       cap = pinned_class(cap);
       p = pinned_pool().take(cap, &cap);
-      if (!p) ck(cudaHostAlloc(&p, cap, cudaHostAllocDefault));
+      if (!p) p = pin_alloc(cap);
+      if (!p) ck(cudaErrorMemoryAllocation);
     } else {
       p = std::malloc(std::max<size_t>(n, 1));
       if (!p) throw std::bad_alloc();
@@ -3338,8 +3397,7 @@ checl_status checl_image_read(const char* path, uint32_t flags, checl_image** ou
     void* p = nullptr;
     size_t pcap = cap;
     // pinned when a device is present (restore then fills over PCIe at full rate)
-    if (device_count() > 0 && ((p = pinned_pool().take(cap, &pcap)) != nullptr ||
-                               cudaHostAlloc(&p, cap, cudaHostAllocDefault) == cudaSuccess)) {
+    if (device_count() > 0 && ((p = pinned_pool().take(cap, &pcap)) != nullptr || (p = pin_alloc(cap)) != nullptr)) {
       img->pinned = true;
     } else {
       cudaGetLastError();
