@@ -89,9 +89,9 @@ std::atomic<checl_ctx*> g_signal_ctx[kMaxSignal];
 // boxes (page by page, one thread); a large buffer is instead taken 2 MiB-aligned with
 // transparent huge pages requested, faulted in by several threads at once and
 // registered with one cudaHostRegister: 26-30 GB/s for 4-8 GiB, copies at the same
-// PCIe rate (tools/microbench/pin_rate.cu, profiles/r02/pin_rate.txt). Small buffers
-// keep cudaHostAlloc. pin_free knows which is which.
-constexpr size_t kFastPinMin = 64ull << 20;
+// PCIe rate (tools/microbench/pin_rate.cu, profiles/r02/pin_rate.txt). Buffers under
+// 8 MiB keep cudaHostAlloc. pin_free knows which is which.
+constexpr size_t kFastPinMin = 8ull << 20;
 std::mutex g_reg_mu;
 std::unordered_set<void*> g_registered;  // buffers of pin_alloc's registered path
 
@@ -100,16 +100,18 @@ void* pin_alloc(size_t n) {
     void* p = nullptr;
     if (posix_memalign(&p, 2u << 20, n) == 0) {
       madvise(p, n, MADV_HUGEPAGE);  // (advice only: 4 KiB pages still work)
+      // one thread per 32 MiB, at most 16 (and the machine's count)
       const unsigned hw = std::thread::hardware_concurrency();
-      const size_t T = std::max<size_t>(1, std::min<size_t>(16, hw ? hw : 4));
+      const size_t T = std::max<size_t>(1, std::min<size_t>({16, hw ? hw : 4, n >> 25}));
       const size_t piece = (n / T + (2u << 20) - 1) & ~(size_t)((2u << 20) - 1);
+      auto touch = [=](size_t t) {
+        volatile uint8_t* q = static_cast<uint8_t*>(p) + t * piece;
+        const size_t m = std::min(piece, n - t * piece);
+        for (size_t o = 0; o < m; o += 4096) q[o] = 0;
+      };
       std::vector<std::thread> th;
-      for (size_t t = 0; t < T && t * piece < n; ++t)
-        th.emplace_back([=] {
-          volatile uint8_t* q = static_cast<uint8_t*>(p) + t * piece;
-          const size_t m = std::min(piece, n - t * piece);
-          for (size_t o = 0; o < m; o += 4096) q[o] = 0;
-        });
+      for (size_t t = 1; t < T && t * piece < n; ++t) th.emplace_back(touch, t);
+      touch(0);
       for (auto& x : th) x.join();
       if (cudaHostRegister(p, n, cudaHostRegisterPortable | cudaHostRegisterMapped) == cudaSuccess) {
         std::lock_guard<std::mutex> lk(g_reg_mu);
