@@ -92,8 +92,16 @@ std::atomic<checl_ctx*> g_signal_ctx[kMaxSignal];
 // PCIe rate (tools/microbench/pin_rate.cu, profiles/r02/pin_rate.txt). Buffers under
 // 8 MiB keep cudaHostAlloc. pin_free knows which is which.
 constexpr size_t kFastPinMin = 8ull << 20;
-std::mutex g_reg_mu;
-std::unordered_set<void*> g_registered;  // buffers of pin_alloc's registered path
+// buffers of pin_alloc's registered path (never destroyed: images may be freed while
+// the process exits, after static destructors ran)
+struct Registered {
+  std::mutex mu;
+  std::unordered_set<void*> set;
+};
+Registered& registered() {
+  static Registered* r = new Registered();
+  return *r;
+}
 
 void* pin_alloc(size_t n) {
   if (n >= kFastPinMin) {
@@ -114,8 +122,8 @@ void* pin_alloc(size_t n) {
       touch(0);
       for (auto& x : th) x.join();
       if (cudaHostRegister(p, n, cudaHostRegisterPortable | cudaHostRegisterMapped) == cudaSuccess) {
-        std::lock_guard<std::mutex> lk(g_reg_mu);
-        g_registered.insert(p);
+        std::lock_guard<std::mutex> lk(registered().mu);
+        registered().set.insert(p);
         return p;
       }
       cudaGetLastError();
@@ -134,8 +142,8 @@ void pin_free(void* p) {
   if (!p) return;
   bool reg = false;
   {
-    std::lock_guard<std::mutex> lk(g_reg_mu);
-    reg = g_registered.erase(p) != 0;
+    std::lock_guard<std::mutex> lk(registered().mu);
+    reg = registered().set.erase(p) != 0;
   }
   if (reg) {
     cudaHostUnregister(p);
