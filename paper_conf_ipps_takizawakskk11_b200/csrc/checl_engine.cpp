@@ -333,8 +333,8 @@ TableParams table_params() {
   tp.horner = gf_x8n(kRoundBytes - kSegBytes);
   for (int l = 0; l < 32; ++l) tp.lanepow[l] = gf_x8n((uint64_t)kSegBytes * (31 - l));
   for (int k = 0; k < 16; ++k) tp.unitpow[k] = gf_x8n((uint64_t)kRoundBytes * k);
-  tp.col_shift = gf_x8n(kSegBytes);
-  for (int k = 0; k < kFoldLevels; ++k) {
+  tp.col_shift = gf_x8n((uint64_t)kSegBytes * kColChains);
+  for (int k = 0; k < kColFoldLevels; ++k) {
     uint32_t r = kOne;
     for (int i = 0; i < 32 << k; ++i) r = gf_divx(r);  // x^(-32 * 2^k)
     tp.col_fold[k] = r;

@@ -127,11 +127,19 @@ constexpr int kHornerWords = 8 * 16 * 32;       // x^(8*3968) nibble tables, 16 
 constexpr int kFoldWords = kFoldLevels * 8 * 16; // fold nibble tables, 2.5 KiB
 constexpr int kPosWords = 8 * 16 * 32;          // sweep: lane-position nibble tables, 16 KiB
 constexpr int kUnitWords = 16 * 32;             // sweep: x^(8*4096*k) * x^i, 2 KiB
-// TMA kernel (column CRC): lane l chains word l of every 128-byte row,
-// so its step is v -> v * x^(8*128) (slicing-by-4 tables of that shift, same
-// lane-private layout), and the lanes are combined with shifts x^(-32*2^k).
+// TMA kernel (column CRC): lane l takes word l of every 128-byte row
+// in kColChains independent chains (chain c: the rows = c mod kColChains), so a
+// chain's step is v -> v * x^(8*128*kColChains) (slicing-by-4 tables of that shift,
+// same lane-private layout); a lane's chains are combined with the shift x^(-1024)
+// (fold level kFoldLevels) and the lanes with shifts x^(-32*2^k).
+#ifndef CHECL_COL_CHAINS
+#define CHECL_COL_CHAINS 4
+#endif
+constexpr int kColChains = CHECL_COL_CHAINS;
+static_assert(kColChains == 1 || kColChains == 2 || kColChains == 4 || kColChains == 8, "chains divide 32 rows");
+constexpr int kColFoldLevels = kFoldLevels + 1;  // + x^(-32*32): one row of the tile
 constexpr int kColWords = 4 * 256 * 32;          // 128 KiB
-constexpr int kColFoldWords = kFoldLevels * 8 * 16;  // 2.5 KiB
+constexpr int kColFoldWords = kColFoldLevels * 8 * 16;  // 3 KiB
 constexpr int kTabOff = 0;
 constexpr int kHornerOff = kTabOff + kTabWords;
 constexpr int kFoldOff = kHornerOff + kHornerWords;
@@ -148,8 +156,8 @@ struct TableParams {
   uint32_t horner;             // x^(8 * (kRoundBytes - kSegBytes)) mod P
   uint32_t lanepow[32];        // x^(8 * 128 * (31 - l)) mod P
   uint32_t unitpow[16];        // x^(8 * 4096 * k) mod P
-  uint32_t col_shift;          // x^(8 * 128) mod P
-  uint32_t col_fold[kFoldLevels];  // x^(-32 * 2^k) mod P
+  uint32_t col_shift;          // x^(8 * 128 * kColChains) mod P
+  uint32_t col_fold[kColFoldLevels];  // x^(-32 * 2^k) mod P
 };
 
 // Parameters of one launch over the chunk range [c0, c1) of `desc`. Payload byte

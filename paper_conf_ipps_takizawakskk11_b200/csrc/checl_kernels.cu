@@ -657,13 +657,16 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) balanced_kernel(const Launc
 // the LSU carries only the CRC's shared loads. Partial, misaligned or remote rounds
 // take the register path (16-byte loads, stores from registers, exact tails) and
 // are written into the same tile. The tile is contiguous, so the CRC reads it by
-// columns: lane l chains word l of every 128-byte row (conflict-free LDS.32), a
-// chain of stride 128 B that runs across rounds unchanged:
-//   h <- (h ^ w) * x^(8*128)           (slicing-by-4 over tables of that shift)
+// columns: lane l reads word l of every 128-byte row (conflict-free LDS.32) and
+// chains it, a column of stride 128 B that runs across rounds unchanged:
+//   h <- (h ^ w) * x^(8*128)
 // With D = the part's bytes zero-padded to whole rounds, n = |D|, word i = l + 32k,
 //   R(D, s) = XOR_i R(w_i, 0) x^(8(n - 4i - 4)) = XOR_l h_l x^(-32 l),
 // (s folded into lane 0's first word), the lanes combined by a shuffle tree with
-// shifts x^(-32*2^k). The rest (zero-padding correction, split-chunk terms) is the
+// shifts x^(-32*2^k). The column is split into kColChains independent chains (rows
+// = c mod kColChains, step x^(8*128*kColChains), slicing-by-4 over tables of that
+// shift) so that a lane has kColChains lookups in flight instead of one:
+//   h_l = XOR_c ch_c x^(-1024 c). The rest (zero-padding correction, split-chunk terms) is the
 // balanced kernel's.
 constexpr int kTmaTiles = 2;
 constexpr size_t kTmaColOff = 0;
@@ -851,7 +854,10 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
       srb = p.round_base[s_c];
     }
     Part nxt = cur;
-    uint32_t ch = (lane == 0 && cur.r0 == 0) ? 0xFFFFFFFFu : 0u;
+    uint32_t ch[kColChains];  // chain c: rows = c mod kColChains (the CRC init enters row 0)
+    ch[0] = (lane == 0 && cur.r0 == 0) ? 0xFFFFFFFFu : 0u;
+#pragma unroll
+    for (int c = 1; c < kColChains; ++c) ch[c] = 0u;
     for (int r = cur.r0; r < cur.r1; ++r) {
       uint8_t* tile = tiles + t * kRoundBytes;
       // the bulk stores of earlier rounds have finished reading their tiles
@@ -912,14 +918,19 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
       if (O::kCrc) {
 #pragma unroll
         for (int q = 0; q < 32; ++q)
-          ch = crc_step4(ch, *reinterpret_cast<const uint32_t*>(tile + q * kSegBytes + l4), tb, l4);
+          ch[q % kColChains] =
+              crc_step4(ch[q % kColChains], *reinterpret_cast<const uint32_t*>(tile + q * kSegBytes + l4), tb, l4);
       }
       fence_proxy_async();  // this round's shared reads before the next bulk copy into the tile
       __syncwarp();
       t ^= 1;
     }
-    uint32_t f = ch;
+    // chain c stepped every row it holds by x^(1024*kColChains), i.e. c rows too far:
+    // h = XOR_c ch[c] * x^(-1024 c) (Horner), then the lanes as before
+    uint32_t f = ch[kColChains - 1];
     if (O::kCrc) {
+#pragma unroll
+      for (int c = kColChains - 2; c >= 0; --c) f = fold_mul(f, ftab + kFoldLevels * 128) ^ ch[c];
 #pragma unroll
       for (int k = 0; k < kFoldLevels; ++k) {
         const uint32_t o = __shfl_down_sync(full, f, 1 << k);
@@ -1136,9 +1147,9 @@ __global__ void build_tables_kernel(const TableParams tp, uint32_t* __restrict__
     for (int m = 0; m < (t & 31); ++m) b = gf_mulx(b);
     out[kUnitOff + t] = b;
   }
-  // column tables (TMA kernel): C_j[e] = (e << 8j) * x^(8*128), byte j of the
-  // register, in the super-table layout (A = [C_0 | C_1], B = [C_2 | C_3]); fold
-  // tables of the shifts x^(-32*2^k)
+  // column tables (TMA kernel): C_j[e] = (e << 8j) * x^(8*128*kColChains), byte j of
+  // the register, in the super-table layout (A = [C_0 | C_1], B = [C_2 | C_3]); fold
+  // tables of the shifts x^(-32*2^k), k <= kFoldLevels (the last one combines chains)
   __syncthreads();
   for (int e = threadIdx.x; e < 1024; e += blockDim.x) scratch[e] = gf_mul((uint32_t)(e & 255) << (8 * (e >> 8)), tp.col_shift);
   __syncthreads();

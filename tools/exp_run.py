@@ -15,6 +15,7 @@ ap = argparse.ArgumentParser()
 ap.add_argument("--config", default="C2")
 ap.add_argument("--reps", type=int, default=10)
 ap.add_argument("--kind", type=int, default=0)
+ap.add_argument("--incr", action="store_true", help="also time the CRC-rule incremental pass (nothing dirty)")
 a = ap.parse_args()
 w = synth.CONFIGS[a.config]()
 ts = [torch.empty(b.size, dtype=torch.uint8, device=0) for b in w.buffers]
@@ -38,5 +39,15 @@ for i in range(a.reps + 2):
         vf.append(tv)
 S = w.total_bytes
 p, v = statistics.median(pk), statistics.median(vf)
+if a.incr:
+    base = ctx.checkpoint(0, epoch=0)
+    ci = []
+    for i in range(a.reps + 2):
+        d = ctx.checkpoint_incremental(0, base, epoch=i + 1, rule=checl.DIRTY_CRC)
+        if i >= 2:
+            ci.append(ctx.last_timing()["kernel_ms"])
+        d.free()
+    c = statistics.median(ci)
+    print(f"  crc-rule incremental kernels {c*1e3:.1f} us ({S/c/1e6:.0f} GB/s read)")
 print(f"{os.path.basename(os.path.dirname(os.environ.get('CHECL_LIB', 'default/x')))} op={os.environ.get('CHECL_EXP_PACK_OP', 0)} {a.config}: pack {p*1e3:.1f} us "
       f"({2*S/p/1e6:.0f} GB/s 2S), verify {v*1e3:.1f} us ({2*S/v/1e6:.0f} GB/s 2S)")
