@@ -207,7 +207,11 @@ class Image:
         _check(lib.checl_image_view(self.handle, C.byref(b), C.byref(n)), "checl_image_view")
         if n.value == 0:
             return np.zeros(0, dtype=np.uint8)
-        arr = np.ctypeslib.as_array(C.cast(b, C.POINTER(C.c_uint8)), shape=(n.value,))
+        # the array keeps this Image alive (a view of a temporary, e.g. a.merge(d).view(),
+        # must not outlive the image's memory); free() still ends it
+        buf = (C.c_uint8 * n.value).from_address(b.value)
+        buf._image = self
+        arr = np.frombuffer(buf, dtype=np.uint8)
         arr.flags.writeable = False
         return arr
 

@@ -174,6 +174,17 @@ F = checl.Image.read(os.path.join(tmp, "full1.checl"))
 D = checl.Image.read(os.path.join(tmp, "delta1.checl"))
 st, want = O.merge(full, delta)
 assert st == 0 and np.array_equal(F.merge(D).view(), want)
+# a view keeps its image alive (the merged image above is a temporary)
+import gc, weakref
+m = F.merge(D)
+w = weakref.ref(m)
+v = m.view()
+del m
+gc.collect()
+assert w() is not None and np.array_equal(v, want)
+del v
+gc.collect()
+assert w() is None
 # a delta of the exact (bytes) dirty rule parses and merges in the library like the
 # oracle's (FORMAT.md dirty_rule = 1); an unknown rule value is BAD_IMAGE
 delta_b = O.checkpoint_incremental(ents, full, device=0, epoch=8, rule=O.RULE_BYTES, base_full=full)
