@@ -16,11 +16,16 @@ ap.add_argument("--config", default="C2")
 ap.add_argument("--reps", type=int, default=10)
 ap.add_argument("--kind", type=int, default=0)
 ap.add_argument("--incr", action="store_true", help="also time the CRC-rule incremental pass (nothing dirty)")
+ap.add_argument("--mib", type=int, default=0, help="one buffer of this many MiB instead of a config")
 a = ap.parse_args()
-w = synth.CONFIGS[a.config]()
-ts = [torch.empty(b.size, dtype=torch.uint8, device=0) for b in w.buffers]
-for t, b in zip(ts, w.buffers):
-    checl.debug_fill(t, w.seed, b.stream, a.kind)
+if a.mib:
+    sizes, seed, streams = [a.mib << 20], 1, [0]
+else:
+    w = synth.CONFIGS[a.config]()
+    sizes, seed, streams = [b.size for b in w.buffers], w.seed, [b.stream for b in w.buffers]
+ts = [torch.empty(n, dtype=torch.uint8, device=0) for n in sizes]
+for t, st in zip(ts, streams):
+    checl.debug_fill(t, seed, st, a.kind)
 torch.cuda.synchronize()
 ctx = checl.Context()
 hs = [ctx.register(t) for t in ts]
@@ -37,7 +42,7 @@ for i in range(a.reps + 2):
     if i >= 2:
         pk.append(tp)
         vf.append(tv)
-S = w.total_bytes
+S = sum(sizes)
 p, v = statistics.median(pk), statistics.median(vf)
 if a.incr:
     base = ctx.checkpoint(0, epoch=0)
@@ -49,5 +54,5 @@ if a.incr:
         d.free()
     c = statistics.median(ci)
     print(f"  crc-rule incremental kernels {c*1e3:.1f} us ({S/c/1e6:.0f} GB/s read)")
-print(f"{os.path.basename(os.path.dirname(os.environ.get('CHECL_LIB', 'default/x')))} op={os.environ.get('CHECL_EXP_PACK_OP', 0)} {a.config}: pack {p*1e3:.1f} us "
+print(f"{os.path.basename(os.path.dirname(os.environ.get('CHECL_LIB', 'default/x')))} op={os.environ.get('CHECL_EXP_PACK_OP', 0)} {a.config if not a.mib else str(a.mib) + 'MiB'}: pack {p*1e3:.1f} us "
       f"({2*S/p/1e6:.0f} GB/s 2S), verify {v*1e3:.1f} us ({2*S/v/1e6:.0f} GB/s 2S)")
