@@ -1260,27 +1260,40 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
   // CHECL_DYN_MIN_ROUNDS overrides (sweeps, and the kernel-shape tests that force the
   // tail on at small sizes)
 #ifdef CHECL_EXPERIMENTS
-  static const uint32_t static_pm = [] {
+  static const int env_pm = [] {
     const char* e = std::getenv("CHECL_STATIC_PERMILLE");
-    return e ? (uint32_t)std::min(1000, std::max(0, std::atoi(e))) : 750u;
+    return e ? std::min(1000, std::max(0, std::atoi(e))) : -1;
   }();
-  static const uint32_t dyn_block = [] {
+  static const int env_blk = [] {
     const char* e = std::getenv("CHECL_DYN_BLOCK");
-    return e ? (uint32_t)std::max(1, std::atoi(e)) : 8u;
+    return e ? std::max(1, std::atoi(e)) : -1;
   }();
   static const uint64_t dyn_min = [] {
     const char* e = std::getenv("CHECL_DYN_MIN_ROUNDS");
     return e ? (uint64_t)std::strtoull(e, nullptr, 10) : ~0ull;
   }();
 #else
-  constexpr uint32_t static_pm = 750u, dyn_block = 8u;
+  constexpr int env_pm = -1, env_blk = -1;
   constexpr uint64_t dyn_min = ~0ull;
 #endif
+  // The split by rounds per warp (rpw; chunks x 16 bounds the rounds), from the sweeps
+  // in profiles/r02/split_sweep (pack / verify us, static permille : block rounds):
+  //   rpw < 16 (64 MiB: 11)   static only   (37 us; 500:4 40, 640:2 42)
+  //   rpw < 64 (128-256 MiB)  500 : 4       (128 MiB 59 vs 64 static; 256 MiB 99 vs 112)
+  //   rpw < 256 (C2: 76)      500 : 8       (C2 159.5 vs 166 with 750 : 8)
+  //   otherwise (C3, 4 GiB)   750 : 8       (C3 1626; 850 : 8 1640, 950 : 8 1775;
+  //                                          4 GiB 1295; 900 : 8 1380)
+  // A larger static share loses to the SMs' position-dependent bulk-copy rate (the
+  // slowest stretch sets the end), a smaller one or smaller blocks to the per-block
+  // fetch, chunk search and split-chunk accounting.
   // (kernel 3 keeps static stretches only: measured slower with the dynamic tail)
-  // (a dynamic tail pays when a warp has tens of rounds: measured 64 MiB launches (11
-  // rounds per warp) 37 -> 49 us with it, 463 MB (76 per warp) 169 -> 164 us)
-  const uint64_t min_rounds = dyn_min != ~0ull ? dyn_min : (uint64_t)ds.n_sms * kWarpsPerCta * 48;
-  if (kernel == 4 && static_pm < 1000 && chunks * (kChunkBytes / kRoundBytes) >= min_rounds) {
+  const uint64_t rounds_ub = chunks * (kChunkBytes / kRoundBytes);
+  const uint64_t rpw = rounds_ub / ((uint64_t)ds.n_sms * kWarpsPerCta);
+  const uint64_t min_rounds = dyn_min != ~0ull ? dyn_min : (uint64_t)ds.n_sms * kWarpsPerCta * 16;
+  uint32_t static_pm = rpw < 256 ? 500u : 750u, dyn_block = rpw < 64 ? 4u : 8u;
+  if (env_pm >= 0) static_pm = (uint32_t)env_pm;
+  if (env_blk >= 0) dyn_block = (uint32_t)env_blk;
+  if (kernel == 4 && static_pm < 1000 && rounds_ub >= min_rounds) {
     p.work = ds.work.p;
     p.static_permille = static_pm;
     p.dyn_block = dyn_block;
