@@ -498,6 +498,34 @@ def meminfo_available() -> int:
     return 0
 
 
+def copy_same_size(torch, dev: int, S: int, achieved: float) -> dict:
+    """Context for the roofline: torch's own device copy (b.copy_(a), the op the
+    MEASURED_PEAKS.json copy peak is taken with, at 2 GiB) of the workload's payload
+    size, CUDA events around each copy, median of 5 after one warm-up. Not the peak:
+    a copy's rate depends on its size."""
+    free, _ = torch.cuda.mem_get_info(dev)
+    if 2 * S + (1 << 30) > free:
+        return {"GBs": None, "reason": f"needs 2 x {S} B of free HBM ({free} B free)"}
+    a = torch.empty(S, dtype=torch.uint8, device=dev)
+    b = torch.empty_like(a)
+    a.fill_(1)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    ts = []
+    for i in range(6):
+        torch.cuda.synchronize(dev)
+        e0.record()
+        b.copy_(a)
+        e1.record()
+        torch.cuda.synchronize(dev)
+        if i:
+            ts.append(e0.elapsed_time(e1))
+    del a, b
+    torch.cuda.empty_cache()
+    ts.sort()
+    rate = 2 * S / (ts[len(ts) // 2] * 1e-3) / 1e9
+    return {"GBs": rate, "frac": achieved / rate, "how": "torch b.copy_(a) of the payload size, median of 5"}
+
+
 def traffic_entry(cfg: str, kernel: str):
     """ncu --set full DRAM bytes per launch of the dominant kernel (profiles/traffic.json)."""
     tf = os.path.join(ROOT, "profiles", "traffic.json")
@@ -653,6 +681,7 @@ class Snapshot:
         achieved = alg / (dom_ms * 1e-3) / 1e9
         traffic, tsrc = traffic_entry(self.cfg, "K1" if dom_name.startswith("pack") else "K2")
         dimg.free()
+        same_size = copy_same_size(torch, dev, S, achieved)
         return {
             "value": value, "ms_max": ms_max, "ms_per_step": ms_max / steps, "verified": n_diff == 0,
             "gpu_launches": sck["n_kernels"] + srs["n_kernels"], "clocks": clk.summary(),
@@ -660,7 +689,7 @@ class Snapshot:
                          "unit": "GB/s", "frac": achieved / hbm_peak, "traffic": traffic, "traffic_source": tsrc,
                          "peak_source": peak_src, "algorithmic_bytes_per_launch": alg,
                          "launches_per_step": {"K1": sck["n_kernels"] / steps, "K2": srs["n_kernels"] / steps},
-                         "pack_ms": pack_ms, "verify_ms": verify_ms},
+                         "pack_ms": pack_ms, "verify_ms": verify_ms, "copy_same_size": same_size},
             "phases": {"checkpoint_ms": ck_ms, "restore_ms": rs_ms, "checkpoint_GBs": S / (ck_ms * 1e-3) / 1e9,
                        "restore_GBs": S / (rs_ms * 1e-3) / 1e9,
                        "pack_GBs_2S": 2 * S / (pack_ms * 1e-3) / 1e9, "verify_GBs_2S": 2 * S / (verify_ms * 1e-3) / 1e9,
