@@ -1,4 +1,4 @@
-# usage: bash tools/exp_sweep2.sh "<libs>" "<configs>" "<ops>" [parity-lib...]
+# usage: bash tools/sessions/exp_sweep2.sh "<libs>" "<configs>" "<ops>" [parity-lib...]
 python -c "import __graft_entry__ as g; g.build()" > /dev/null
 for lib in $1; do
 for cfg in $2; do

@@ -1,7 +1,7 @@
 #!/bin/bash
 # Robustness pass on the final code: compute-sanitizer (memcheck / racecheck / synccheck)
 # x (default dispatch, kernel 3, kernel 4 with the dynamic tail forced), a 400-case GPU
-# fuzz, and the host phase trace of C1. usage: tools/gpu_final_checks.sh <tag>
+# fuzz, and the host phase trace of C1. usage: tools/sessions/gpu_final_checks.sh <tag>
 set -u
 O=gpurun_out/${1:-final}
 mkdir -p $O

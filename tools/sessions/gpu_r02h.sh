@@ -17,5 +17,5 @@ timeout 900 ncu --set full --clock-control none --import-source on --kernel-name
 python tools/ncu_summary.py $R/crc.ncu-rep > $O/crc_summary.txt 2>&1
 timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k regex:"tma_kernel<.int.0" -s 1 -c 1 -o $R/k1 -f python tools/profile_step.py --config C2 --reps 2 > $O/ncu_k1.log 2>&1
 ncu -i $R/k1.ncu-rep --page source --csv --print-source sass > $O/k1_source_sass.csv 2>&1
-bash tools/gpu_final_checks.sh ${1:-r02h}
+bash tools/sessions/gpu_final_checks.sh ${1:-r02h}
 du -sh $O
