@@ -29,4 +29,7 @@ R=/tmp/ncu_$$; mkdir -p $R
 timeout 1200 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k regex:"tma_kernel|meta_crc" -c 6 -o $R/c3 -f python tools/profile_step.py --config C3 --reps 2 > $O/ncu_c3.log 2>&1
 python tools/ncu_summary.py $R/c3.ncu-rep > $O/c3_summary.txt 2>&1
 ncu -i $R/c3.ncu-rep --page details --csv > $O/c3_details.csv 2>&1
+timeout 900 ncu --set full --clock-control none --import-source on --kernel-name-base demangled -k regex:"tma_kernel" -c 4 -o $R/c2 -f python tools/profile_step.py --config C2 --reps 2 > $O/ncu_c2.log 2>&1
+python tools/ncu_summary.py $R/c2.ncu-rep > $O/c2_summary.txt 2>&1
+ncu -i $R/c2.ncu-rep --page raw --csv --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum > $O/c2_dram.csv 2>&1
 du -sh $O
