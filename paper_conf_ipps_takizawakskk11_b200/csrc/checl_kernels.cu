@@ -1011,7 +1011,8 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) sweep_kernel(const LaunchPa
   if (O::kCrc) {
     const TableCopy cp[2] = {{0u, (uint32_t)kTabOff, (uint32_t)kTabWords * 4u},
                              {kPosSm, (uint32_t)kPosOff, (uint32_t)(kPosWords + kUnitWords) * 4u}};
-    load_tables(smem, p.tables, cp, reinterpret_cast<uint64_t*>(smem + kMbarOff));
+    // (waited for after the first unit's loads are issued: the two overlap)
+    load_tables<2, false>(smem, p.tables, cp, reinterpret_cast<uint64_t*>(smem + kMbarOff));
   }
   const uint8_t* tb = smem;
   const uint8_t* pb = smem + kPosSm;
@@ -1054,6 +1055,7 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) sweep_kernel(const LaunchPa
   uint64_t u = (uint64_t)blockIdx.x * kWarpsPerCta + warp;
   Unit cur = get_unit(u);
   if (cur.on) load_round(v, cur.src, cur.len, cur.mode, cur.r, lane_off);
+  if (O::kCrc) wait_tables(reinterpret_cast<uint64_t*>(smem + kMbarOff));
   for (; u < nunits; u += nw) {
     const Unit nxt = get_unit(u + nw);
     if (cur.on) store_round<kOp>(v, cur.dst, cur.len, cur.r, lane_off, tile_w);
