@@ -507,8 +507,12 @@ def copy_same_size(torch, dev: int, S: int, achieved: float) -> dict:
     n = min(S, (free - (1 << 30)) // 2 // (1 << 20) * (1 << 20))  # C4 in restart mode: what fits
     if n < (256 << 20):
         return {"GBs": None, "reason": f"{free} B of free HBM"}
-    a = torch.empty(n, dtype=torch.uint8, device=dev)
-    b = torch.empty_like(a)
+    try:
+        a = torch.empty(n, dtype=torch.uint8, device=dev)
+        b = torch.empty_like(a)
+    except torch.cuda.OutOfMemoryError as e:  # context only: never fail the run for it
+        torch.cuda.empty_cache()
+        return {"GBs": None, "reason": f"allocation failed: {str(e)[:80]}"}
     a.fill_(1)
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     ts = []
