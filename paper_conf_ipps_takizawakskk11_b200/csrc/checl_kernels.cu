@@ -339,8 +339,10 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
   extern __shared__ __align__(128) uint8_t smem[];
   if (O::kCrc) {
     const TableCopy cp[1] = {{0u, (uint32_t)kTabOff, (uint32_t)kSnapTabWords * 4u}};
-    load_tables(smem, p.tables, cp, reinterpret_cast<uint64_t*>(smem + kMbarOff));
+    // (waited for before the first CRC: the first chunk's loads overlap the copy)
+    load_tables<1, false>(smem, p.tables, cp, reinterpret_cast<uint64_t*>(smem + kMbarOff));
   }
+  bool tables_ready = false;
   const uint8_t* tb = smem + kTabOff * 4;
   const uint8_t* hb = smem + kHornerOff * 4;
   const uint32_t* ftab = reinterpret_cast<const uint32_t*>(smem + kFoldOff * 4);
@@ -372,6 +374,10 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
       store_round<kOp>(v, dst, len, r, lane_off, tile_w);
       __syncwarp();
       if (r + kPrefetch < nrounds) load_round(v, src, len, mode, r + kPrefetch, lane_off);
+      if (O::kCrc && !tables_ready) {
+        wait_tables(reinterpret_cast<uint64_t*>(smem + kMbarOff));
+        tables_ready = true;
+      }
       if (O::kCrc) {
         // lane l: segment 32r + l; Horner step over the rest of the round first
         if (r > 0) ch = horner_mul(ch, hb, l4);
@@ -409,6 +415,8 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) snapshot_kernel(const Launc
     }
     finish_chunk<kOp>(p, c, src, dst, len, pad, nrounds, f, lane);
   }
+  // no warp exits while the table copy into its CTA's shared memory is in flight
+  if (O::kCrc && !tables_ready) wait_tables(reinterpret_cast<uint64_t*>(smem + kMbarOff));
   publish_status<kOp>(p);
 }
 
