@@ -1422,6 +1422,14 @@ void timed_launch(DevState& ds, KernelTimer& kt, int op, const LaunchParams& p0,
                  op, kernel, st.size(), ms * 1e3, q(st, 0.5), q(st, 1.0), q(tb, 0.5), q(tb, 1.0), q(en, 0.0), q(en, 0.1),
                  q(en, 0.5), q(en, 0.9), q(en, 1.0));
     const char* wt = std::getenv("CHECL_WARP_TRACE");
+    if (wt && std::atoi(wt) == 3) {  // raw, one line per warp: cta warp slot3 start slot1 slot2 (us)
+      for (uint64_t w = 0; w < n_tr / 4; ++w) {
+        if (!h[4 * w]) continue;
+        std::fprintf(stderr, "[checl] w %llu %llu %llu %llu %.2f %.2f %.2f\n", (unsigned long long)(w / kWarpsPerCta),
+                     (unsigned long long)(w % kWarpsPerCta), h[4 * w + 3] & 0xFFFFFFFFull, h[4 * w + 3] >> 32,
+                     (h[4 * w] - t0) * 1e-3, h[4 * w + 1] ? (h[4 * w + 1] - t0) * 1e-3 : -1.0, (h[4 * w + 2] - t0) * 1e-3);
+      }
+    }
     if (wt && std::atoi(wt) == 2) {  // raw end times, one line per CTA
       for (int c = 0; c < ds.n_sms; ++c) {
         std::string line = "[checl] cta " + std::to_string(c) + " sm " + std::to_string(h[4 * (uint64_t)c * kWarpsPerCta + 3]);
