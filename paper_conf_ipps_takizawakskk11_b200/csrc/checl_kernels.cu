@@ -835,6 +835,9 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
   }
   uint64_t ng = 0, nge = 0, nlo = 0;  // the next stretch (dynamic block), once fetched
   int t = 0;                          // tile of the round being consumed
+#ifdef CHECL_TRACE_LOOPEND  // experiment: slot 2 = the warp's last round done, slot 3 = smid | rounds << 32
+  unsigned long long n_done = 0;
+#endif
   Part cur{};
   if (have) {
     cur = open_part(c, p.round_base[c], p.desc[c], g, g_end);
@@ -932,6 +935,9 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
       fence_proxy_async();  // this round's shared reads before the next bulk copy into the tile
       __syncwarp();
       t ^= 1;
+#ifdef CHECL_TRACE_LOOPEND
+      ++n_done;
+#endif
     }
     // chain c stepped every row it holds by x^(1024*kColChains), i.e. c rows too far:
     // h = XOR_c ch[c] * x^(-1024 c) (Horner), then the lanes as before
@@ -970,16 +976,23 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
     }
     cur = nxt;
   }
+#ifdef CHECL_TRACE_LOOPEND
+  warp_trace(p, 2, gtimer());
+#endif
   if (!tables_ready) wait_tables(mbars + kWarpsPerCta * kTmaTiles);
   if (lane == 0) bulk_wait_all();  // the bulk stores have landed before the kernel ends
   release_work(p);
   if constexpr (kMc) cluster_sync();  // neither CTA exits while a multicast it issued is in flight
   warp_trace(p, 0, t_start);
-  warp_trace(p, 2, gtimer());
   {
     unsigned smid;
     asm("mov.u32 %0, %%smid;" : "=r"(smid));
+#ifdef CHECL_TRACE_LOOPEND
+    warp_trace(p, 3, smid | (n_done << 32));
+#else
+    warp_trace(p, 2, gtimer());
     warp_trace(p, 3, smid);
+#endif
   }
   publish_status<kOp>(p);
 }
