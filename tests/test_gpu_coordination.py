@@ -162,3 +162,58 @@ def test_coordinated_checkpoint_real_images_commit_and_abort():
         for k in ("host_commit", "into_commit", "device_commit", "host_abort", "device_abort", "into_abort",
                   "pair"):
             assert res.get(k), (rank, k, res)
+
+
+def _nccl_worker(port, q):
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from oracle import oracle as O
+    from paper_conf_ipps_takizawakskk11_b200 import checl
+    from paper_conf_ipps_takizawakskk11_b200.coordination import agree, coordinated, coordinated_checkpoint
+    from tests.gpu_util import make_set, oracle_entries
+
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    torch.cuda.set_device(0)
+    dist.init_process_group("nccl", rank=0, world_size=1, device_id=torch.device("cuda", 0))
+    res = {}
+    try:
+        res["backend"] = dist.get_backend()
+        # the status vector on the GPU through NCCL: world 1 returns the inputs
+        res["agree"] = agree(False, 7, 12345, (3 << 48) | 77, device=0) == (0, 7, 12345, True, (3 << 48) | 77)
+        ctx = checl.Context()
+        ds = make_set(ctx, [1 << 20, 65537, 0, 4097], seed=9)
+        for on_device in (False, True):
+            snap = coordinated_checkpoint(ctx, 0, epoch=5, on_device=on_device)
+            want = O.checkpoint(oracle_entries(ds), device=0, epoch=5)
+            got = snap.image.to_host().view() if on_device else snap.image.view()
+            res[f"commit_{on_device}"] = snap.committed and np.array_equal(got, want)
+            snap.image.free()
+
+        def failing():
+            raise RuntimeError("local snapshot failed")
+
+        snap = coordinated(failing, epoch=6, device=0)
+        res["abort"] = (not snap.committed) and snap.image is None and snap.failures == 1
+        ctx.close()
+    except Exception as e:
+        res["error"] = repr(e)
+    q.put(res)
+    dist.destroy_process_group()
+
+
+def test_status_allreduce_over_nccl_world1():
+    """The coordination all-reduce as it runs on a GPU box: NCCL backend, the status
+    vector in HBM (one rank: NCCL refuses two ranks on one GPU). Commit with a host
+    and an HBM image equal to the oracle's; a failed local snapshot aborts."""
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    p = ctx.Process(target=_nccl_worker, args=(_free_port(), q))
+    p.start()
+    res = q.get(timeout=600)
+    p.join(timeout=120)
+    assert "error" not in res, res
+    assert res["backend"] == "nccl"
+    for k in ("agree", "commit_False", "commit_True", "abort"):
+        assert res.get(k), (k, res)
