@@ -984,13 +984,15 @@ __global__ void __launch_bounds__(kThreadsPerCta, 1) tma_kernel(const LaunchPara
   release_work(p);
   if constexpr (kMc) cluster_sync();  // neither CTA exits while a multicast it issued is in flight
   warp_trace(p, 0, t_start);
+#ifndef CHECL_TRACE_LOOPEND
+  warp_trace(p, 2, gtimer());
+#endif
   {
     unsigned smid;
     asm("mov.u32 %0, %%smid;" : "=r"(smid));
 #ifdef CHECL_TRACE_LOOPEND
     warp_trace(p, 3, smid | (n_done << 32));
 #else
-    warp_trace(p, 2, gtimer());
     warp_trace(p, 3, smid);
 #endif
   }
